@@ -1,0 +1,343 @@
+#!/usr/bin/env python
+"""bench.py — input tuples/s of a fused RA chain on 1..8 B200 (BASELINE.json metric).
+
+Default workload (N=1): configs[1] = C2, SELECT -> PROJECT -> SELECT over 2^29
+4-column int32 tuples per GPU (weak scaling: rank r owns rows [r*2^29, (r+1)*2^29)
+of a 2^29*N-row relation, no data-path collective).  One step = one
+rw_plan_execute of the whole fused chain over the rank's relation.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c1|c3|c4|c5]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+    python bench.py --impl reference ...     # the oracle (CPU) as the reference arm
+
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads  # noqa: E402
+
+W = {"i32": 4, "u32": 4, "i64": 8, "u64": 8, "u8": 1}
+
+CONFIGS = {
+    "c1": dict(name="C1: SELECT->SELECT (50%, 50%) over 2^20 (u32 key, u32 val)", rows=workloads.C1_ROWS),
+    "c2": dict(name="C2: SELECT->PROJECT->SELECT over 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
+    "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
+    "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="rw", choices=["rw", "reference"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--rows", type=int, default=0, help="override rows per GPU (testing)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-unfused", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-rows", type=int, default=0)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def spec_and_inputs(cfg: str, rows: int, start: int, device):
+    if cfg == "c1":
+        return workloads.c1_spec(), workloads.c1_inputs(rows, start, device)
+    if cfg == "c2":
+        return workloads.c2_spec(), workloads.c2_inputs(rows, start, device)
+    if cfg == "c3":
+        return workloads.c3_spec(), workloads.c3_inputs(rows, device=device)
+    if cfg == "c4":
+        return workloads.c4_spec(), workloads.c4_inputs(rows, start, device)
+    raise ValueError(cfg)
+
+
+def spec_rows(spec, ins):
+    return {k: int(v[0].numel()) for k, v in ins.items()}
+
+
+class ClockSampler:
+    """NVML clocks / throttle reasons sampled every 5 ms during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting", 0x10: "sync_boost"}
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.ok = False
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def result(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def measured_peak():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy kernel)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(cfg: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu capture, else None."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(p) as f:
+            j = json.load(f)
+        return j.get(cfg)
+    except Exception:
+        return None
+
+
+def cpu_oracle_sample(cfg: str, rows: int, sample_rows: int):
+    """Time the oracle (single thread) on a bounded prefix sample of the same workload."""
+    import oracle
+    from tests.planspec import run_oracle
+    m = min(rows, sample_rows)
+    if cfg == "c3":
+        spec, ins = spec_and_inputs(cfg, m, 0, "cpu")
+    else:
+        spec, ins = spec_and_inputs(cfg, m, 0, "cpu")
+    rels = {}
+    import numpy as np
+    npt = {"i32": np.int32, "u32": np.uint32, "i64": np.int64, "u64": np.uint64, "u8": np.uint8}
+    for name, inp in spec["inputs"].items():
+        rels[name] = oracle.Relation(inp["types"], [c.numpy().view(npt[t]) for c, t in zip(ins[name], inp["types"])])
+    t0 = time.perf_counter()
+    oracle.evaluate(spec, rels)
+    dt = time.perf_counter() - t0
+    n_in = sum(r.n for r in rels.values())
+    return n_in / dt, dt, n_in
+
+
+def run_reference(args):
+    rank, world, local = dist_env()
+    if rank != 0:
+        return 0
+    cfg = args.config
+    rows = args.rows or CONFIGS[cfg]["rows"]
+    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23}[cfg]
+    import oracle
+    oracle.build()
+    vals = []
+    for i in range(args.warmup + args.steps):
+        v, dt, n_in = cpu_oracle_sample(cfg, rows, sample)
+        if i >= args.warmup:
+            vals.append((v, dt, n_in))
+    value = statistics.median(v for v, _, _ in vals)
+    ms = statistics.median(dt for _, dt, _ in vals) * 1e3
+    line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic (rwgen seeded generators)", "impl": "reference",
+            "config": {"workload": CONFIGS[cfg]["name"], "sample_rows": vals[0][2],
+                       "note": "reference arm = the CPU oracle (single thread) on a bounded prefix sample"},
+            "cpu_baseline": {"value": value, "unit": "tuples/s", "cores": 1, "kind": "oracle",
+                             "sample": f"first {vals[0][2]} input tuples of {cfg}"},
+            "e2e": {"value": value, "unit": "tuples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = f"cuda:{local}"
+    pg = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device(dev))
+        pg = dist
+    from paper_conf_micro_wudcy12_b200 import rw
+    from tests.planspec import build_gpu_plan
+
+    cfg = args.config
+    rows = args.rows or CONFIGS[cfg]["rows"]
+    spec, ins = spec_and_inputs(cfg, rows, rank * rows, dev)
+    nrows = spec_rows(spec, ins)
+    n_in = sum(nrows.values())
+    in_bytes = workloads.input_bytes(spec, nrows)
+    stream = torch.cuda.current_stream()
+
+    def make(fuse):
+        plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse)
+        out_types = plan.node_schema(ids[spec["out"]])
+        cap = {"c4": 6}.get(cfg, max(nrows.values()))
+        if cfg == "c3":
+            cap = 400_000_000 if rows == workloads.C3_ROWS else 8 * rows + 1024
+        dt = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
+        outs = [torch.empty(cap, dtype=dt[t], device=dev) for t in out_types]
+        return plan, ids, outs, cap, out_types
+
+    inputs = [(nrows[k], ins[k]) for k in spec["inputs"]]
+    n_dev = torch.zeros(1, dtype=torch.int64, device=dev)
+
+    def timed(plan, ids, outs, cap, steps, warmup):
+        for _ in range(warmup):
+            plan.execute(inputs, ids[spec["out"]], outs, cap, n_dev=n_dev)
+        torch.cuda.synchronize()
+        if pg:
+            pg.barrier()
+        torch.cuda.synchronize()
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        launches = 0
+        sampler = ClockSampler(local)
+        with sampler:
+            evs[0].record(stream)
+            for i in range(steps):
+                plan.execute(inputs, ids[spec["out"]], outs, cap, n_dev=n_dev)
+                launches += plan.last_launches()
+                evs[i + 1].record(stream)
+            torch.cuda.synchronize()
+        per = [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
+        total_ms = evs[0].elapsed_time(evs[-1])
+        if pg:
+            t = torch.tensor([total_ms], device=dev)
+            pg.all_reduce(t, op=pg.ReduceOp.MAX)
+            total_ms = float(t.item())
+        return total_ms, per, launches, sampler.result()
+
+    plan, ids, outs, cap, out_types = make(True)
+    total_ms, per, launches, clocks = timed(plan, ids, outs, cap, args.steps, args.warmup)
+    n_out = int(n_dev.item())
+    ms_step = total_ms / args.steps
+    value = n_in * world / (total_ms / 1e3 / args.steps)
+
+    # roofline of the dominant kernel (the fused chain kernel is the whole step for C1/C2;
+    # for C4 the finalize kernel is ~µs; for C3 the expansion kernel dominates)
+    out_w = sum(W[t] for t in out_types)
+    alg_bytes = in_bytes + n_out * out_w
+    peak, peak_src = measured_peak()
+    kern_ms = statistics.mean(per)
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": ncu_traffic(cfg), "kernel": "k_scan_chain" if cfg != "c3" else "join (k_join_runs+k_join_expand)",
+                "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+                "note": "achieved = (input bytes + compacted output bytes) / CUDA-event time per step"}
+
+    line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else "i32",
+            "data": "synthetic (rwgen seeded SplitMix64 generators, generated on device)",
+            "config": {"workload": CONFIGS[cfg]["name"], "rows_per_gpu": nrows, "output_rows_per_gpu": n_out,
+                       "parallelism": f"row-shard x{world}", "l2": "inputs larger than L2 (no flush needed)",
+                       "fused": True},
+            "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
+
+    if not args.no_unfused and cfg in ("c1", "c2", "c4", "c3"):
+        del outs
+        torch.cuda.empty_cache()
+        uplan, uids, uouts, ucap, _ = make(False)
+        ut, uper, ul, _ = timed(uplan, uids, uouts, ucap, max(3, args.steps // 4), 2)
+        uv = n_in * world / (ut / 1e3 / max(3, args.steps // 4))
+        line["unfused"] = {"value": uv, "ms_per_step": ut / max(3, args.steps // 4), "gpu_launches_per_step":
+                           ul / max(3, args.steps // 4), "speedup_fused_vs_unfused": value / uv,
+                           "roofline_frac_same_numerator": alg_bytes / (ut / max(3, args.steps // 4) / 1e3) / 1e9 / peak}
+        del uouts, uplan
+        torch.cuda.empty_cache()
+
+    if not args.no_e2e and cfg in ("c1", "c2", "c4"):
+        # end to end through rw_plan_execute_host: pinned host inputs copied H2D and the
+        # result copied D2H inside the timed region
+        host_in = [(n, [c.cpu().pin_memory() for c in cols]) for n, cols in inputs]
+        eplan, eids, _, ecap, etypes = None, None, None, None, None
+        eplan, eids = build_gpu_plan(spec, device=local, stream=stream)
+        etypes = eplan.node_schema(eids[spec["out"]])
+        ecap = {"c4": 6}.get(cfg, max(nrows.values()))
+        dtn = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
+        host_out = [torch.empty(ecap, dtype=dtn[t]).pin_memory() for t in etypes]
+        esteps = max(2, min(args.steps, 5))
+        for _ in range(1):
+            eplan.execute_host(host_in, eids[spec["out"]], host_out, ecap)
+        if pg:
+            pg.barrier()
+        t0 = time.perf_counter()
+        n_e = 0
+        for _ in range(esteps):
+            n_e = eplan.execute_host(host_in, eids[spec["out"]], host_out, ecap)
+        et = (time.perf_counter() - t0) / esteps
+        if pg:
+            t = torch.tensor([et], device=dev)
+            pg.all_reduce(t, op=pg.ReduceOp.MAX)
+            et = float(t.item())
+        line["e2e"] = {"value": n_in * world / et, "unit": "tuples/s", "h2d_bytes_per_step": in_bytes,
+                       "d2h_bytes_per_step": n_e * sum(W[t] for t in etypes), "ms_per_step": et * 1e3,
+                       "api": "rw_plan_execute_host (pinned host buffers)"}
+        del host_in, host_out
+
+    if rank == 0 and not args.no_cpu:
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24}[cfg]
+        v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
+        line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
+                                "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if pg:
+        pg.barrier()
+        pg.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,122 @@
+// internal.h — structures shared by the plan builder (host C++) and the sm_100a
+// kernels.  Not part of the public ABI (that is include/rw.h).
+//
+// A fused group is lowered to a ChainProg: a small register-free "micro-op"
+// program over SLOTS.  A slot is one column of the current tile held in shared
+// memory (input slots are filled by TMA bulk copies or by the join expansion;
+// computed slots hold PROJECT/arithmetic results).  The paper passes
+// thread-dependent intermediates in registers (§4.3.1); here the whole
+// tile is resident in smem and the per-row `match` bit stays in a register,
+// which keeps the program interpretable without code generation (DESIGN.md
+// "What differs from the paper").
+#pragma once
+#include <stdint.h>
+
+#if !defined(__CUDACC__) && !defined(__host__)
+#define __host__
+#define __device__
+#endif
+
+namespace rw {
+
+constexpr int kMaxSlots = 24;
+constexpr int kMaxOps = 48;
+constexpr int kMaxOut = 32;
+constexpr int kMaxGroupCols = 8;
+constexpr int kMaxAggs = 16;
+constexpr int kThreads = 256;        // threads per CTA for every chain kernel
+constexpr int kScanItems = 8;        // rows per thread per tile in the scan kernel (T = 2048)
+constexpr int kJoinItems = 9;        // outputs per thread per tile in the join expansion (T = 2304,
+                                     // odd stride -> conflict-free thread-contiguous smem writes)
+constexpr int kMaxAggSlots = 4096;   // D * (nagg + 1) upper bound for the agg terminal
+
+enum Type : uint8_t { T_I32 = 0, T_U32 = 1, T_I64 = 2, T_U64 = 3, T_U8 = 4 };
+enum Cmp : uint8_t { C_LT = 0, C_LE = 1, C_GT = 2, C_GE = 3, C_EQ = 4, C_NE = 5 };
+enum OpKind : uint8_t { K_PRED = 0, K_EXPR = 1 };
+enum ExprOp : uint8_t { E_COPY = 0, E_CONST = 1, E_ADD = 2, E_SUB = 3, E_MUL = 4, E_DIVC = 5, E_RSUB = 6 };
+
+__host__ __device__ inline int type_width(int t) { return t == T_U8 ? 1 : (t == T_I64 || t == T_U64) ? 8 : 4; }
+__host__ __device__ inline bool type_signed(int t) { return t == T_I32 || t == T_I64; }
+
+struct SlotDesc {
+    uint8_t type;
+    uint8_t is_input;   // 1: lives in the (multi-buffered) stage; 0: lives in scratch
+    uint16_t pad;
+    uint32_t off;       // byte offset of the slot column inside stage / scratch
+};
+
+struct DevOp {
+    uint8_t kind;       // K_PRED / K_EXPR
+    uint8_t op;         // Cmp or ExprOp
+    uint8_t type;       // compare type (PRED) or result type (EXPR)
+    uint8_t b_is_slot;  // PRED: rhs is a slot; EXPR: operand b is a slot (else constant k)
+    int16_t dst;        // EXPR destination slot
+    int16_t a;          // operand a slot
+    int16_t b;          // operand b slot
+    int16_t pad;
+    int64_t k;          // constant (rhs / operand b / divisor), already wrapped to `type`
+};
+
+struct ChainProg {
+    int32_t nslots;
+    int32_t nin;                        // slots [0, nin) are input slots
+    int32_t nops;
+    int32_t nout;
+    SlotDesc slot[kMaxSlots];
+    const void *in_ptr[kMaxSlots];      // scan kernel: global column base of each input slot
+    DevOp ops[kMaxOps];
+    int16_t out_slot[kMaxOut];
+    void *out_ptr[kMaxOut];
+    int64_t out_capacity;
+    // aggregate terminal (is_agg): group code g = sum code_c * stride_c
+    int32_t is_agg;
+    int32_t ngc;
+    int16_t gslot[kMaxGroupCols];
+    int32_t gdomain[kMaxGroupCols];
+    int32_t D;                          // product of domains
+    int32_t nagg;                       // number of SUM accumulators (count is implicit, index 0)
+    int16_t agg_slot[kMaxAggs];
+    uint8_t agg_unsigned[kMaxAggs];     // 1: u64 sum (unsigned partials)
+    int64_t flush_rows;                 // rows a thread may add before its int64 partials can overflow
+    uint32_t stage_bytes;               // bytes of one stage (all input slots, aligned)
+    uint32_t scratch_bytes;             // bytes of scratch (computed slots)
+};
+
+// Launch-time scalars for the scan / join-expand kernels.
+struct TileLaunch {
+    int64_t n;                 // rows (scan) or join outputs (expand), if n_ptr == nullptr
+    const int64_t *n_ptr;      // device row count written by an earlier kernel (else nullptr)
+    int32_t stages;
+    int32_t use_tma;           // input slots may be bulk-copied (16B-aligned bases)
+    uint32_t epoch;            // look-back epoch tag (1..65535)
+    uint64_t *status;          // look-back status words, >= ntiles
+    uint32_t *ctrs;            // [0] tile counter, [1] done counter (reset by the last CTA)
+    int64_t *n_dev;            // output row count
+    unsigned long long *agg_acc;   // global 128-bit accumulators: D * (nagg+1) * 2 u64
+    int32_t *err;              // [0] domain errors
+};
+
+// Join expansion inputs (run records written by k_join_runs).
+struct JoinRuns {
+    const uint32_t *s;         // first L row of the run
+    const uint32_t *lenL;
+    const uint32_t *lo;        // first matching R row
+    const uint32_t *lenR;
+    const uint64_t *off;       // exclusive output offset of the run
+    int64_t nruns;
+    int64_t total;             // total join candidates
+    // gather sources: output column j of the join = L col (j < nl) else R col (nkey + j - nl)
+    int32_t ncols;             // number of join output columns that are live (gathered)
+    const void *src[kMaxSlots];
+    uint8_t from_right[kMaxSlots];
+    int16_t dst_slot[kMaxSlots];
+};
+
+struct JoinKeys {
+    const void *lkey;
+    const void *rkey;
+    int32_t key_type;
+    int64_t nl, nr;
+};
+
+}  // namespace rw

@@ -1,0 +1,692 @@
+// kernels.cu — the sm_100a kernels of the fused relational-algebra hot path.
+//
+//   k_scan_chain<ITEMS, AGG>  fused SELECT / PROJECT / arithmetic chain over one
+//                             input relation, terminal =
+//                             compacted store or group-by aggregate (a9).
+//   k_agg_finalize            128-bit accumulators -> output relation (groups with
+//                             count > 0, ascending code).
+//   k_join_runs<K>            merge-path partitioned sorted-key JOIN, phase 1:
+//                             matched key runs + output offsets (a7).
+//   k_tile_runs               first run of every expansion tile.
+//   k_join_expand             JOIN phase 2: output-balanced expansion fused with
+//                             the downstream SELECT / PROJECT chain (a8).
+//
+// Every persistent kernel claims tiles with a global atomic counter (so the
+// decoupled look-back always has forward progress) and the last CTA to leave
+// resets the counter for the next launch.
+#include <type_traits>
+#include "chain.cuh"
+#include "kernels.h"
+
+namespace rw {
+
+static __host__ __device__ inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+template <int ITEMS>
+struct CtlSmem {
+    uint64_t mbar[kMaxStages];
+    int64_t tile_id[kMaxStages];
+    EmitSmem<ITEMS> es;
+};
+
+__device__ inline void cta_exit_reset(uint32_t *ctrs)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&ctrs[1], 1u) == gridDim.x - 1) {
+            ctrs[0] = 0;
+            ctrs[1] = 0;
+            __threadfence();
+        }
+    }
+}
+
+// ===========================================================================
+// Fused scan chain.  Tiles of T = 256 * ITEMS rows are staged into smem by TMA
+// bulk copies (one cp.async.bulk per live column, completion on an mbarrier),
+// L.stages tiles in flight per CTA; thread 0 is the producer and refills a stage
+// as soon as every thread has finished with it.
+// ===========================================================================
+template <int ITEMS, bool AGG>
+__global__ void __launch_bounds__(kThreads) k_scan_chain(const __grid_constant__ ChainProg P,
+                                                         const __grid_constant__ TileLaunch L)
+{
+    constexpr int T = kThreads * ITEMS;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    CtlSmem<ITEMS> *ctl = (CtlSmem<ITEMS> *)smem_raw;
+    char *stages = (char *)smem_raw + align_up(sizeof(CtlSmem<ITEMS>), 128);
+    char *scratch = stages + (size_t)L.stages * P.stage_bytes;
+    unsigned long long *part = (unsigned long long *)(scratch + P.scratch_bytes);
+    const int NA = P.nagg + 1;
+    unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * kThreads : 0);
+    const int tid = threadIdx.x;
+    const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
+    const int64_t ntiles = (n + T - 1) / T;
+
+    if (tid == 0) {
+        for (int s = 0; s < L.stages; s++)
+            mbar_init(&ctl->mbar[s], 1);
+        fence_mbar_init();
+    }
+    if (AGG) {
+        for (int q = tid; q < P.D * NA * kThreads; q += kThreads)
+            part[q] = 0;
+        for (int q = tid; q < P.D * NA * 2; q += kThreads)
+            cta_acc[q] = 0;
+    }
+    __syncthreads();
+
+    uint32_t tx_bytes = 0;
+    for (int i = 0; i < P.nin; i++)
+        tx_bytes += (uint32_t)T * type_width(P.slot[i].type);
+    const uint64_t policy = policy_evict_first();
+
+    auto refill = [&](int s) {
+        int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
+        ctl->tile_id[s] = t;
+        if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
+            char *st = stages + (size_t)s * P.stage_bytes;
+            fence_proxy_async_smem();
+            mbar_arrive_expect_tx(&ctl->mbar[s], tx_bytes);
+            for (int i = 0; i < P.nin; i++) {
+                const int w = type_width(P.slot[i].type);
+                bulk_g2s(st + P.slot[i].off, (const char *)P.in_ptr[i] + (size_t)t * T * w, (uint32_t)T * w,
+                         &ctl->mbar[s], policy);
+            }
+        } else {
+            mbar_arrive(&ctl->mbar[s]);
+        }
+    };
+
+    if (tid == 0)
+        for (int s = 0; s < L.stages; s++)
+            refill(s);
+
+    int64_t since_flush = 0;
+    for (int64_t it = 0;; ++it) {
+        const int s = (int)(it % L.stages);
+        const uint32_t parity = (uint32_t)((it / L.stages) & 1);
+        mbar_wait(&ctl->mbar[s], parity);
+        const int64_t t = ctl->tile_id[s];
+        if (t >= ntiles)
+            break;
+        char *st = stages + (size_t)s * P.stage_bytes;
+        const int64_t row0 = t * T;
+        const int rows = (int)min((int64_t)T, n - row0);
+        if (!(L.use_tma && rows == T)) {
+            // ragged last tile or unaligned column bases: plain coalesced loads
+            for (int i = 0; i < P.nin; i++) {
+                const int w = type_width(P.slot[i].type);
+                char *dst = st + P.slot[i].off;
+                const char *src = (const char *)P.in_ptr[i] + (size_t)row0 * w;
+                if (w == 4) {
+                    for (int r = tid; r < rows; r += kThreads)
+                        ((uint32_t *)dst)[r] = ((const uint32_t *)src)[r];
+                } else if (w == 8) {
+                    for (int r = tid; r < rows; r += kThreads)
+                        ((uint64_t *)dst)[r] = ((const uint64_t *)src)[r];
+                } else {
+                    for (int r = tid; r < rows; r += kThreads)
+                        dst[r] = src[r];
+                }
+            }
+            __syncthreads();
+        }
+        uint32_t mask = 0;
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++)
+            if (k * kThreads + tid < rows)
+                mask |= 1u << k;
+        mask = run_ops<ITEMS>(P, st, scratch, mask);
+        if (AGG)
+            agg_tile<ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
+        else
+            emit_tile<ITEMS>(P, st, scratch, mask, t, ntiles, L, &ctl->es);
+        __syncthreads();
+        if (tid == 0)
+            refill(s);
+    }
+
+    if (AGG) {
+        agg_flush(P, part, cta_acc);
+        __syncthreads();
+        for (int q = tid; q < P.D * NA; q += kThreads) {
+            unsigned long long lo = cta_acc[2 * q], hi = cta_acc[2 * q + 1];
+            if (lo | hi)
+                atomic_add128(&L.agg_acc[2 * q], &L.agg_acc[2 * q + 1], lo, hi);
+        }
+    } else if (ntiles == 0 && blockIdx.x == 0 && tid == 0) {
+        *L.n_dev = 0;
+    }
+    cta_exit_reset(L.ctrs);
+}
+
+// ===========================================================================
+// Aggregate finalisation: one CTA scans the D groups, emits those with count>0
+// in ascending code order (reading A12), and zeroes the accumulators.
+// ===========================================================================
+__global__ void __launch_bounds__(kThreads) k_agg_finalize(const __grid_constant__ AggFinal F)
+{
+    __shared__ uint32_t wsum[kWarps];
+    __shared__ int64_t base;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0)
+        base = 0;
+    __syncthreads();
+    for (int g0 = 0; g0 < F.D; g0 += kThreads) {
+        const int g = g0 + tid;
+        unsigned long long cnt = 0;
+        if (g < F.D)
+            cnt = F.acc[2 * ((size_t)g * F.NA)];
+        const bool live = cnt > 0;
+        uint32_t b = __ballot_sync(0xffffffffu, live);
+        if (lane == 0)
+            wsum[warp] = __popc(b);
+        __syncthreads();
+        uint32_t before = 0, total = 0;
+        for (int w = 0; w < kWarps; w++) {
+            if (w < warp)
+                before += wsum[w];
+            total += wsum[w];
+        }
+        const int64_t pos = base + before + __popc(b & lanemask_lt());
+        if (live && pos < F.capacity) {
+            int oc = 0;
+            int rem = g;
+            int codes[kMaxGroupCols];
+            for (int c = F.ngc - 1; c >= 0; c--) {
+                codes[c] = rem % F.gdomain[c];
+                rem /= F.gdomain[c];
+            }
+            for (int c = 0; c < F.ngc; c++, oc++) {
+                switch (type_width(F.gtype[c])) {
+                case 1: ((uint8_t *)F.out[oc])[pos] = (uint8_t)codes[c]; break;
+                case 4: ((uint32_t *)F.out[oc])[pos] = (uint32_t)codes[c]; break;
+                default: ((uint64_t *)F.out[oc])[pos] = (uint64_t)codes[c]; break;
+                }
+            }
+            for (int q = 0; q < F.nreq; q++) {
+                const size_t a = (size_t)g * F.NA + F.req_acc[q];
+                if (F.req_is_sum[q]) {
+                    ((unsigned long long *)F.out[oc++])[pos] = F.acc[2 * a];
+                    ((unsigned long long *)F.out[oc++])[pos] = F.acc[2 * a + 1];
+                } else {
+                    ((unsigned long long *)F.out[oc++])[pos] = F.acc[2 * a];
+                }
+            }
+        }
+        __syncthreads();
+        if (g < F.D)
+            for (int a = 0; a < F.NA; a++) {
+                F.acc_w[2 * ((size_t)g * F.NA + a)] = 0;
+                F.acc_w[2 * ((size_t)g * F.NA + a) + 1] = 0;
+            }
+        if (tid == 0)
+            base += total;
+        __syncthreads();
+    }
+    if (tid == 0) {
+        *F.n_dev = base;
+        F.err[1] = F.err[0];
+        F.err[0] = 0;
+    }
+}
+
+// ===========================================================================
+// JOIN phase 1 — merge-path partitions of the merged key sequence (L before R on
+// ties, §4.3.2 binary-search partitioning).  For every L element that
+// starts a key run inside the partition: R range [lo, hi) by binary search in
+// the partition's smem copy of R (lo always lies inside it), galloping past the
+// partition end for long runs; L run length likewise.  Runs with a match are
+// compacted (ballot + look-back) into run records with their output offsets.
+// ===========================================================================
+constexpr int kRunItems = 8;
+constexpr int kRunT = kThreads * kRunItems;
+
+template <typename K>
+__device__ __forceinline__ int64_t merge_path(const K *L, int64_t nl, const K *R, int64_t nr, int64_t d)
+{
+    int64_t lo = d > nr ? d - nr : 0;
+    int64_t hi = d < nl ? d : nl;
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if (L[mid] <= R[d - mid - 1])
+            lo = mid + 1;
+        else
+            hi = mid;
+    }
+    return lo;
+}
+
+template <typename K>
+__device__ __forceinline__ int lower_bound_smem(const K *a, int n, K key)
+{
+    int lo = 0, hi = n;
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (a[mid] < key) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+template <typename K>
+__device__ __forceinline__ int upper_bound_smem(const K *a, int n, K key)
+{
+    int lo = 0, hi = n;
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (a[mid] <= key) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// first index >= start with A[idx] > key (A[start..] sorted, A[start-1] <= key)
+template <typename K>
+__device__ int64_t gallop_upper(const K *A, int64_t start, int64_t n, K key)
+{
+    int64_t lo = start, hi = n, step = 1;
+    while (true) {
+        int64_t probe = lo + step - 1;
+        if (probe >= n) { hi = n; break; }
+        if (A[probe] > key) { hi = probe; break; }
+        lo = probe + 1;
+        step <<= 1;
+    }
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if (A[mid] <= key) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// exclusive block scan of per-(item, thread) 64-bit values in (k, warp, lane) order
+template <int ITEMS>
+__device__ inline void block_scan_u64(uint64_t (&v)[ITEMS], uint64_t *wtot /* ITEMS*kWarps */, uint64_t &total)
+{
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        uint64_t x = v[k], inc = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o)
+                inc += y;
+        }
+        v[k] = inc - x;   // exclusive within the warp
+        if (lane == 31)
+            wtot[k * kWarps + warp] = inc;
+    }
+    __syncthreads();
+    if (warp == 0) {
+        constexpr int NV = ITEMS * kWarps;
+        constexpr int PER = (NV + 31) / 32;
+        uint64_t a[PER];
+        uint64_t s = 0;
+#pragma unroll
+        for (int q = 0; q < PER; q++) {
+            int idx = lane * PER + q;
+            a[q] = idx < NV ? wtot[idx] : 0;
+            s += a[q];
+        }
+        uint64_t inc = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o)
+                inc += y;
+        }
+        uint64_t run = inc - s;
+#pragma unroll
+        for (int q = 0; q < PER; q++) {
+            int idx = lane * PER + q;
+            if (idx < NV)
+                wtot[idx] = run;
+            run += a[q];
+        }
+        if (lane == 31)
+            wtot[NV] = inc;
+    }
+    __syncthreads();
+    total = wtot[ITEMS * kWarps];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++)
+        v[k] += wtot[k * kWarps + warp];
+}
+
+template <typename K>
+__global__ void __launch_bounds__(kThreads) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
+{
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    uint64_t *wtot = (uint64_t *)smem_raw;                        // kRunItems*kWarps + 1
+    K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT
+    K *sR = sL + kRunT;                                           // kRunT
+    __shared__ int64_t sh_part, sh_i0, sh_i1, sh_base_runs, sh_base_outs;
+    const K *L = (const K *)J.lkey;
+    const K *R = (const K *)J.rkey;
+    const int tid = threadIdx.x;
+    const int64_t ntot = J.nl + J.nr;
+
+    while (true) {
+        if (tid == 0)
+            sh_part = (int64_t)atomicAdd(&J.ctrs[0], 1u);
+        __syncthreads();
+        const int64_t p = sh_part;
+        if (p >= J.nparts)
+            break;
+        const int64_t d0 = p * kRunT, d1 = min(d0 + kRunT, ntot);
+        if (tid == 0)
+            sh_i0 = merge_path(L, J.nl, R, J.nr, d0);
+        if (tid == 32)
+            sh_i1 = merge_path(L, J.nl, R, J.nr, d1);
+        __syncthreads();
+        const int64_t i0 = sh_i0, i1 = sh_i1, j0 = d0 - i0, j1 = d1 - i1;
+        const int nL = (int)(i1 - i0), nR = (int)(j1 - j0);
+        for (int q = tid; q < nL; q += kThreads)
+            sL[q] = L[i0 + q];
+        for (int q = tid; q < nR; q += kThreads)
+            sR[q] = R[j0 + q];
+        __syncthreads();
+
+        uint64_t idx[kRunItems], cnt[kRunItems];
+        uint32_t rlenL[kRunItems], rlo[kRunItems], rlenR[kRunItems];
+        uint32_t emitted = 0;
+#pragma unroll
+        for (int k = 0; k < kRunItems; k++) {
+            const int li = k * kThreads + tid;
+            idx[k] = 0;
+            cnt[k] = 0;
+            rlenL[k] = rlo[k] = rlenR[k] = 0;
+            if (li < nL) {
+                const K key = sL[li];
+                const int64_t gi = i0 + li;
+                const bool start = gi == 0 || (li > 0 ? sL[li - 1] != key : L[gi - 1] != key);
+                if (start) {
+                    const int lo_l = lower_bound_smem(sR, nR, key);
+                    const int hi_l = upper_bound_smem(sR, nR, key);
+                    int64_t hi = j0 + hi_l;
+                    if (hi_l == nR)
+                        hi = gallop_upper(R, hi, J.nr, key);
+                    const int64_t lo = j0 + lo_l;
+                    if (hi > lo) {
+                        const int e_l = li + upper_bound_smem(sL + li, nL - li, key);
+                        int64_t iend = i0 + e_l;
+                        if (e_l == nL)
+                            iend = gallop_upper(L, iend, J.nl, key);
+                        emitted |= 1u << k;
+                        idx[k] = 1;
+                        cnt[k] = (uint64_t)(iend - gi) * (uint64_t)(hi - lo);
+                        rlenL[k] = (uint32_t)(iend - gi);
+                        rlo[k] = (uint32_t)lo;
+                        rlenR[k] = (uint32_t)(hi - lo);
+                    }
+                }
+            }
+        }
+        uint64_t tot_runs, tot_outs;
+        block_scan_u64<kRunItems>(idx, wtot, tot_runs);
+        block_scan_u64<kRunItems>(cnt, wtot, tot_outs);
+        if (tid < 32) {
+            const uint64_t br = lookback_warp(J.status_runs, p, tot_runs, J.epoch_runs);
+            const uint64_t bo = lookback_warp(J.status_outs, p, tot_outs, J.epoch_outs);
+            if (tid == 0) {
+                sh_base_runs = (int64_t)br;
+                sh_base_outs = (int64_t)bo;
+                if (p == J.nparts - 1) {
+                    J.totals[0] = (int64_t)(br + tot_runs);
+                    J.totals[1] = (int64_t)(bo + tot_outs);
+                }
+            }
+        }
+        __syncthreads();
+        const int64_t br = sh_base_runs, bo = sh_base_outs;
+#pragma unroll
+        for (int k = 0; k < kRunItems; k++) {
+            if ((emitted >> k) & 1u) {
+                const int64_t r = br + (int64_t)idx[k];
+                if (r < J.cap_runs) {
+                    J.s[r] = (uint32_t)(i0 + k * kThreads + tid);
+                    J.lenL[r] = rlenL[k];
+                    J.lo[r] = rlo[k];
+                    J.lenR[r] = rlenR[k];
+                    J.off[r] = bo + cnt[k];
+                }
+            }
+        }
+        __syncthreads();
+    }
+    if (J.nparts == 0 && blockIdx.x == 0 && tid == 0) {
+        J.totals[0] = 0;
+        J.totals[1] = 0;
+    }
+    cta_exit_reset(J.ctrs);
+}
+
+// first run of every expansion tile: tile_run[t] = upper_bound(off, t*T) - 1
+__global__ void k_tile_runs(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run)
+{
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= ntiles)
+        return;
+    const uint64_t o = (uint64_t)(t * T);
+    int64_t lo = 0, hi = nruns;
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if (off[mid] <= o) lo = mid + 1;
+        else hi = mid;
+    }
+    tile_run[t] = lo - 1;
+}
+
+// ===========================================================================
+// JOIN phase 2 — output-balanced expansion.  Tile = 2304 consecutive join
+// candidates (so a hot key's lenL x lenR block is spread over many CTAs).  The
+// tile's run records are cached in smem; thread t expands candidates
+// [t*9, t*9+9) of the tile (one binary search, then a forward walk), gathers
+// the live join columns into smem slots, and the fused downstream chain runs on
+// the tile exactly as in the scan kernel (§4.3.2: JOIN inside the CTA,
+// then the consumer operators, then one compacted dump).
+// ===========================================================================
+struct JoinCtl {
+    int64_t tile;
+    EmitSmem<kJoinItems> es;
+};
+
+__global__ void __launch_bounds__(kThreads) k_join_expand(const __grid_constant__ ChainProg P,
+                                                          const __grid_constant__ TileLaunch L,
+                                                          const __grid_constant__ JoinExpand X)
+{
+    constexpr int T = kThreads * kJoinItems;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    JoinCtl *ctl = (JoinCtl *)smem_raw;
+    uint64_t *c_off = (uint64_t *)(smem_raw + align_up(sizeof(JoinCtl), 128));   // T + 1
+    uint32_t *c_s = (uint32_t *)(c_off + (T + 1));
+    uint32_t *c_lo = c_s + (T + 1);
+    uint32_t *c_lenR = c_lo + (T + 1);
+    char *tilebuf = (char *)smem_raw + align_up(sizeof(JoinCtl), 128) + align_up((size_t)(T + 1) * 20, 128);
+    char *scratch = tilebuf + P.stage_bytes;
+    const int tid = threadIdx.x;
+    const int64_t ntiles = (L.n + T - 1) / T;
+
+    while (true) {
+        if (tid == 0)
+            ctl->tile = (int64_t)atomicAdd(&L.ctrs[0], 1u);
+        __syncthreads();
+        const int64_t t = ctl->tile;
+        if (t >= ntiles)
+            break;
+        const int64_t o0 = t * T;
+        const int rows = (int)min((int64_t)T, L.n - o0);
+        const int64_t r0 = X.tile_run[t];
+        const int64_t r1 = (t + 1 < ntiles) ? X.tile_run[t + 1] : X.nruns - 1;
+        const int nr = (int)(r1 - r0 + 1);
+        for (int q = tid; q < nr; q += kThreads) {
+            c_off[q] = X.off[r0 + q];
+            c_s[q] = X.s[r0 + q];
+            c_lo[q] = X.lo[r0 + q];
+            c_lenR[q] = X.lenR[r0 + q];
+        }
+        __syncthreads();
+
+        uint32_t ii[kJoinItems], jj[kJoinItems];
+        const int first = tid * kJoinItems;
+        if (first < rows) {
+            const uint64_t o = (uint64_t)(o0 + first);
+            int lo = 0, hi = nr;
+            while (lo < hi) {
+                int mid = (lo + hi) >> 1;
+                if (c_off[mid] <= o) lo = mid + 1;
+                else hi = mid;
+            }
+            int r = lo - 1;
+#pragma unroll
+            for (int k = 0; k < kJoinItems; k++) {
+                const uint64_t oo = o + k;
+                ii[k] = jj[k] = 0;
+                if (first + k < rows) {
+                    while (r + 1 < nr && c_off[r + 1] <= oo)
+                        r++;
+                    const uint64_t d = oo - c_off[r];
+                    const uint32_t lr = c_lenR[r];
+                    uint64_t qi, qj;
+                    if (d < 0xffffffffull) {
+                        qi = (uint32_t)d / lr;
+                        qj = (uint32_t)d - (uint32_t)qi * lr;
+                    } else {
+                        qi = d / lr;
+                        qj = d - qi * lr;
+                    }
+                    ii[k] = c_s[r] + (uint32_t)qi;
+                    jj[k] = c_lo[r] + (uint32_t)qj;
+                }
+            }
+            for (int c = 0; c < X.ncols; c++) {
+                char *dst = tilebuf + P.slot[X.dst_slot[c]].off;
+                const int w = type_width(P.slot[X.dst_slot[c]].type);
+                const char *src = (const char *)X.src[c];
+                const bool right = X.from_right[c];
+#pragma unroll
+                for (int k = 0; k < kJoinItems; k++) {
+                    if (first + k < rows) {
+                        const size_t row = right ? jj[k] : ii[k];
+                        if (w == 4)
+                            ((uint32_t *)dst)[first + k] = ((const uint32_t *)src)[row];
+                        else if (w == 8)
+                            ((uint64_t *)dst)[first + k] = ((const uint64_t *)src)[row];
+                        else
+                            ((uint8_t *)dst)[first + k] = ((const uint8_t *)src)[row];
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        uint32_t mask = 0;
+#pragma unroll
+        for (int k = 0; k < kJoinItems; k++)
+            if (k * kThreads + tid < rows)
+                mask |= 1u << k;
+        mask = run_ops<kJoinItems>(P, tilebuf, scratch, mask);
+        emit_tile<kJoinItems>(P, tilebuf, scratch, mask, t, ntiles, L, &ctl->es);
+        __syncthreads();
+    }
+    if (ntiles == 0 && blockIdx.x == 0 && tid == 0)
+        *L.n_dev = 0;
+    cta_exit_reset(L.ctrs);
+}
+
+// ===========================================================================
+// Host launchers
+// ===========================================================================
+size_t scan_ctl_bytes() { return align_up(sizeof(CtlSmem<kScanItems>), 128); }   // >= CtlSmem<4>
+size_t join_ctl_bytes() { return align_up(sizeof(JoinCtl), 128); }
+size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
+int scan_tile() { return kThreads * kScanItems; }
+int join_expand_tile() { return kThreads * kJoinItems; }
+
+size_t join_runs_smem(int key_type)
+{
+    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)kRunT * type_width(key_type);
+}
+
+template <typename F>
+static int occ(F f, size_t smem)
+{
+    int n = 0;
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, kThreads, smem) != cudaSuccess)
+        return 0;
+    return n;
+}
+
+int chain_occupancy(int which, int items, size_t smem)
+{
+    switch (which) {
+    case 0: return items == 4 ? occ(k_scan_chain<4, false>, smem) : occ(k_scan_chain<8, false>, smem);
+    case 1: return items == 4 ? occ(k_scan_chain<4, true>, smem) : occ(k_scan_chain<8, true>, smem);
+    case 2: return occ(k_join_expand, smem);
+    default: return occ(k_join_runs<uint64_t>, smem);
+    }
+}
+
+template <int ITEMS, bool AGG>
+static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
+{
+    cudaFuncSetAttribute(k_scan_chain<ITEMS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_scan_chain<ITEMS, AGG><<<grid, kThreads, smem, s>>>(P, L);
+    return cudaGetLastError();
+}
+
+cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int items, size_t smem, int grid,
+                              cudaStream_t s)
+{
+    if (items == 4)
+        return agg ? sc<4, true>(P, L, smem, grid, s) : sc<4, false>(P, L, smem, grid, s);
+    return agg ? sc<8, true>(P, L, smem, grid, s) : sc<8, false>(P, L, smem, grid, s);
+}
+
+cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s)
+{
+    k_agg_finalize<<<1, kThreads, 0, s>>>(F);
+    return cudaGetLastError();
+}
+
+template <typename K>
+static cudaError_t jr(const JoinRunsLaunch &J, size_t smem, int grid, cudaStream_t s)
+{
+    cudaFuncSetAttribute(k_join_runs<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_join_runs<K><<<grid, kThreads, smem, s>>>(J);
+    return cudaGetLastError();
+}
+
+cudaError_t join_runs_launch(const JoinRunsLaunch &J, int key_type, size_t smem, int grid, cudaStream_t s)
+{
+    switch (key_type) {
+    case T_I32: return jr<int32_t>(J, smem, grid, s);
+    case T_U32: return jr<uint32_t>(J, smem, grid, s);
+    case T_I64: return jr<int64_t>(J, smem, grid, s);
+    case T_U64: return jr<uint64_t>(J, smem, grid, s);
+    default: return jr<uint8_t>(J, smem, grid, s);
+    }
+}
+
+cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run,
+                             cudaStream_t s)
+{
+    if (ntiles > 0)
+        k_tile_runs<<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(off, nruns, ntiles, T, tile_run);
+    return cudaGetLastError();
+}
+
+cudaError_t join_expand_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem,
+                               int grid, cudaStream_t s)
+{
+    cudaFuncSetAttribute(k_join_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_join_expand<<<grid, kThreads, smem, s>>>(P, L, X);
+    return cudaGetLastError();
+}
+
+}  // namespace rw

@@ -1,0 +1,66 @@
+// kernels.h — host-side launch interface of the sm_100a kernels (internal).
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include "internal.h"
+
+namespace rw {
+
+constexpr int kMaxStages = 8;
+
+struct AggFinal {
+    const unsigned long long *acc;   // D * NA * 2 (lo, hi); zeroed by the finalize kernel after reading
+    unsigned long long *acc_w;       // same pointer, writable
+    int32_t D, NA, ngc;
+    int32_t gdomain[kMaxGroupCols];
+    uint8_t gtype[kMaxGroupCols];
+    int32_t nreq;                    // requested aggregates in output order
+    uint8_t req_is_sum[kMaxAggs];
+    int16_t req_acc[kMaxAggs];       // accumulator index a (0 = count)
+    void *out[kMaxOut];
+    int64_t capacity;
+    int64_t *n_dev;
+    int32_t *err;                    // err[0] -> err[1], err[0] = 0
+};
+
+struct JoinRunsLaunch {
+    const void *lkey, *rkey;
+    int64_t nl, nr;
+    int64_t nparts;
+    uint32_t *s, *lenL, *lo, *lenR;
+    uint64_t *off;
+    int64_t cap_runs;
+    uint64_t *status_runs, *status_outs;
+    uint32_t epoch_runs, epoch_outs;
+    uint32_t *ctrs;
+    int64_t *totals;                 // [0] runs, [1] join candidates
+};
+
+struct JoinExpand {
+    const uint32_t *s, *lo, *lenR;
+    const uint64_t *off;
+    const int64_t *tile_run;
+    int64_t nruns;
+    int32_t ncols;                   // gathered (live) join output columns
+    const void *src[kMaxSlots];
+    uint8_t from_right[kMaxSlots];
+    int16_t dst_slot[kMaxSlots];
+};
+
+size_t scan_ctl_bytes();
+size_t join_ctl_bytes();
+size_t join_run_cache_bytes();
+int chain_occupancy(int which, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs
+cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int items, size_t smem, int grid,
+                              cudaStream_t s);
+cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s);
+cudaError_t join_runs_launch(const JoinRunsLaunch &J, int key_type, size_t smem, int grid, cudaStream_t s);
+size_t join_runs_smem(int key_type);
+cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run,
+                             cudaStream_t s);
+cudaError_t join_expand_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem,
+                               int grid, cudaStream_t s);
+int join_expand_tile();
+int scan_tile();
+
+}  // namespace rw

@@ -1,0 +1,1562 @@
+// rw_api.cpp — C ABI (include/rw.h), plan builder, fusion legality / grouping
+// (Algorithm 1 and 2 analogues, §4.1-4.2), lowering of each fused
+// group to a ChainProg, and the stream-ordered executor.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "plan.h"
+
+using namespace rw;
+
+namespace {
+
+thread_local std::string g_err;
+
+struct RwError {
+    rw_status s;
+    std::string msg;
+};
+
+[[noreturn]] void raise(rw_status s, const std::string &m) { throw RwError{s, m}; }
+
+void cuda_check(cudaError_t e, const char *what)
+{
+    if (e != cudaSuccess)
+        raise(RW_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+const i128 I128_BIG = ((i128)1) << 120;
+
+i128 clampi(i128 v) { return v > I128_BIG ? I128_BIG : (v < -I128_BIG ? -I128_BIG : v); }
+
+}  // namespace
+
+namespace rw {
+
+const char *dep_name(int d) { return d == DEP_THREAD ? "thread" : d == DEP_CTA ? "CTA" : "kernel"; }
+
+Interval type_range(int t)
+{
+    switch (t) {
+    case T_I32: return {INT32_MIN, INT32_MAX};
+    case T_U32: return {0, UINT32_MAX};
+    case T_I64: return {INT64_MIN, INT64_MAX};
+    case T_U64: return {0, (i128)UINT64_MAX};
+    default: return {0, 255};
+    }
+}
+
+bool fits(const Interval &v, int t)
+{
+    Interval r = type_range(t);
+    return v.lo >= r.lo && v.hi <= r.hi;
+}
+
+i128 wrap_to(int t, i128 v)
+{
+    unsigned __int128 u = (unsigned __int128)v;
+    switch (t) {
+    case T_I32: return (int32_t)(uint32_t)u;
+    case T_U32: return (uint32_t)u;
+    case T_I64: return (int64_t)(uint64_t)u;
+    case T_U64: return (uint64_t)u;
+    default: return (uint8_t)u;
+    }
+}
+
+}  // namespace rw
+
+// ===========================================================================
+// Plan object
+// ===========================================================================
+struct Rel {
+    std::vector<int> types;
+    std::vector<const void *> cols;
+    int64_t n_host = -1;          // known row count, or -1
+    const int64_t *n_dev = nullptr;
+    int64_t cap = 0;              // upper bound on rows
+};
+
+struct Lowered {
+    ChainProg P;
+    std::vector<int> in_src;      // input slot i <- source column in_src[i]
+    int items = 8, stages = 2, ctas = 1;
+    size_t smem = 0;
+    bool agg = false;
+    AggFinal F;
+};
+
+struct rw_plan {
+    rw_plan_opts o;
+    cudaStream_t stream = nullptr;
+    int sms = 148;
+    std::vector<Node> nodes;
+    std::vector<int> inputs;      // node id of each declared input, declaration order
+    // persistent scratch
+    uint64_t *status = nullptr;
+    int64_t status_cap = 0;
+    uint32_t *ctrs = nullptr;     // 2 counters
+    int64_t *cnt = nullptr;       // per-group row counts (grown)
+    int cnt_cap = 0;
+    int64_t *jtot = nullptr;      // join totals: 2 int64 per join group
+    int64_t *jtot_host = nullptr; // pinned mirror
+    int32_t *err = nullptr;       // [0] running domain errors, [1] last finalised
+    std::map<int, unsigned long long *> agg_acc;
+    uint32_t epoch = 0;
+    int64_t launches = 0;
+    std::vector<void *> temps;    // freed (stream-ordered) at the end of every execute
+};
+
+namespace {
+
+void *dev_alloc(rw_plan *p, size_t bytes)
+{
+    void *ptr = nullptr;
+    if (bytes == 0)
+        bytes = 16;
+    cudaError_t e = cudaMallocAsync(&ptr, bytes, p->stream);
+    if (e == cudaErrorMemoryAllocation)
+        raise(RW_E_OOM, "cudaMallocAsync: out of device memory");
+    cuda_check(e, "cudaMallocAsync");
+    return ptr;
+}
+
+void *temp_alloc(rw_plan *p, size_t bytes)
+{
+    void *ptr = dev_alloc(p, bytes);
+    p->temps.push_back(ptr);
+    return ptr;
+}
+
+void free_temps(rw_plan *p)
+{
+    for (void *t : p->temps)
+        cudaFreeAsync(t, p->stream);
+    p->temps.clear();
+}
+
+void ensure_status(rw_plan *p, int64_t need)
+{
+    if (need <= p->status_cap)
+        return;
+    int64_t cap = std::max<int64_t>(need, 2 * p->status_cap);
+    cap = std::max<int64_t>(cap, 4096);
+    if (p->status)
+        cudaFreeAsync(p->status, p->stream);
+    p->status = (uint64_t *)dev_alloc(p, (size_t)cap * 8);
+    cuda_check(cudaMemsetAsync(p->status, 0, (size_t)cap * 8, p->stream), "memset status");
+    p->status_cap = cap;
+}
+
+uint32_t next_epoch(rw_plan *p)
+{
+    p->epoch++;
+    if (p->epoch > 0xffff) {
+        p->epoch = 1;
+        if (p->status)
+            cuda_check(cudaMemsetAsync(p->status, 0, (size_t)p->status_cap * 8, p->stream), "memset status");
+    }
+    return p->epoch;
+}
+
+const Node &node_at(const rw_plan *p, int id)
+{
+    if (id < 0 || id >= (int)p->nodes.size())
+        raise(RW_E_ARG, "node id " + std::to_string(id) + " out of range");
+    return p->nodes[id];
+}
+
+bool is_unary_chain(NodeKind k) { return k == N_SELECT || k == N_PROJECT; }
+
+// ---------------------------------------------------------------------------
+// Interval analysis of PROJECT expressions (reading A8; strict mode rejects wrap)
+// ---------------------------------------------------------------------------
+Interval expr_interval(const Node &in, const std::vector<rw_expr> &e, int i, std::vector<Interval> &memo,
+                       std::vector<char> &done, bool strict)
+{
+    if (done[i])
+        return memo[i];
+    const rw_expr &x = e[i];
+    Interval r;
+    auto finish = [&](Interval v) {
+        if (!fits(v, x.type)) {
+            if (strict && (x.type == T_I64 || x.type == T_U64))
+                raise(RW_E_OVERFLOW, "expression node " + std::to_string(i) + " may wrap in its 64-bit type");
+            v = type_range(x.type);
+        }
+        return v;
+    };
+    switch (x.op) {
+    case RW_COL: r = finish(in.bounds[x.a]); break;
+    case RW_CONST: {
+        i128 v = wrap_to(x.type, x.k);
+        r = {v, v};
+        break;
+    }
+    case RW_ADD: case RW_SUB: case RW_MUL: {
+        Interval a = expr_interval(in, e, x.a, memo, done, strict);
+        Interval b = expr_interval(in, e, x.b, memo, done, strict);
+        // operands are first converted into x.type
+        if (!fits(a, x.type)) a = type_range(x.type);
+        if (!fits(b, x.type)) b = type_range(x.type);
+        if (x.op == RW_ADD) r = {clampi(a.lo + b.lo), clampi(a.hi + b.hi)};
+        else if (x.op == RW_SUB) r = {clampi(a.lo - b.hi), clampi(a.hi - b.lo)};
+        else {
+            auto m = [](i128 u, i128 v) {
+                i128 au = u < 0 ? -u : u, av = v < 0 ? -v : v;
+                if (au != 0 && av > I128_BIG / au)
+                    return ((u < 0) != (v < 0)) ? -I128_BIG : I128_BIG;
+                return u * v;
+            };
+            i128 c[4] = {m(a.lo, b.lo), m(a.lo, b.hi), m(a.hi, b.lo), m(a.hi, b.hi)};
+            r = {*std::min_element(c, c + 4), *std::max_element(c, c + 4)};
+        }
+        r = finish(r);
+        break;
+    }
+    case RW_DIVC: {
+        Interval a = expr_interval(in, e, x.a, memo, done, strict);
+        if (!fits(a, x.type)) a = type_range(x.type);
+        i128 k = wrap_to(x.type, x.k);
+        i128 c1 = a.lo / k, c2 = a.hi / k;
+        r = {std::min(c1, c2), std::max(c1, c2)};
+        if (a.lo <= 0 && a.hi >= 0) {
+            r.lo = std::min<i128>(r.lo, 0);
+            r.hi = std::max<i128>(r.hi, 0);
+        }
+        r = finish(r);
+        break;
+    }
+    default: raise(RW_E_ARG, "bad expression op");
+    }
+    memo[i] = r;
+    done[i] = 1;
+    return r;
+}
+
+// ---------------------------------------------------------------------------
+// Grouping: Algorithm 1 (drop kernel-dependence edges, connected components)
+// and Algorithm 2 (greedy, earliest operator first, under the resource budget)
+// analogues.  Each group becomes one kernel template instance.
+// ---------------------------------------------------------------------------
+struct Grouping {
+    std::vector<Group> groups;
+    std::map<int, int> produced_by;     // node -> group index
+    std::vector<int> consumers;         // within the reachable sub-DAG
+    std::vector<char> reach;
+    std::vector<std::string> notes;
+};
+
+void mark_reach(const rw_plan *p, int id, Grouping &G)
+{
+    if (G.reach[id])
+        return;
+    G.reach[id] = 1;
+    const Node &n = p->nodes[id];
+    if (n.in >= 0) mark_reach(p, n.in, G);
+    if (n.left >= 0) mark_reach(p, n.left, G);
+    if (n.right >= 0) mark_reach(p, n.right, G);
+}
+
+int make_group(const rw_plan *p, int id, Grouping &G);
+
+int dep_group(const rw_plan *p, int id, Grouping &G)
+{
+    if (p->nodes[id].kind == N_INPUT)
+        return -1;
+    return make_group(p, id, G);
+}
+
+int make_group(const rw_plan *p, int id, Grouping &G)
+{
+    auto it = G.produced_by.find(id);
+    if (it != G.produced_by.end())
+        return it->second;
+    const bool fuse = p->o.fuse != 0;
+    const Node &n = p->nodes[id];
+    Group g;
+    g.out = id;
+    int cur = id;
+    if (n.kind == N_AGG) {
+        g.agg = id;
+        cur = n.in;
+        if (!fuse || !is_unary_chain(p->nodes[cur].kind) || G.consumers[cur] != 1) {
+            // AGG directly over a relation (or operator-at-a-time mode)
+            g.kind = G_SCAN;
+            g.source = cur;
+            int d = dep_group(p, cur, G);
+            if (d >= 0) g.deps.push_back(d);
+            G.groups.push_back(g);
+            return G.produced_by[id] = (int)G.groups.size() - 1;
+        }
+    }
+    if (n.kind == N_JOIN) {
+        g.kind = G_JOIN;
+        g.join = id;
+        int a = dep_group(p, n.left, G), b = dep_group(p, n.right, G);
+        if (a >= 0) g.deps.push_back(a);
+        if (b >= 0) g.deps.push_back(b);
+        G.groups.push_back(g);
+        return G.produced_by[id] = (int)G.groups.size() - 1;
+    }
+    // cur is SELECT / PROJECT: absorb producers while the edge is thread dependence
+    // with a single consumer (§4.3.1)
+    std::vector<int> chain{cur};
+    int src = p->nodes[cur].in;
+    while (fuse && is_unary_chain(p->nodes[src].kind) && G.consumers[src] == 1) {
+        chain.insert(chain.begin(), src);
+        src = p->nodes[src].in;
+    }
+    if (!fuse) {
+        // operator-at-a-time: one operator per group
+        chain.assign(1, cur);
+        src = p->nodes[cur].in;
+    }
+    if (g.agg >= 0 && fuse && p->nodes[src].kind == N_JOIN && G.consumers[src] == 1) {
+        // JOIN -> chain -> AGG: the join expansion materialises the chain's output and
+        // the aggregate scans it (the expansion kernel has no aggregate terminal yet)
+        const int mid = chain.back();
+        g.kind = G_SCAN;
+        g.source = mid;
+        g.deps.push_back(make_group(p, mid, G));
+        G.groups.push_back(g);
+        return G.produced_by[id] = (int)G.groups.size() - 1;
+    }
+    g.chain = chain;
+    if (fuse && p->nodes[src].kind == N_JOIN && G.consumers[src] == 1) {
+        // JOIN -> SELECT/PROJECT: fused into the join expansion (CTA dependence)
+        g.kind = G_JOIN;
+        g.join = src;
+        const Node &j = p->nodes[src];
+        int a = dep_group(p, j.left, G), b = dep_group(p, j.right, G);
+        if (a >= 0) g.deps.push_back(a);
+        if (b >= 0) g.deps.push_back(b);
+    } else {
+        g.kind = G_SCAN;
+        g.source = src;
+        int d = dep_group(p, src, G);
+        if (d >= 0) g.deps.push_back(d);
+    }
+    G.groups.push_back(g);
+    return G.produced_by[id] = (int)G.groups.size() - 1;
+}
+
+Grouping build_groups(const rw_plan *p, int out_node)
+{
+    Grouping G;
+    G.consumers.assign(p->nodes.size(), 0);
+    G.reach.assign(p->nodes.size(), 0);
+    mark_reach(p, out_node, G);
+    for (size_t i = 0; i < p->nodes.size(); i++) {
+        if (!G.reach[i]) continue;
+        const Node &n = p->nodes[i];
+        if (n.in >= 0) G.consumers[n.in]++;
+        if (n.left >= 0) G.consumers[n.left]++;
+        if (n.right >= 0) G.consumers[n.right]++;
+    }
+    G.consumers[out_node]++;   // the caller consumes the output
+    make_group(p, out_node, G);
+    return G;
+}
+
+// Dependence class of edge producer -> consumer (legality rules SURVEY §8(a)).
+int classify_edge(const rw_plan *p, int prod, int cons)
+{
+    const Node &a = p->nodes[prod];
+    const Node &b = p->nodes[cons];
+    if (a.kind == N_AGG)
+        return DEP_KERNEL;                       // AGG behaves like a global barrier
+    if (b.kind == N_SELECT || b.kind == N_PROJECT)
+        return DEP_THREAD;                       // Fig. 8(a)
+    if (b.kind == N_JOIN)
+        return a.nkey_sorted >= b.nkey ? DEP_CTA : DEP_KERNEL;   // Fig. 8(b); unsorted -> SORT boundary
+    if (b.kind == N_AGG)
+        return DEP_CTA;                          // block reduction + one global atomic stage
+    return DEP_KERNEL;
+}
+
+// ---------------------------------------------------------------------------
+// Lowering of one group to a ChainProg
+// ---------------------------------------------------------------------------
+struct SlotB {
+    int type;
+    bool input;
+    int src;
+    int last_use;
+    int region;
+};
+
+constexpr int kInf = 1 << 30;
+constexpr size_t kSmemLimit = 227 * 1024;
+
+size_t al128(size_t x) { return (x + 127) / 128 * 128; }
+
+void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowered &L)
+{
+    std::memset(&L.P, 0, sizeof(L.P));
+    std::memset(&L.F, 0, sizeof(L.F));
+    std::vector<SlotB> slots;
+    std::vector<DevOp> ops;
+    std::vector<int> src_slot(src_types.size(), -1);
+    auto get_src = [&](int c) {
+        if (src_slot[c] < 0) {
+            slots.push_back({src_types[c], true, c, -1, -1});
+            src_slot[c] = (int)slots.size() - 1;
+        }
+        return src_slot[c];
+    };
+    auto new_slot = [&](int type) {
+        slots.push_back({type, false, -1, -1, -1});
+        return (int)slots.size() - 1;
+    };
+    std::vector<int> cur(src_types.size());
+    for (size_t c = 0; c < cur.size(); c++)
+        cur[c] = -1 - (int)c;
+    auto resolve = [&](int v) { return v >= 0 ? v : get_src(-1 - v); };
+    auto push = [&](const DevOp &o) {
+        if ((int)ops.size() >= kMaxOps)
+            raise(RW_E_UNSUPPORTED, "fused group exceeds the micro-op budget");
+        ops.push_back(o);
+    };
+
+    for (int nid : g.chain) {
+        const Node &nd = p->nodes[nid];
+        if (nd.kind == N_SELECT) {
+            for (const rw_pred &a : nd.preds) {
+                DevOp o{};
+                o.kind = K_PRED;
+                o.op = (uint8_t)a.op;
+                o.a = (int16_t)resolve(cur[a.col]);
+                o.type = (uint8_t)slots[o.a].type;
+                o.dst = -1;
+                if (a.rhs_is_col) {
+                    o.b_is_slot = 1;
+                    o.b = (int16_t)resolve(cur[a.rhs_col]);
+                } else {
+                    o.b = -1;
+                    o.k = (int64_t)wrap_to(o.type, a.rhs_const);
+                }
+                push(o);
+            }
+        } else {   // PROJECT
+            const std::vector<rw_expr> &e = nd.exprs;
+            // value of an expression node: slot id (>= 0) or a constant
+            std::vector<int> vslot(e.size(), -2);
+            std::vector<i128> vconst(e.size(), 0);
+            std::vector<char> isconst(e.size(), 0);
+            std::function<void(int)> ev = [&](int i) {
+                if (vslot[i] != -2 || isconst[i])
+                    return;
+                const rw_expr &x = e[i];
+                if (x.op == RW_COL) {
+                    int s = resolve(cur[x.a]);
+                    if (slots[s].type == x.type) {
+                        vslot[i] = s;
+                    } else {
+                        int d = new_slot(x.type);
+                        DevOp o{};
+                        o.kind = K_EXPR; o.op = E_COPY; o.type = (uint8_t)x.type;
+                        o.dst = (int16_t)d; o.a = (int16_t)s; o.b = -1;
+                        push(o);
+                        vslot[i] = d;
+                    }
+                    return;
+                }
+                if (x.op == RW_CONST) {
+                    isconst[i] = 1;
+                    vconst[i] = wrap_to(x.type, x.k);
+                    return;
+                }
+                ev(x.a);
+                if (x.op != RW_DIVC)
+                    ev(x.b);
+                const int t = x.type;
+                auto fold = [&](i128 a, i128 b) -> i128 {
+                    unsigned __int128 ua = (unsigned __int128)wrap_to(t, a), ub = (unsigned __int128)wrap_to(t, b);
+                    switch (x.op) {
+                    case RW_ADD: return wrap_to(t, (i128)(ua + ub));
+                    case RW_SUB: return wrap_to(t, (i128)(ua - ub));
+                    case RW_MUL: return wrap_to(t, (i128)(ua * ub));
+                    default: {
+                        i128 sa = wrap_to(t, a), sb = wrap_to(t, b);
+                        return wrap_to(t, sa / sb);
+                    }
+                    }
+                };
+                if (x.op == RW_DIVC) {
+                    if (isconst[x.a]) {
+                        isconst[i] = 1;
+                        vconst[i] = fold(vconst[x.a], x.k);
+                        return;
+                    }
+                    int d = new_slot(t);
+                    DevOp o{};
+                    o.kind = K_EXPR; o.op = E_DIVC; o.type = (uint8_t)t;
+                    o.dst = (int16_t)d; o.a = (int16_t)vslot[x.a]; o.b = -1;
+                    o.k = (int64_t)wrap_to(t, x.k);
+                    push(o);
+                    vslot[i] = d;
+                    return;
+                }
+                if (isconst[x.a] && isconst[x.b]) {
+                    isconst[i] = 1;
+                    vconst[i] = fold(vconst[x.a], vconst[x.b]);
+                    return;
+                }
+                int d = new_slot(t);
+                DevOp o{};
+                o.kind = K_EXPR; o.type = (uint8_t)t; o.dst = (int16_t)d; o.b = -1;
+                const uint8_t base = x.op == RW_ADD ? E_ADD : x.op == RW_SUB ? E_SUB : E_MUL;
+                if (isconst[x.b]) {
+                    o.op = base; o.a = (int16_t)vslot[x.a]; o.k = (int64_t)wrap_to(t, vconst[x.b]);
+                } else if (isconst[x.a]) {
+                    o.op = base == E_SUB ? E_RSUB : base;
+                    o.a = (int16_t)vslot[x.b]; o.k = (int64_t)wrap_to(t, vconst[x.a]);
+                } else {
+                    o.op = base; o.a = (int16_t)vslot[x.a]; o.b = (int16_t)vslot[x.b]; o.b_is_slot = 1;
+                }
+                push(o);
+                vslot[i] = d;
+            };
+            std::vector<int> next;
+            for (int r : nd.roots) {
+                ev(r);
+                if (isconst[r]) {
+                    int d = new_slot(e[r].type);
+                    DevOp o{};
+                    o.kind = K_EXPR; o.op = E_CONST; o.type = (uint8_t)e[r].type;
+                    o.dst = (int16_t)d; o.a = -1; o.b = -1; o.k = (int64_t)vconst[r];
+                    push(o);
+                    next.push_back(d);
+                } else {
+                    next.push_back(vslot[r]);
+                }
+            }
+            cur = next;
+        }
+    }
+
+    // terminal
+    std::vector<int> term;
+    if (g.agg >= 0) {
+        const Node &a = p->nodes[g.agg];
+        L.agg = true;
+        L.P.is_agg = 1;
+        L.P.ngc = (int)a.gcols.size();
+        L.P.D = a.D;
+        for (size_t c = 0; c < a.gcols.size(); c++) {
+            int s = resolve(cur[a.gcols[c]]);
+            L.P.gslot[c] = (int16_t)s;
+            L.P.gdomain[c] = a.gdomain[c];
+            term.push_back(s);
+        }
+        int ns = 0;
+        const Node &an = p->nodes[a.in];
+        // flush period: rows whose |values| sum cannot leave int64 (uint64 for u64 sums)
+        unsigned __int128 flush = ((unsigned __int128)1) << 40;
+        L.F.nreq = (int)a.aggs.size();
+        for (size_t q = 0; q < a.aggs.size(); q++) {
+            if (a.aggs[q].op == RW_SUM) {
+                int s = resolve(cur[a.aggs[q].col]);
+                L.P.agg_slot[ns] = (int16_t)s;
+                const bool uns = slots[s].type == T_U64;
+                L.P.agg_unsigned[ns] = uns;
+                term.push_back(s);
+                Interval b = an.bounds[a.aggs[q].col];
+                unsigned __int128 mx = (unsigned __int128)(b.hi < 0 ? -b.hi : b.hi);
+                unsigned __int128 mn = (unsigned __int128)(b.lo < 0 ? -b.lo : b.lo);
+                if (mn > mx) mx = mn;
+                if (mx == 0) mx = 1;
+                unsigned __int128 lim = uns ? (unsigned __int128)UINT64_MAX : (unsigned __int128)INT64_MAX;
+                flush = std::min(flush, std::max<unsigned __int128>(1, lim / mx));
+                L.F.req_is_sum[q] = 1;
+                L.F.req_acc[q] = (int16_t)(1 + ns);
+                ns++;
+            } else {
+                L.F.req_is_sum[q] = 0;
+                L.F.req_acc[q] = 0;
+            }
+        }
+        L.P.nagg = ns;
+        L.P.flush_rows = (int64_t)flush;
+        L.F.D = a.D;
+        L.F.NA = ns + 1;
+        L.F.ngc = L.P.ngc;
+        for (int c = 0; c < L.P.ngc; c++) {
+            L.F.gdomain[c] = a.gdomain[c];
+            L.F.gtype[c] = (uint8_t)p->nodes[g.out].types[c];
+        }
+    } else {
+        for (int v : cur)
+            term.push_back(resolve(v));
+    }
+    if ((int)slots.size() > kMaxSlots)
+        raise(RW_E_UNSUPPORTED, "fused group needs more than 24 tile columns");
+
+    // liveness
+    for (size_t i = 0; i < ops.size(); i++) {
+        const DevOp &o = ops[i];
+        if (o.a >= 0) slots[o.a].last_use = std::max(slots[o.a].last_use, (int)i);
+        if (o.b_is_slot && o.b >= 0) slots[o.b].last_use = std::max(slots[o.b].last_use, (int)i);
+    }
+    for (int s : term)
+        slots[s].last_use = kInf;
+
+    // renumber: input slots first
+    std::vector<int> order, remap(slots.size());
+    for (size_t s = 0; s < slots.size(); s++)
+        if (slots[s].input) order.push_back((int)s);
+    const int nin = (int)order.size();
+    for (size_t s = 0; s < slots.size(); s++)
+        if (!slots[s].input) order.push_back((int)s);
+    for (size_t i = 0; i < order.size(); i++)
+        remap[order[i]] = (int)i;
+
+    // scratch regions for computed slots (reuse freed regions of equal width)
+    struct Region { int width; int owner; };
+    std::vector<Region> regions;
+    std::vector<int> dst_of_op(ops.size(), -1);
+    for (size_t i = 0; i < ops.size(); i++) {
+        if (ops[i].kind != K_EXPR) continue;
+        for (Region &r : regions)
+            if (r.owner >= 0 && slots[r.owner].last_use <= (int)i)
+                r.owner = -1;
+        const int d = ops[i].dst;
+        const int w = type_width(slots[d].type);
+        int got = -1;
+        for (size_t r = 0; r < regions.size(); r++)
+            if (regions[r].owner < 0 && regions[r].width == w) { got = (int)r; break; }
+        if (got < 0) {
+            regions.push_back({w, d});
+            got = (int)regions.size() - 1;
+        }
+        regions[got].owner = d;
+        slots[d].region = got;
+    }
+
+    // write ChainProg
+    ChainProg &P = L.P;
+    P.nslots = (int)slots.size();
+    P.nin = nin;
+    P.nops = (int)ops.size();
+    for (size_t i = 0; i < order.size(); i++) {
+        const SlotB &sb = slots[order[i]];
+        P.slot[i].type = (uint8_t)sb.type;
+        P.slot[i].is_input = sb.input ? 1 : 0;
+    }
+    L.in_src.clear();
+    for (int i = 0; i < nin; i++)
+        L.in_src.push_back(slots[order[i]].src);
+    for (size_t i = 0; i < ops.size(); i++) {
+        DevOp o = ops[i];
+        if (o.a >= 0) o.a = (int16_t)remap[o.a];
+        if (o.b_is_slot && o.b >= 0) o.b = (int16_t)remap[o.b];
+        if (o.dst >= 0) o.dst = (int16_t)remap[o.dst];
+        P.ops[i] = o;
+    }
+    if (L.agg) {
+        for (int c = 0; c < P.ngc; c++) P.gslot[c] = (int16_t)remap[P.gslot[c]];
+        for (int q = 0; q < P.nagg; q++) P.agg_slot[q] = (int16_t)remap[P.agg_slot[q]];
+    } else {
+        if ((int)term.size() > kMaxOut)
+            raise(RW_E_UNSUPPORTED, "more than 32 output columns");
+        P.nout = (int)term.size();
+        for (size_t j = 0; j < term.size(); j++)
+            P.out_slot[j] = (int16_t)remap[term[j]];
+    }
+
+    // tile geometry, stages and CTAs per SM (resource budget, §4.3.3)
+    auto layout = [&](int T) {
+        uint32_t off = 0;
+        for (int i = 0; i < nin; i++) {
+            P.slot[i].off = off;
+            off += (uint32_t)al128((size_t)T * type_width(P.slot[i].type));
+        }
+        P.stage_bytes = off;
+        std::vector<uint32_t> roff(regions.size());
+        uint32_t so = 0;
+        for (size_t r = 0; r < regions.size(); r++) {
+            roff[r] = so;
+            so += (uint32_t)al128((size_t)T * regions[r].width);
+        }
+        P.scratch_bytes = so;
+        for (size_t i = nin; i < order.size(); i++) {
+            const SlotB &sb = slots[order[i]];
+            P.slot[i].off = sb.region >= 0 ? roff[sb.region] : 0;
+        }
+    };
+    const size_t agg_bytes =
+        L.agg ? (size_t)P.D * (P.nagg + 1) * kThreads * 8 + al128((size_t)P.D * (P.nagg + 1) * 16) : 0;
+    if (L.agg && (size_t)P.D * (P.nagg + 1) > (size_t)kMaxAggSlots)
+        raise(RW_E_UNSUPPORTED, "aggregate needs more than 4096 accumulators");
+
+    if (g.kind == G_JOIN) {
+        const int T = join_expand_tile();
+        layout(T);
+        L.items = kJoinItems;
+        L.stages = 1;
+        L.smem = join_ctl_bytes() + join_run_cache_bytes() + P.stage_bytes + P.scratch_bytes;
+        if (L.smem > kSmemLimit)
+            raise(RW_E_UNSUPPORTED, "join group exceeds the shared-memory budget");
+        L.ctas = std::max(1, chain_occupancy(2, kJoinItems, L.smem));
+        return;
+    }
+    const int want_stages = p->o.stages > 0 ? std::min(p->o.stages, kMaxStages) : 0;
+    double best = -1;
+    for (int items : {8, 4}) {
+        const int T = kThreads * items;
+        layout(T);
+        for (int S = kMaxStages; S >= 1; S--) {
+            if (want_stages && S != want_stages) continue;
+            if (!want_stages && S > 4) continue;
+            size_t smem = scan_ctl_bytes() + (size_t)S * P.stage_bytes + P.scratch_bytes + agg_bytes;
+            if (smem > kSmemLimit) continue;
+            int occ = chain_occupancy(L.agg ? 1 : 0, items, smem);
+            if (occ <= 0) continue;
+            if (p->o.ctas_per_sm > 0) occ = std::min(occ, p->o.ctas_per_sm);
+            double inflight = (double)occ * S * std::max<uint32_t>(P.stage_bytes, 1);
+            double score = inflight + (items == 8 ? 1.0 : 0.0) + 0.01 * occ;
+            if (score > best) {
+                best = score;
+                L.items = items;
+                L.stages = S;
+                L.smem = smem;
+                L.ctas = occ;
+            }
+        }
+    }
+    if (best < 0)
+        raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
+    layout(kThreads * L.items);
+}
+
+// ---------------------------------------------------------------------------
+// Execution
+// ---------------------------------------------------------------------------
+struct ExecCtx {
+    rw_plan *p;
+    const rw_relation_in *in;
+    int nin;
+    Grouping G;
+    std::vector<Rel> rels;             // per group output
+    std::vector<char> done;
+    int final_group;
+    rw_relation_out *out;
+    int64_t *final_n_dev;
+};
+
+Rel input_rel(ExecCtx &X, int node)
+{
+    const Node &n = X.p->nodes[node];
+    const rw_relation_in &ri = X.in[n.input_index];
+    Rel r;
+    r.types = n.types;
+    for (size_t c = 0; c < n.types.size(); c++)
+        r.cols.push_back(ri.cols[c]);
+    r.n_host = ri.n;
+    r.cap = ri.n;
+    return r;
+}
+
+Rel rel_of(ExecCtx &X, int node)
+{
+    if (X.p->nodes[node].kind == N_INPUT)
+        return input_rel(X, node);
+    return X.rels[X.G.produced_by.at(node)];
+}
+
+int64_t host_count(ExecCtx &X, const Rel &r)
+{
+    if (r.n_host >= 0)
+        return r.n_host;
+    rw_plan *p = X.p;
+    cuda_check(cudaMemcpyAsync(p->jtot_host + 2, r.n_dev, 8, cudaMemcpyDeviceToHost, p->stream), "copy count");
+    cuda_check(cudaStreamSynchronize(p->stream), "sync");
+    return p->jtot_host[2];
+}
+
+void make_output(ExecCtx &X, int gi, const std::vector<int> &types, int64_t cap, Rel &o, std::vector<void *> &outp,
+                 int64_t &capacity, int64_t *&n_dev)
+{
+    rw_plan *p = X.p;
+    o.types = types;
+    outp.clear();
+    if (gi == X.final_group) {
+        for (size_t c = 0; c < types.size(); c++)
+            outp.push_back(X.out->cols[c]);
+        capacity = X.out->capacity;
+        n_dev = X.final_n_dev;
+    } else {
+        for (int t : types)
+            outp.push_back(temp_alloc(p, (size_t)std::max<int64_t>(cap, 1) * type_width(t)));
+        capacity = cap;
+        n_dev = p->cnt + gi;
+    }
+    for (void *q : outp)
+        o.cols.push_back(q);
+    o.n_dev = n_dev;
+    o.cap = std::min(cap, capacity);
+}
+
+unsigned long long *agg_buffer(rw_plan *p, int node, size_t words)
+{
+    auto it = p->agg_acc.find(node);
+    if (it != p->agg_acc.end())
+        return it->second;
+    unsigned long long *b = (unsigned long long *)dev_alloc(p, words * 8);
+    cuda_check(cudaMemsetAsync(b, 0, words * 8, p->stream), "memset agg");
+    p->agg_acc[node] = b;
+    return b;
+}
+
+void run_group(ExecCtx &X, int gi)
+{
+    if (X.done[gi])
+        return;
+    const Group &g = X.G.groups[gi];
+    for (int d : g.deps)
+        run_group(X, d);
+    rw_plan *p = X.p;
+    const Node &outn = p->nodes[g.out];
+    Rel o;
+    std::vector<void *> outp;
+    int64_t capacity = 0;
+    int64_t *n_dev = nullptr;
+
+    if (g.kind == G_SCAN && !p->o.fuse && p->o.zero_copy_project && g.agg < 0 && g.chain.size() == 1 &&
+        gi != X.final_group && p->nodes[g.chain[0]].kind == N_PROJECT) {
+        // operator-at-a-time variant with a zero-copy PROJECT: alias plain column references
+        const Node &pn = p->nodes[g.chain[0]];
+        bool plain = true;
+        for (int r : pn.roots)
+            plain = plain && pn.exprs[r].op == RW_COL && pn.exprs[r].type == p->nodes[pn.in].types[pn.exprs[r].a];
+        if (plain) {
+            Rel src = rel_of(X, g.source);
+            o = src;
+            o.types = pn.types;
+            o.cols.clear();
+            for (int r : pn.roots)
+                o.cols.push_back(src.cols[pn.exprs[r].a]);
+            X.rels[gi] = o;
+            X.done[gi] = 1;
+            return;
+        }
+    }
+    if (g.kind == G_SCAN) {
+        Rel src = rel_of(X, g.source);
+        Lowered L;
+        lower(p, g, src.types, L);
+        const int T = kThreads * L.items;
+        int64_t cap_out = L.agg ? p->nodes[g.agg].D : src.cap;
+        make_output(X, gi, outn.types, cap_out, o, outp, capacity, n_dev);
+        bool aligned = true;
+        for (int i = 0; i < L.P.nin; i++) {
+            L.P.in_ptr[i] = src.cols[L.in_src[i]];
+            if (((uintptr_t)L.P.in_ptr[i]) & 15)
+                aligned = false;
+        }
+        const int64_t max_tiles = (src.cap + T - 1) / T;
+        ensure_status(p, max_tiles + 1);
+        TileLaunch TL{};
+        TL.n = src.n_host >= 0 ? src.n_host : 0;
+        TL.n_ptr = src.n_host >= 0 ? nullptr : src.n_dev;
+        TL.stages = L.stages;
+        TL.use_tma = aligned ? 1 : 0;
+        TL.epoch = next_epoch(p);
+        TL.status = p->status;
+        TL.ctrs = p->ctrs;
+        TL.err = p->err;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(max_tiles, (int64_t)p->sms * L.ctas));
+        if (L.agg) {
+            const Node &an = p->nodes[g.agg];
+            const size_t words = (size_t)an.D * (L.P.nagg + 1) * 2;
+            unsigned long long *acc = agg_buffer(p, g.agg, words);
+            TL.agg_acc = acc;
+            TL.n_dev = n_dev;
+            cuda_check(scan_chain_launch(L.P, TL, true, L.items, L.smem, grid, p->stream), "k_scan_chain<agg>");
+            p->launches++;
+            L.F.acc = acc;
+            L.F.acc_w = acc;
+            for (size_t c = 0; c < outp.size(); c++)
+                L.F.out[c] = outp[c];
+            L.F.capacity = capacity;
+            L.F.n_dev = n_dev;
+            L.F.err = p->err;
+            cuda_check(agg_finalize_launch(L.F, p->stream), "k_agg_finalize");
+            p->launches++;
+        } else {
+            for (size_t c = 0; c < outp.size(); c++)
+                L.P.out_ptr[c] = outp[c];
+            L.P.out_capacity = capacity;
+            TL.n_dev = n_dev;
+            cuda_check(scan_chain_launch(L.P, TL, false, L.items, L.smem, grid, p->stream), "k_scan_chain");
+            p->launches++;
+        }
+    } else {
+        const Node &jn = p->nodes[g.join];
+        Rel lr = rel_of(X, jn.left), rr = rel_of(X, jn.right);
+        const int64_t nl = host_count(X, lr), nr = host_count(X, rr);
+        const int kt = lr.types[0];
+        // phase 1: run records
+        const int64_t T1 = 2048;
+        const int64_t nparts = (nl + nr + T1 - 1) / T1;
+        const int64_t cap_runs = std::max<int64_t>(1, std::min(nl, nr));
+        JoinRunsLaunch J{};
+        J.lkey = lr.cols[0];
+        J.rkey = rr.cols[0];
+        J.nl = nl;
+        J.nr = nr;
+        J.nparts = nparts;
+        J.s = (uint32_t *)temp_alloc(p, cap_runs * 4);
+        J.lenL = (uint32_t *)temp_alloc(p, cap_runs * 4);
+        J.lo = (uint32_t *)temp_alloc(p, cap_runs * 4);
+        J.lenR = (uint32_t *)temp_alloc(p, cap_runs * 4);
+        J.off = (uint64_t *)temp_alloc(p, cap_runs * 8);
+        J.cap_runs = cap_runs;
+        ensure_status(p, 2 * nparts + 2);
+        J.status_runs = p->status;
+        J.status_outs = p->status + nparts + 1;
+        J.epoch_runs = next_epoch(p);
+        J.epoch_outs = next_epoch(p);
+        J.ctrs = p->ctrs;
+        J.totals = p->jtot;
+        const size_t smem1 = join_runs_smem(kt);
+        const int occ1 = std::max(1, chain_occupancy(3, 8, smem1));
+        const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
+        cuda_check(join_runs_launch(J, kt, smem1, grid1, p->stream), "k_join_runs");
+        p->launches++;
+        cuda_check(cudaMemcpyAsync(p->jtot_host, p->jtot, 16, cudaMemcpyDeviceToHost, p->stream), "copy totals");
+        cuda_check(cudaStreamSynchronize(p->stream), "sync after join runs");
+        const int64_t nruns = p->jtot_host[0], total = p->jtot_host[1];
+        // phase 2: expansion fused with the downstream chain
+        std::vector<int> jtypes = jn.types;
+        Lowered L;
+        lower(p, g, jtypes, L);
+        make_output(X, gi, outn.types, total, o, outp, capacity, n_dev);
+        const int64_t T2 = join_expand_tile();
+        const int64_t ntiles = (total + T2 - 1) / T2;
+        int64_t *tile_run = (int64_t *)temp_alloc(p, (size_t)std::max<int64_t>(ntiles, 1) * 8);
+        cuda_check(tile_runs_launch(J.off, nruns, ntiles, T2, tile_run, p->stream), "k_tile_runs");
+        if (ntiles > 0) p->launches++;
+        JoinExpand XJ{};
+        XJ.s = J.s;
+        XJ.lo = J.lo;
+        XJ.lenR = J.lenR;
+        XJ.off = J.off;
+        XJ.tile_run = tile_run;
+        XJ.nruns = nruns;
+        const int nlc = (int)lr.types.size();
+        XJ.ncols = L.P.nin;
+        for (int i = 0; i < L.P.nin; i++) {
+            const int c = L.in_src[i];
+            if (c < nlc) {
+                XJ.src[i] = lr.cols[c];
+                XJ.from_right[i] = 0;
+            } else {
+                XJ.src[i] = rr.cols[c - nlc + jn.nkey];
+                XJ.from_right[i] = 1;
+            }
+            XJ.dst_slot[i] = (int16_t)i;
+        }
+        for (size_t c = 0; c < outp.size(); c++)
+            L.P.out_ptr[c] = outp[c];
+        L.P.out_capacity = capacity;
+        ensure_status(p, ntiles + 1);
+        TileLaunch TL{};
+        TL.n = total;
+        TL.stages = 1;
+        TL.epoch = next_epoch(p);
+        TL.status = p->status;
+        TL.ctrs = p->ctrs;
+        TL.n_dev = n_dev;
+        TL.err = p->err;
+        const int grid2 = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (int64_t)p->sms * L.ctas));
+        cuda_check(join_expand_launch(L.P, TL, XJ, L.smem, grid2, p->stream), "k_join_expand");
+        p->launches++;
+    }
+    X.rels[gi] = o;
+    X.done[gi] = 1;
+}
+
+std::vector<int> &schema_types(rw_plan *p, int node) { return p->nodes[node].types; }
+
+void check_inputs(rw_plan *p, const rw_relation_in *in, int nin)
+{
+    if (nin != (int)p->inputs.size())
+        raise(RW_E_ARG, "expected " + std::to_string(p->inputs.size()) + " input relations, got " + std::to_string(nin));
+    for (int i = 0; i < nin; i++) {
+        if (in[i].n < 0)
+            raise(RW_E_ARG, "negative row count");
+        if (in[i].n > (int64_t)UINT32_MAX)
+            raise(RW_E_UNSUPPORTED, "relations above 2^32 rows per GPU: shard across ranks");
+        if (in[i].n > 0 && !in[i].cols)
+            raise(RW_E_ARG, "null column array");
+    }
+}
+
+void execute(rw_plan *p, const rw_relation_in *in, int nin, int out_node, rw_relation_out *out)
+{
+    node_at(p, out_node);
+    if (!out || (!out->cols && out->capacity > 0))
+        raise(RW_E_ARG, "null output");
+    check_inputs(p, in, nin);
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    p->launches = 0;
+    if (p->nodes[out_node].kind == N_INPUT)
+        raise(RW_E_UNSUPPORTED, "output node is an input relation");
+    ExecCtx X;
+    X.p = p;
+    X.in = in;
+    X.nin = nin;
+    X.G = build_groups(p, out_node);
+    X.rels.resize(X.G.groups.size());
+    X.done.assign(X.G.groups.size(), 0);
+    X.final_group = X.G.produced_by.at(out_node);
+    X.out = out;
+    if ((int)X.G.groups.size() + 1 > p->cnt_cap) {
+        if (p->cnt) cudaFreeAsync(p->cnt, p->stream);
+        p->cnt_cap = (int)X.G.groups.size() + 8;
+        p->cnt = (int64_t *)dev_alloc(p, (size_t)p->cnt_cap * 8);
+    }
+    X.final_n_dev = out->n_dev ? out->n_dev : p->cnt + (p->cnt_cap - 1);
+    try {
+        run_group(X, X.final_group);
+    } catch (...) {
+        free_temps(p);
+        throw;
+    }
+    free_temps(p);
+    out->n = -1;
+    if (!out->n_dev) {
+        cuda_check(cudaMemcpyAsync(p->jtot_host + 2, X.final_n_dev, 8, cudaMemcpyDeviceToHost, p->stream), "copy n");
+        cuda_check(cudaMemcpyAsync(p->jtot_host + 3, p->err + 1, 4, cudaMemcpyDeviceToHost, p->stream), "copy err");
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+        out->n = p->jtot_host[2];
+        const int32_t derr = ((int32_t *)(p->jtot_host + 3))[0];
+        if (derr)
+            raise(RW_E_DOMAIN, std::to_string(derr) + " rows had a group value outside its domain");
+        if (out->n > out->capacity)
+            raise(RW_E_CAPACITY, "output needs " + std::to_string(out->n) + " rows, capacity " +
+                                     std::to_string(out->capacity));
+    }
+}
+
+std::string explain(rw_plan *p, int out_node)
+{
+    node_at(p, out_node);
+    std::ostringstream s;
+    static const char *kn[] = {"INPUT", "SELECT", "PROJECT", "JOIN", "AGG"};
+    Grouping G = build_groups(p, out_node);
+    s << "plan: " << p->nodes.size() << " nodes, output node " << out_node << ", fuse=" << p->o.fuse << "\n";
+    s << "edges:\n";
+    for (size_t i = 0; i < p->nodes.size(); i++) {
+        if (!G.reach[i]) continue;
+        const Node &n = p->nodes[i];
+        for (int pr : {n.in, n.left, n.right}) {
+            if (pr < 0) continue;
+            int gp = p->nodes[pr].kind == N_INPUT ? -1 : G.produced_by.count(pr) ? G.produced_by[pr] : -2;
+            int gc = -3;
+            for (size_t q = 0; q < G.groups.size(); q++) {
+                const Group &g = G.groups[q];
+                if (g.out == (int)i || g.join == (int)i || g.agg == (int)i ||
+                    std::find(g.chain.begin(), g.chain.end(), (int)i) != g.chain.end())
+                    gc = (int)q;
+            }
+            bool fused = false;
+            if (gc >= 0) {
+                const Group &g = G.groups[gc];
+                fused = pr == g.join || std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end();
+            }
+            (void)gp;
+            s << "  " << pr << "(" << kn[p->nodes[pr].kind] << ") -> " << i << "(" << kn[n.kind]
+              << "): " << dep_name(classify_edge(p, pr, (int)i)) << " dependence, "
+              << (fused ? "fused" : "materialised") << "\n";
+        }
+    }
+    s << "groups:\n";
+    for (size_t q = 0; q < G.groups.size(); q++) {
+        const Group &g = G.groups[q];
+        s << "  group " << q << ": " << (g.kind == G_SCAN ? "k_scan_chain" : "k_join_runs+k_join_expand");
+        if (g.agg >= 0) s << "<agg>+k_agg_finalize";
+        s << " nodes [";
+        if (g.kind == G_SCAN) s << "src " << g.source;
+        else s << "join " << g.join;
+        for (int c : g.chain) s << ", " << kn[p->nodes[c].kind] << " " << c;
+        if (g.agg >= 0) s << ", AGG " << g.agg;
+        s << "] -> node " << g.out;
+        try {
+            Lowered L;
+            std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
+            lower(p, g, st, L);
+            s << " | tile " << kThreads * L.items << " rows, stages " << L.stages << ", smem " << L.smem
+              << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
+              << L.P.nops;
+        } catch (const RwError &e) {
+            s << " | not lowerable: " << e.msg;
+        }
+        s << "\n";
+    }
+    return s.str();
+}
+
+}  // namespace
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+#define RW_TRY try {
+#define RW_CATCH                                          \
+    }                                                     \
+    catch (const RwError &e)                              \
+    {                                                     \
+        g_err = e.msg;                                    \
+        return e.s;                                       \
+    }                                                     \
+    catch (const std::bad_alloc &)                        \
+    {                                                     \
+        g_err = "host out of memory";                     \
+        return RW_E_OOM;                                  \
+    }                                                     \
+    catch (...)                                           \
+    {                                                     \
+        g_err = "unexpected internal error";              \
+        return RW_E_STATE;                                \
+    }
+
+extern "C" {
+
+const char *rw_status_str(rw_status s)
+{
+    switch (s) {
+    case RW_OK: return "RW_OK";
+    case RW_E_ARG: return "RW_E_ARG";
+    case RW_E_TYPE: return "RW_E_TYPE";
+    case RW_E_UNSORTED: return "RW_E_UNSORTED";
+    case RW_E_OVERFLOW: return "RW_E_OVERFLOW";
+    case RW_E_UNSUPPORTED: return "RW_E_UNSUPPORTED";
+    case RW_E_CAPACITY: return "RW_E_CAPACITY";
+    case RW_E_OOM: return "RW_E_OOM";
+    case RW_E_CUDA: return "RW_E_CUDA";
+    case RW_E_DOMAIN: return "RW_E_DOMAIN";
+    case RW_E_STATE: return "RW_E_STATE";
+    }
+    return "RW_E_?";
+}
+
+const char *rw_last_error(void) { return g_err.c_str(); }
+
+rw_status rw_plan_create(rw_plan **out, const rw_plan_opts *opts)
+{
+    RW_TRY
+    if (!out)
+        raise(RW_E_ARG, "null out");
+    rw_plan_opts o{};
+    o.fuse = 1;
+    if (opts)
+        o = *opts;
+    int ndev = 0;
+    cuda_check(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
+    if (o.device < 0 || o.device >= ndev)
+        raise(RW_E_ARG, "no such CUDA device");
+    cuda_check(cudaSetDevice(o.device), "cudaSetDevice");
+    int major = 0;
+    cuda_check(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, o.device), "attr");
+    if (major != 10)
+        raise(RW_E_CUDA, "librw is built for sm_100a (B200) only");
+    rw_plan *p = new rw_plan();
+    p->o = o;
+    p->stream = (cudaStream_t)o.cuda_stream;
+    cuda_check(cudaDeviceGetAttribute(&p->sms, cudaDevAttrMultiProcessorCount, o.device), "attr");
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, o.device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    try {
+        p->ctrs = (uint32_t *)dev_alloc(p, 64);
+        cuda_check(cudaMemsetAsync(p->ctrs, 0, 64, p->stream), "memset");
+        p->jtot = (int64_t *)dev_alloc(p, 64);
+        p->err = (int32_t *)dev_alloc(p, 64);
+        cuda_check(cudaMemsetAsync(p->err, 0, 64, p->stream), "memset");
+        cuda_check(cudaMallocHost(&p->jtot_host, 64), "cudaMallocHost");
+        ensure_status(p, 4096);
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+    } catch (...) {
+        delete p;
+        throw;
+    }
+    *out = p;
+    return RW_OK;
+    RW_CATCH
+}
+
+void rw_plan_destroy(rw_plan *p)
+{
+    if (!p)
+        return;
+    cudaSetDevice(p->o.device);
+    cudaStreamSynchronize(p->stream);
+    for (auto &kv : p->agg_acc)
+        cudaFree(kv.second);
+    if (p->status) cudaFree(p->status);
+    if (p->ctrs) cudaFree(p->ctrs);
+    if (p->cnt) cudaFree(p->cnt);
+    if (p->jtot) cudaFree(p->jtot);
+    if (p->err) cudaFree(p->err);
+    if (p->jtot_host) cudaFreeHost(p->jtot_host);
+    delete p;
+}
+
+static int add_node(rw_plan *p, Node &&n, int32_t *node)
+{
+    p->nodes.push_back(std::move(n));
+    int id = (int)p->nodes.size() - 1;
+    if (node)
+        *node = id;
+    return id;
+}
+
+static void check_type(int t)
+{
+    if (t < RW_I32 || t > RW_U8)
+        raise(RW_E_TYPE, "unknown attribute type " + std::to_string(t));
+}
+
+rw_status rw_plan_add_input(rw_plan *p, int32_t ncols, const int32_t *types, int32_t nkey_sorted,
+                            const int64_t *lo, const int64_t *hi, int32_t *node)
+{
+    RW_TRY
+    if (!p || ncols < 1 || ncols > kMaxOut || !types || nkey_sorted < 0 || nkey_sorted > ncols)
+        raise(RW_E_ARG, "bad input declaration");
+    Node n;
+    n.kind = N_INPUT;
+    for (int c = 0; c < ncols; c++) {
+        check_type(types[c]);
+        n.types.push_back(types[c]);
+        Interval r = type_range(types[c]);
+        if (lo) r.lo = std::max<i128>(r.lo, lo[c]);
+        if (hi) r.hi = std::min<i128>(r.hi, types[c] == T_U64 ? (i128)(uint64_t)hi[c] : (i128)hi[c]);
+        if (r.lo > r.hi)
+            raise(RW_E_ARG, "empty bound interval for column " + std::to_string(c));
+        n.bounds.push_back(r);
+    }
+    n.nkey_sorted = nkey_sorted;
+    n.input_index = (int)p->inputs.size();
+    int id = add_node(p, std::move(n), node);
+    p->inputs.push_back(id);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_add_select(rw_plan *p, int32_t in, const rw_pred *pr, int32_t np, int32_t *node)
+{
+    RW_TRY
+    if (!p || np < 0 || (np > 0 && !pr))
+        raise(RW_E_ARG, "bad select");
+    const Node &src = node_at(p, in);
+    Node n;
+    n.kind = N_SELECT;
+    n.in = in;
+    n.types = src.types;
+    n.bounds = src.bounds;
+    n.nkey_sorted = src.nkey_sorted;
+    const int nc = (int)src.types.size();
+    for (int i = 0; i < np; i++) {
+        const rw_pred &a = pr[i];
+        if (a.col < 0 || a.col >= nc || a.op < RW_LT || a.op > RW_NE)
+            raise(RW_E_ARG, "bad select atom " + std::to_string(i));
+        if (a.rhs_is_col) {
+            if (a.rhs_col < 0 || a.rhs_col >= nc)
+                raise(RW_E_ARG, "bad select atom rhs column");
+            if (src.types[a.rhs_col] != src.types[a.col])
+                raise(RW_E_TYPE, "column-vs-column atom needs identical types");
+        }
+        n.preds.push_back(a);
+    }
+    add_node(p, std::move(n), node);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_add_project(rw_plan *p, int32_t in, const rw_expr *e, int32_t ne, const int32_t *roots,
+                              int32_t nout, int32_t *node)
+{
+    RW_TRY
+    if (!p || ne < 1 || !e || !roots || nout < 1 || nout > kMaxOut)
+        raise(RW_E_ARG, "bad project");
+    const Node &src = node_at(p, in);
+    const int nc = (int)src.types.size();
+    for (int i = 0; i < ne; i++) {
+        const rw_expr &x = e[i];
+        if (x.op < RW_COL || x.op > RW_DIVC)
+            raise(RW_E_ARG, "bad expression op");
+        check_type(x.type);
+        if (x.type == RW_U8 && x.op != RW_COL)
+            raise(RW_E_TYPE, "u8 results only for column references");
+        if (x.op == RW_COL && (x.a < 0 || x.a >= nc))
+            raise(RW_E_ARG, "expression column out of range");
+        if ((x.op == RW_ADD || x.op == RW_SUB || x.op == RW_MUL) &&
+            (x.a < 0 || x.a >= i || x.b < 0 || x.b >= i))
+            raise(RW_E_ARG, "expression operands must be earlier nodes");
+        if (x.op == RW_DIVC) {
+            if (x.a < 0 || x.a >= i)
+                raise(RW_E_ARG, "expression operands must be earlier nodes");
+            if (wrap_to(x.type, x.k) == 0)
+                raise(RW_E_ARG, "division by zero constant");
+        }
+    }
+    Node n;
+    n.kind = N_PROJECT;
+    n.in = in;
+    n.exprs.assign(e, e + ne);
+    std::vector<Interval> memo(ne);
+    std::vector<char> done(ne, 0);
+    for (int j = 0; j < nout; j++) {
+        if (roots[j] < 0 || roots[j] >= ne)
+            raise(RW_E_ARG, "bad root");
+        n.roots.push_back(roots[j]);
+        n.types.push_back(e[roots[j]].type);
+        n.bounds.push_back(expr_interval(src, n.exprs, roots[j], memo, done, p->o.strict_overflow != 0));
+    }
+    // key-preserving prefix: leading outputs that are plain references to the
+    // input's leading sorted columns, in order, with unchanged type
+    int k = 0;
+    while (k < nout && k < src.nkey_sorted) {
+        const rw_expr &x = e[roots[k]];
+        if (x.op != RW_COL || x.a != k || x.type != src.types[k]) break;
+        k++;
+    }
+    n.nkey_sorted = k;
+    add_node(p, std::move(n), node);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_add_join(rw_plan *p, int32_t left, int32_t right, int32_t nkey, int32_t *node)
+{
+    RW_TRY
+    if (!p)
+        raise(RW_E_ARG, "null plan");
+    const Node &L = node_at(p, left);
+    const Node &R = node_at(p, right);
+    if (nkey < 1 || nkey > (int)L.types.size() || nkey > (int)R.types.size())
+        raise(RW_E_ARG, "bad nkey");
+    if (nkey != 1)
+        raise(RW_E_UNSUPPORTED, "this build joins on a single key column");
+    for (int c = 0; c < nkey; c++)
+        if (L.types[c] != R.types[c])
+            raise(RW_E_TYPE, "join key types differ");
+    if (L.nkey_sorted < nkey || R.nkey_sorted < nkey)
+        raise(RW_E_UNSORTED, "join inputs must be sorted on the key (kernel dependence: sort first)");
+    if (L.kind == N_AGG || R.kind == N_AGG)
+        ;  // AGG output is sorted by group code: legal, materialised (kernel dependence)
+    Node n;
+    n.kind = N_JOIN;
+    n.left = left;
+    n.right = right;
+    n.nkey = nkey;
+    for (size_t c = 0; c < L.types.size(); c++) {
+        n.types.push_back(L.types[c]);
+        Interval b = L.bounds[c];
+        if (c < (size_t)nkey) {
+            b.lo = std::max(b.lo, R.bounds[c].lo);
+            b.hi = std::min(b.hi, R.bounds[c].hi);
+            if (b.lo > b.hi) b = L.bounds[c];
+        }
+        n.bounds.push_back(b);
+    }
+    for (size_t c = nkey; c < R.types.size(); c++) {
+        n.types.push_back(R.types[c]);
+        n.bounds.push_back(R.bounds[c]);
+    }
+    if ((int)n.types.size() > kMaxOut)
+        raise(RW_E_UNSUPPORTED, "join output wider than 32 columns");
+    n.nkey_sorted = nkey;
+    add_node(p, std::move(n), node);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_add_agg(rw_plan *p, int32_t in, const int32_t *gcols, const int32_t *gdomain, int32_t ng,
+                          const rw_agg *a, int32_t na, int32_t *node)
+{
+    RW_TRY
+    if (!p || ng < 0 || ng > kMaxGroupCols || na < 0 || na > kMaxAggs || (ng && (!gcols || !gdomain)) ||
+        (na && !a))
+        raise(RW_E_ARG, "bad agg");
+    const Node &src = node_at(p, in);
+    const int nc = (int)src.types.size();
+    Node n;
+    n.kind = N_AGG;
+    n.in = in;
+    int64_t D = 1;
+    int nsum = 0, ncols = ng;
+    for (int c = 0; c < ng; c++) {
+        if (gcols[c] < 0 || gcols[c] >= nc || gdomain[c] < 1)
+            raise(RW_E_ARG, "bad group column");
+        D *= gdomain[c];
+        if (D > kMaxAggSlots)
+            raise(RW_E_UNSUPPORTED, "group domain product above 4096");
+        n.gcols.push_back(gcols[c]);
+        n.gdomain.push_back(gdomain[c]);
+        n.types.push_back(src.types[gcols[c]]);
+        n.bounds.push_back({0, gdomain[c] - 1});
+    }
+    for (int q = 0; q < na; q++) {
+        if (a[q].op == RW_SUM) {
+            if (a[q].col < 0 || a[q].col >= nc)
+                raise(RW_E_ARG, "bad aggregate column");
+            nsum++;
+            n.types.push_back(RW_U64);
+            n.bounds.push_back(type_range(T_U64));
+            n.types.push_back(RW_I64);
+            n.bounds.push_back(type_range(T_I64));
+            ncols += 2;
+        } else if (a[q].op == RW_COUNT) {
+            n.types.push_back(RW_I64);
+            n.bounds.push_back({0, INT64_MAX});
+            ncols += 1;
+        } else {
+            raise(RW_E_ARG, "bad aggregate op");
+        }
+        n.aggs.push_back(a[q]);
+    }
+    if (ncols > kMaxOut || D * (nsum + 1) > kMaxAggSlots)
+        raise(RW_E_UNSUPPORTED, "aggregate too wide");
+    n.D = (int)D;
+    n.nkey_sorted = ng;
+    add_node(p, std::move(n), node);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_node_schema(const rw_plan *p, int32_t node, int32_t *ncols, int32_t *types)
+{
+    RW_TRY
+    if (!p || !ncols)
+        raise(RW_E_ARG, "null argument");
+    const Node &n = node_at(p, node);
+    *ncols = (int32_t)n.types.size();
+    if (types)
+        for (size_t c = 0; c < n.types.size(); c++)
+            types[c] = n.types[c];
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_execute(rw_plan *p, const rw_relation_in *in, int32_t nin, int32_t out_node,
+                          rw_relation_out *out)
+{
+    RW_TRY
+    if (!p)
+        raise(RW_E_ARG, "null plan");
+    execute(p, in, nin, out_node, out);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_execute_host(rw_plan *p, const rw_relation_in *in, int32_t nin, int32_t out_node,
+                               rw_relation_out *out)
+{
+    RW_TRY
+    if (!p || !out)
+        raise(RW_E_ARG, "null argument");
+    check_inputs(p, in, nin);
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    std::vector<void *> dev;
+    std::vector<std::vector<const void *>> dcols(nin);
+    std::vector<rw_relation_in> din(nin);
+    auto cleanup = [&]() {
+        for (void *d : dev)
+            cudaFreeAsync(d, p->stream);
+    };
+    try {
+        for (int i = 0; i < nin; i++) {
+            const Node &n = p->nodes[p->inputs[i]];
+            for (size_t c = 0; c < n.types.size(); c++) {
+                size_t bytes = (size_t)in[i].n * type_width(n.types[c]);
+                void *d = dev_alloc(p, bytes);
+                dev.push_back(d);
+                if (bytes)
+                    cuda_check(cudaMemcpyAsync(d, in[i].cols[c], bytes, cudaMemcpyHostToDevice, p->stream), "H2D");
+                dcols[i].push_back(d);
+            }
+            din[i].n = in[i].n;
+            din[i].cols = dcols[i].data();
+        }
+        const Node &on = node_at(p, out_node);
+        std::vector<void *> ocols;
+        for (int t : on.types) {
+            void *d = dev_alloc(p, (size_t)std::max<int64_t>(out->capacity, 1) * type_width(t));
+            dev.push_back(d);
+            ocols.push_back(d);
+        }
+        rw_relation_out dout{ocols.data(), out->capacity, nullptr, -1};
+        rw_status st = RW_OK;
+        try {
+            execute(p, din.data(), nin, out_node, &dout);
+        } catch (const RwError &e) {
+            if (e.s != RW_E_CAPACITY)
+                throw;
+            st = e.s;
+            g_err = e.msg;
+        }
+        const int64_t rows = std::min(dout.n, out->capacity);
+        for (size_t c = 0; c < on.types.size(); c++)
+            if (rows > 0)
+                cuda_check(cudaMemcpyAsync(out->cols[c], ocols[c], (size_t)rows * type_width(on.types[c]),
+                                           cudaMemcpyDeviceToHost, p->stream),
+                           "D2H");
+        cleanup();
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+        out->n = dout.n;
+        return st;
+    } catch (...) {
+        cleanup();
+        throw;
+    }
+    RW_CATCH
+}
+
+rw_status rw_plan_explain(rw_plan *p, int32_t out_node, char *buf, size_t cap)
+{
+    RW_TRY
+    if (!p || !buf || cap == 0)
+        raise(RW_E_ARG, "bad buffer");
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    std::string s = explain(p, out_node);
+    size_t n = std::min(cap - 1, s.size());
+    std::memcpy(buf, s.data(), n);
+    buf[n] = 0;
+    return s.size() < cap ? RW_OK : RW_E_CAPACITY;
+    RW_CATCH
+}
+
+int64_t rw_plan_last_launches(const rw_plan *p) { return p ? p->launches : -1; }
+
+rw_status rw_split_by_splitters(const void *keys_dev, int64_t n, int32_t key_type, const void *splitters_dev,
+                                int32_t nsplit, int64_t *bounds_dev, void *cuda_stream)
+{
+    g_err = "rw_split_by_splitters: not built yet";
+    (void)keys_dev; (void)n; (void)key_type; (void)splitters_dev; (void)nsplit; (void)bounds_dev; (void)cuda_stream;
+    return RW_E_UNSUPPORTED;
+}
+
+rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t ncols, const int64_t *run_off,
+                        int32_t nrun, void *const *out_cols, void *cuda_stream)
+{
+    g_err = "rw_merge_runs: not built yet";
+    (void)cols; (void)types; (void)ncols; (void)run_off; (void)nrun; (void)out_cols; (void)cuda_stream;
+    return RW_E_UNSUPPORTED;
+}
+
+}  // extern "C"

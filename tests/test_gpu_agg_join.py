@@ -1,0 +1,122 @@
+"""GPU parity: group-by aggregate (Q1, k_scan_chain<agg> + k_agg_finalize) and the
+merge-path JOIN (k_join_runs + k_join_expand) fused with downstream operators."""
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from tests.planspec import assert_same, build_gpu_plan, run_gpu, run_oracle
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+
+
+@pytest.mark.parametrize("n", [0, 1, 2047, 2049, 100_003, 1_000_000])
+@pytest.mark.parametrize("fuse", [True, False])
+def test_q1_aggregate(n, fuse):
+    spec = workloads.c4_spec()
+    ins = workloads.c4_inputs(n, device=DEV, cfg=0x91)
+    got, plan = run_gpu(spec, ins, capacity=6, fuse=fuse)
+    assert_same(got, run_oracle(spec, ins))
+
+
+def test_q1_without_bounds_flushes_every_row():
+    spec = workloads.c4_spec()
+    spec["inputs"]["lineitem"] = {"types": workloads.Q1_TYPES}          # no declared bounds
+    ins = workloads.c4_inputs(60_000, device=DEV, cfg=0x92)
+    got, _ = run_gpu(spec, ins, capacity=6)
+    assert_same(got, run_oracle(spec, ins))
+
+
+def test_sum_beyond_int64_is_exact():
+    import torch
+    n = 50_000
+    v = torch.full((n,), 2**62 + 7, dtype=torch.int64, device=DEV)
+    g = (torch.arange(n, device=DEV) % 3).to(torch.uint8)
+    u = torch.full((n,), -1, dtype=torch.int64, device=DEV)              # u64 max
+    spec = {"inputs": {"R": {"types": ["u8", "i64", "u64"]}},
+            "nodes": [{"id": "a", "op": "agg", "in": "R", "gcols": [0], "gdomain": [3],
+                       "aggs": [("sum", 1), ("count",), ("sum", 2)]}], "out": "a"}
+    ins = {"R": [g, v, u]}
+    got, _ = run_gpu(spec, ins, capacity=3)
+    ref = run_oracle(spec, ins)
+    assert_same(got, ref)
+    assert oracle.sum128(got.cols[1], got.cols[2])[0] == 16667 * (2**62 + 7)
+
+
+def test_agg_domain_error():
+    import torch
+    from paper_conf_micro_wudcy12_b200 import rw
+    g = torch.tensor([0, 1, 7], dtype=torch.uint8, device=DEV)
+    spec = {"inputs": {"R": {"types": ["u8"]}},
+            "nodes": [{"id": "a", "op": "agg", "in": "R", "gcols": [0], "gdomain": [3], "aggs": [("count",)]}],
+            "out": "a"}
+    with pytest.raises(rw.RwError) as e:
+        run_gpu(spec, {"R": [g]}, capacity=3)
+    assert e.value.name == "RW_E_DOMAIN"
+
+
+@pytest.mark.parametrize("n", [0, 1, 100, 5000, 200_000])
+@pytest.mark.parametrize("fuse", [True, False])
+def test_c3_zipf_join_select_project(n, fuse):
+    spec = workloads.c3_spec()
+    ins = workloads.c3_inputs(n, device=DEV, cfg=0x93)
+    ref = run_oracle(spec, ins)
+    got, _ = run_gpu(spec, ins, capacity=max(ref.n, 1), fuse=fuse)
+    assert_same(got, ref)
+
+
+def test_join_hot_key_spans_many_tiles():
+    import torch
+    # one key with 3000 x 2000 matches (6M candidates, > 2600 expansion tiles) plus noise
+    lk = torch.cat([torch.arange(0, 500, device=DEV), torch.full((3000,), 777, device=DEV),
+                    torch.arange(1000, 1500, device=DEV)]).to(torch.int32)
+    rk = torch.cat([torch.arange(0, 800, 2, device=DEV), torch.full((2000,), 777, device=DEV),
+                    torch.arange(1000, 3000, 3, device=DEV)]).to(torch.int32)
+    lv = torch.arange(lk.numel(), device=DEV, dtype=torch.int32) * 7
+    rv = torch.arange(rk.numel(), device=DEV, dtype=torch.int32) * 5 + 3
+    lk, _ = torch.sort(lk)
+    rk, _ = torch.sort(rk)
+    spec = workloads.c3_spec()
+    ins = {"L": [lk, lv], "R": [rk, rv]}
+    ref = run_oracle(spec, ins)
+    got, _ = run_gpu(spec, ins, capacity=ref.n)
+    assert_same(got, ref)
+
+
+def test_join_signed_and_64bit_keys():
+    import torch
+    rng = np.random.default_rng(4)
+    for kt, st in (("i32", np.int32), ("i64", np.int64), ("u64", np.int64)):
+        a = np.sort(rng.integers(-50, 50, 3000).astype(st)) if kt != "u64" else \
+            np.sort(rng.integers(0, 100, 3000).astype(np.uint64)).view(np.int64)
+        b = np.sort(rng.integers(-50, 50, 2500).astype(st)) if kt != "u64" else \
+            np.sort(rng.integers(0, 100, 2500).astype(np.uint64)).view(np.int64)
+        spec = {"inputs": {"L": {"types": [kt, "u8"], "nkey_sorted": 1},
+                           "R": {"types": [kt, "i64", "u32"], "nkey_sorted": 1}},
+                "nodes": [{"id": "j", "op": "join", "left": "L", "right": "R", "nkey": 1}], "out": "j"}
+        ins = {"L": [torch.from_numpy(a).to(DEV), torch.from_numpy((np.arange(3000) % 251).astype(np.uint8)).to(DEV)],
+               "R": [torch.from_numpy(b).to(DEV), torch.from_numpy(np.arange(2500, dtype=np.int64) * -3).to(DEV),
+                     torch.from_numpy(np.arange(2500, dtype=np.int32)).to(DEV)]}
+        ref = run_oracle(spec, ins)
+        got, _ = run_gpu(spec, ins, capacity=ref.n)
+        assert_same(got, ref)
+
+
+@pytest.mark.parametrize("n", [0, 1000, 30_000])
+def test_c5_three_way_join(n):
+    spec = workloads.c5_spec()
+    ins = workloads.c5_inputs(n, device=DEV, cfg=0x94)
+    ref = run_oracle(spec, ins)
+    got, _ = run_gpu(spec, ins, capacity=max(ref.n, 1))
+    assert_same(got, ref)
+
+
+def test_join_then_aggregate():
+    spec = workloads.c3_spec()
+    spec["nodes"].append({"id": "g", "op": "agg", "in": "p", "gcols": [], "gdomain": [],
+                          "aggs": [("count",), ("sum", 1)]})
+    spec["out"] = "g"
+    ins = workloads.c3_inputs(20_000, device=DEV, cfg=0x95)
+    got, _ = run_gpu(spec, ins, capacity=1)
+    assert_same(got, run_oracle(spec, ins))
