@@ -49,6 +49,10 @@ def parse():
     ap.add_argument("--no-unfused", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-rows", type=int, default=0)
+    ap.add_argument("--stages", type=int, default=0, help="TMA stages per CTA (0 = auto)")
+    ap.add_argument("--ctas", type=int, default=0, help="CTAs per SM cap (0 = auto)")
+    ap.add_argument("--defer", type=int, default=0, help="scan store delay in tiles (0 = auto)")
+    ap.add_argument("--dbg", type=int, default=0, help="diagnostic ablations (not a bench value)")
     return ap.parse_args()
 
 
@@ -221,7 +225,8 @@ def main():
     stream = torch.cuda.current_stream()
 
     def make(fuse):
-        plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse)
+        plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse, stages=args.stages,
+                                   ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg)
         out_types = plan.node_schema(ids[spec["out"]])
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
         if cfg == "c3":

@@ -31,7 +31,8 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v)
     return v;
 }
 
-__device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_t agg, uint32_t epoch)
+__device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_t agg, uint32_t epoch,
+                                         bool aggregate_published = false)
 {
     const int lane = threadIdx.x & 31;
     const uint64_t tag = (uint64_t)epoch << 48;
@@ -40,30 +41,63 @@ __device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_
             st_relaxed_u64(&status[0], tag | (2ull << 46) | agg);
         return 0;
     }
-    if (lane == 0)
+    if (lane == 0 && !aggregate_published)
         st_relaxed_u64(&status[tile], tag | (1ull << 46) | agg);
+    // Each round inspects 128 predecessors (4 status words per lane): with ~10^2
+    // tiles completing per microsecond chip-wide, a 32-wide window would let the
+    // band of aggregate-only tiles outgrow one round and the walk would never settle.
+    constexpr int Q = 4;
     uint64_t excl = 0;
     int64_t j = tile - 1;
     while (true) {
-        int64_t idx = j - lane;
-        uint32_t flag = 2;
-        uint64_t val = 0;
-        if (idx >= 0) {
-            uint64_t w;
-            do {
-                w = ld_relaxed_u64(&status[idx]);
-                flag = ((uint32_t)(w >> 48) == epoch) ? (uint32_t)(w >> 46) & 3u : 0u;
-            } while (flag == 0);
-            val = w & kValMask;
+        uint64_t w[Q];
+        uint32_t pending = 0;
+#pragma unroll
+        for (int q = 0; q < Q; q++) {
+            const int64_t idx = j - lane * Q - q;
+            w[q] = idx >= 0 ? ld_relaxed_u64(&status[idx]) : ((uint64_t)epoch << 48) | (2ull << 46);
+            if ((uint32_t)(w[q] >> 48) != epoch || ((w[q] >> 46) & 3u) == 0)
+                pending |= 1u << q;
         }
-        uint32_t pmask = __ballot_sync(0xffffffffu, flag == 2);
+        uint32_t backoff = 32;
+        while (pending) {
+            // back off: hundreds of look-back warps polling the same few status
+            // lines would otherwise starve the stores that publish them
+            __nanosleep(backoff);
+            backoff = backoff < 1024 ? backoff * 2 : 1024;
+#pragma unroll
+            for (int q = 0; q < Q; q++) {
+                if ((pending >> q) & 1u) {
+                    w[q] = ld_relaxed_u64(&status[j - lane * Q - q]);
+                    if ((uint32_t)(w[q] >> 48) == epoch && ((w[q] >> 46) & 3u) != 0)
+                        pending &= ~(1u << q);
+                }
+            }
+        }
+        int firstq = Q;                             // nearest inclusive prefix within this lane
+#pragma unroll
+        for (int q = Q - 1; q >= 0; q--)
+            if (((w[q] >> 46) & 3u) == 2u)
+                firstq = q;
+        const uint32_t pmask = __ballot_sync(0xffffffffu, firstq < Q);
+        uint64_t s = 0;
         if (pmask) {
-            int first = __ffs(pmask) - 1;          // nearest predecessor holding an inclusive prefix
-            excl += warp_sum_u64(lane <= first ? val : 0);
+            const int first = __ffs(pmask) - 1;     // nearest lane holding an inclusive prefix
+            if (lane < first) {
+#pragma unroll
+                for (int q = 0; q < Q; q++) s += w[q] & kValMask;
+            } else if (lane == first) {
+#pragma unroll
+                for (int q = 0; q < Q; q++)
+                    if (q <= firstq) s += w[q] & kValMask;
+            }
+            excl += warp_sum_u64(s);
             break;
         }
-        excl += warp_sum_u64(val);
-        j -= 32;
+#pragma unroll
+        for (int q = 0; q < Q; q++) s += w[q] & kValMask;
+        excl += warp_sum_u64(s);
+        j -= 32 * Q;
     }
     if (lane == 0)
         st_relaxed_u64(&status[tile], tag | (2ull << 46) | (excl + agg));
@@ -71,8 +105,14 @@ __device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_
 }
 
 // ---------------------------------------------------------------------------
-// Slot access
+// Slot access.  Locations are resolved on the host (kLocScratch | byte offset),
+// so the interpreter never walks a slot table on the device.
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ const char *loc_ptr(uint32_t loc, const char *stage, const char *scratch)
+{
+    return ((loc & kLocScratch) ? scratch : stage) + (loc & ~kLocScratch);
+}
+
 __device__ __forceinline__ const char *slot_ptr(const ChainProg &P, int s, const char *stage, const char *scratch)
 {
     return (P.slot[s].is_input ? stage : scratch) + P.slot[s].off;
@@ -89,6 +129,12 @@ __device__ __forceinline__ uint64_t ld_ext(const char *base, int type, int row)
     }
 }
 
+template <typename T>
+__device__ __forceinline__ T ld_as(const char *base, int row)
+{
+    return ((const T *)base)[row];
+}
+
 template <typename T, int CMP>
 __device__ __forceinline__ bool cmpv(T x, T y)
 {
@@ -101,34 +147,47 @@ __device__ __forceinline__ bool cmpv(T x, T y)
 }
 
 // SELECT atom over the tile: clears bits of rows failing `a CMP b` (reading A4).
-template <int ITEMS, typename T, int CMP>
-__device__ __forceinline__ uint32_t pred_loop(const char *a, const char *b, T k, bool bslot, uint32_t mask)
+template <int ITEMS, typename T, int CMP, bool BSLOT>
+__device__ __forceinline__ uint32_t pred_loop(const char *a, const char *b, T k, uint32_t mask)
 {
     const int tid = threadIdx.x;
     const T *pa = (const T *)a;
     const T *pb = (const T *)b;
+    uint32_t keep = 0;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) {
-        T x = pa[i * kThreads + tid];
-        T y = bslot ? pb[i * kThreads + tid] : k;
-        if (!cmpv<T, CMP>(x, y))
-            mask &= ~(1u << i);
+        const T x = pa[i * kThreads + tid];
+        const T y = BSLOT ? pb[i * kThreads + tid] : k;
+        keep |= (uint32_t)cmpv<T, CMP>(x, y) << i;
     }
-    return mask;
+    return mask & keep;
 }
 
-template <int ITEMS, typename T>
-__device__ __forceinline__ uint32_t pred_t(int cmp, const char *a, const char *b, int64_t k, bool bslot, uint32_t mask)
+#define RW_PRED_CASES(TT, TCODE)                                                                        \
+    case TCODE * 8 + C_LT: return pred_loop<ITEMS, TT, C_LT, false>(a, b, (TT)o.k, mask);           \
+    case TCODE * 8 + C_LE: return pred_loop<ITEMS, TT, C_LE, false>(a, b, (TT)o.k, mask);           \
+    case TCODE * 8 + C_GT: return pred_loop<ITEMS, TT, C_GT, false>(a, b, (TT)o.k, mask);           \
+    case TCODE * 8 + C_GE: return pred_loop<ITEMS, TT, C_GE, false>(a, b, (TT)o.k, mask);           \
+    case TCODE * 8 + C_EQ: return pred_loop<ITEMS, TT, C_EQ, false>(a, b, (TT)o.k, mask);           \
+    case TCODE * 8 + C_NE: return pred_loop<ITEMS, TT, C_NE, false>(a, b, (TT)o.k, mask);           \
+    case 64 + TCODE * 8 + C_LT: return pred_loop<ITEMS, TT, C_LT, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_LE: return pred_loop<ITEMS, TT, C_LE, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_GT: return pred_loop<ITEMS, TT, C_GT, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_GE: return pred_loop<ITEMS, TT, C_GE, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_EQ: return pred_loop<ITEMS, TT, C_EQ, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_NE: return pred_loop<ITEMS, TT, C_NE, true>(a, b, (TT)0, mask);
+
+template <int ITEMS>
+__device__ __noinline__ uint32_t run_pred(const DevOp &o, const char *a, const char *b, uint32_t mask)
 {
-    T kk = (T)k;
-    switch (cmp) {
-    case C_LT: return pred_loop<ITEMS, T, C_LT>(a, b, kk, bslot, mask);
-    case C_LE: return pred_loop<ITEMS, T, C_LE>(a, b, kk, bslot, mask);
-    case C_GT: return pred_loop<ITEMS, T, C_GT>(a, b, kk, bslot, mask);
-    case C_GE: return pred_loop<ITEMS, T, C_GE>(a, b, kk, bslot, mask);
-    case C_EQ: return pred_loop<ITEMS, T, C_EQ>(a, b, kk, bslot, mask);
-    default: return pred_loop<ITEMS, T, C_NE>(a, b, kk, bslot, mask);
+    switch (o.code) {
+        RW_PRED_CASES(int32_t, T_I32)
+        RW_PRED_CASES(uint32_t, T_U32)
+        RW_PRED_CASES(int64_t, T_I64)
+        RW_PRED_CASES(uint64_t, T_U64)
+        RW_PRED_CASES(uint8_t, T_U8)
     }
+    return mask;
 }
 
 // Arithmetic in type T with wrap-around (reading A8): done in the unsigned twin.
@@ -149,32 +208,57 @@ __device__ __forceinline__ T ev(T a, T b)
     return a;                                 // E_COPY (type conversion)
 }
 
-template <int ITEMS, typename T, int OP>
-__device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, const char *b, int tb, bool bslot, T k)
+// dst[r] = a[r] OP (b[r] | k) over the tile.  Operands stored in another type are
+// converted into T (mod 2^w); same-type operands are loaded directly.
+template <int ITEMS, typename T, int OP, bool BSLOT>
+__device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, const char *b, int tb, T k)
 {
     const int tid = threadIdx.x;
+    constexpr int TT = sizeof(T) == 8 ? (std::is_signed<T>::value ? T_I64 : T_U64)
+                                      : (std::is_signed<T>::value ? T_I32 : T_U32);
+    const bool sa = (ta == TT) || (sizeof(T) == 4 && (ta == T_I32 || ta == T_U32)) ||
+                    (sizeof(T) == 8 && (ta == T_I64 || ta == T_U64));
+    const bool sb = (tb == TT) || (sizeof(T) == 4 && (tb == T_I32 || tb == T_U32)) ||
+                    (sizeof(T) == 8 && (tb == T_I64 || tb == T_U64));
+    if (sa && (!BSLOT || sb)) {
 #pragma unroll
-    for (int i = 0; i < ITEMS; i++) {
-        const int r = i * kThreads + tid;
-        T x = (OP == E_CONST) ? (T)0 : (T)ld_ext(a, ta, r);
-        T y = bslot ? (T)ld_ext(b, tb, r) : k;
-        ((T *)dst)[r] = ev<T, OP>(x, y);
+        for (int i = 0; i < ITEMS; i++) {
+            const int r = i * kThreads + tid;
+            const T x = (OP == E_CONST) ? (T)0 : ld_as<T>(a, r);
+            const T y = BSLOT ? ld_as<T>(b, r) : k;
+            ((T *)dst)[r] = ev<T, OP>(x, y);
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < ITEMS; i++) {
+            const int r = i * kThreads + tid;
+            const T x = (OP == E_CONST) ? (T)0 : (T)ld_ext(a, ta, r);
+            const T y = BSLOT ? (T)ld_ext(b, tb, r) : k;
+            ((T *)dst)[r] = ev<T, OP>(x, y);
+        }
     }
 }
 
-template <int ITEMS, typename T>
-__device__ __forceinline__ void expr_t(const DevOp &o, char *dst, const char *a, int ta, const char *b, int tb)
+#define RW_EXPR_CASES(TT, TCODE)                                                                                  \
+    case TCODE * 8 + E_COPY: expr_loop<ITEMS, TT, E_COPY, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
+    case TCODE * 8 + E_CONST: expr_loop<ITEMS, TT, E_CONST, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;     \
+    case TCODE * 8 + E_ADD: expr_loop<ITEMS, TT, E_ADD, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
+    case TCODE * 8 + E_SUB: expr_loop<ITEMS, TT, E_SUB, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
+    case TCODE * 8 + E_MUL: expr_loop<ITEMS, TT, E_MUL, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
+    case TCODE * 8 + E_DIVC: expr_loop<ITEMS, TT, E_DIVC, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
+    case TCODE * 8 + E_RSUB: expr_loop<ITEMS, TT, E_RSUB, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
+    case 64 + TCODE * 8 + E_ADD: expr_loop<ITEMS, TT, E_ADD, true>(dst, a, o.ta, b, o.tb, (TT)0); return;       \
+    case 64 + TCODE * 8 + E_SUB: expr_loop<ITEMS, TT, E_SUB, true>(dst, a, o.ta, b, o.tb, (TT)0); return;       \
+    case 64 + TCODE * 8 + E_MUL: expr_loop<ITEMS, TT, E_MUL, true>(dst, a, o.ta, b, o.tb, (TT)0); return;
+
+template <int ITEMS>
+__device__ __noinline__ void run_expr(const DevOp &o, char *dst, const char *a, const char *b)
 {
-    const bool bs = o.b_is_slot;
-    const T k = (T)o.k;
-    switch (o.op) {
-    case E_COPY: expr_loop<ITEMS, T, E_COPY>(dst, a, ta, b, tb, false, k); break;
-    case E_CONST: expr_loop<ITEMS, T, E_CONST>(dst, a, ta, b, tb, false, k); break;
-    case E_ADD: expr_loop<ITEMS, T, E_ADD>(dst, a, ta, b, tb, bs, k); break;
-    case E_SUB: expr_loop<ITEMS, T, E_SUB>(dst, a, ta, b, tb, bs, k); break;
-    case E_MUL: expr_loop<ITEMS, T, E_MUL>(dst, a, ta, b, tb, bs, k); break;
-    case E_RSUB: expr_loop<ITEMS, T, E_RSUB>(dst, a, ta, b, tb, false, k); break;
-    default: expr_loop<ITEMS, T, E_DIVC>(dst, a, ta, b, tb, false, k); break;
+    switch (o.code) {
+        RW_EXPR_CASES(int32_t, T_I32)
+        RW_EXPR_CASES(uint32_t, T_U32)
+        RW_EXPR_CASES(int64_t, T_I64)
+        RW_EXPR_CASES(uint64_t, T_U64)
     }
 }
 
@@ -183,29 +267,15 @@ __device__ __forceinline__ void expr_t(const DevOp &o, char *dst, const char *a,
 template <int ITEMS>
 __device__ __forceinline__ uint32_t run_ops(const ChainProg &P, const char *stage, char *scratch, uint32_t mask)
 {
+#pragma unroll 1
     for (int i = 0; i < P.nops; i++) {
         const DevOp &o = P.ops[i];
-        const char *a = o.a >= 0 ? slot_ptr(P, o.a, stage, scratch) : nullptr;
-        const char *b = (o.b_is_slot && o.b >= 0) ? slot_ptr(P, o.b, stage, scratch) : nullptr;
-        if (o.kind == K_PRED) {
-            switch (o.type) {
-            case T_I32: mask = pred_t<ITEMS, int32_t>(o.op, a, b, o.k, o.b_is_slot, mask); break;
-            case T_U32: mask = pred_t<ITEMS, uint32_t>(o.op, a, b, o.k, o.b_is_slot, mask); break;
-            case T_I64: mask = pred_t<ITEMS, int64_t>(o.op, a, b, o.k, o.b_is_slot, mask); break;
-            case T_U64: mask = pred_t<ITEMS, uint64_t>(o.op, a, b, o.k, o.b_is_slot, mask); break;
-            default: mask = pred_t<ITEMS, uint8_t>(o.op, a, b, o.k, o.b_is_slot, mask); break;
-            }
-        } else {
-            char *dst = (char *)slot_ptr(P, o.dst, stage, scratch);
-            const int ta = o.a >= 0 ? P.slot[o.a].type : T_I64;
-            const int tb = (o.b_is_slot && o.b >= 0) ? P.slot[o.b].type : T_I64;
-            switch (o.type) {
-            case T_I32: expr_t<ITEMS, int32_t>(o, dst, a, ta, b, tb); break;
-            case T_U32: expr_t<ITEMS, uint32_t>(o, dst, a, ta, b, tb); break;
-            case T_I64: expr_t<ITEMS, int64_t>(o, dst, a, ta, b, tb); break;
-            default: expr_t<ITEMS, uint64_t>(o, dst, a, ta, b, tb); break;
-            }
-        }
+        const char *a = loc_ptr(o.a, stage, scratch);
+        const char *b = loc_ptr(o.b, stage, scratch);
+        if (o.kind == K_PRED)
+            mask = run_pred<ITEMS>(o, a, b, mask);
+        else
+            run_expr<ITEMS>(o, (char *)loc_ptr(o.dst, stage, scratch), a, b);
     }
     return mask;
 }
@@ -285,9 +355,8 @@ __device__ inline void emit_tile(const ChainProg &P, const char *stage, const ch
     __syncthreads();
     const int64_t base = es->tile_off;
     for (int j = 0; j < P.nout; j++) {
-        const int s = P.out_slot[j];
-        const char *src = slot_ptr(P, s, stage, scratch);
-        switch (type_width(P.slot[s].type)) {
+        const char *src = loc_ptr(P.out_loc[j], stage, scratch);
+        switch (P.out_w[j]) {
         case 1: store_col<ITEMS, uint8_t>((uint8_t *)P.out_ptr[j], (const uint8_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
         case 4: store_col<ITEMS, uint32_t>((uint32_t *)P.out_ptr[j], (const uint32_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
         default: store_col<ITEMS, uint64_t>((uint64_t *)P.out_ptr[j], (const uint64_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
@@ -344,9 +413,7 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
         int g = 0;
         bool ok = true;
         for (int c = 0; c < P.ngc; c++) {
-            const int s = P.gslot[c];
-            const int t = P.slot[s].type;
-            uint64_t code = ld_ext(slot_ptr(P, s, stage, scratch), t, r);
+            const uint64_t code = ld_ext(loc_ptr(P.g_loc[c], stage, scratch), P.g_type[c], r);
             // negative signed codes become huge unsigned values -> out of domain
             if (code >= (uint64_t)P.gdomain[c])
                 ok = false;
@@ -358,10 +425,8 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
         }
         unsigned long long *pg = part + (size_t)g * NA * kThreads + tid;
         pg[0] += 1ull;
-        for (int a = 0; a < P.nagg; a++) {
-            const int s = P.agg_slot[a];
-            pg[(a + 1) * kThreads] += ld_ext(slot_ptr(P, s, stage, scratch), P.slot[s].type, r);
-        }
+        for (int a = 0; a < P.nagg; a++)
+            pg[(a + 1) * kThreads] += ld_ext(loc_ptr(P.agg_loc[a], stage, scratch), P.agg_type[a], r);
         if (++since_flush >= P.flush_rows) {
             agg_flush(P, part, cta_acc);
             since_flush = 0;

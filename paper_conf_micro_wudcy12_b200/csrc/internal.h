@@ -45,16 +45,16 @@ struct SlotDesc {
     uint32_t off;       // byte offset of the slot column inside stage / scratch
 };
 
+// A smem location of a slot column, resolved on the host: bit 31 set = in the
+// scratch tile (computed columns), else in the input stage; low bits = byte offset.
+constexpr uint32_t kLocScratch = 0x80000000u;
+
 struct DevOp {
     uint8_t kind;       // K_PRED / K_EXPR
-    uint8_t op;         // Cmp or ExprOp
-    uint8_t type;       // compare type (PRED) or result type (EXPR)
-    uint8_t b_is_slot;  // PRED: rhs is a slot; EXPR: operand b is a slot (else constant k)
-    int16_t dst;        // EXPR destination slot
-    int16_t a;          // operand a slot
-    int16_t b;          // operand b slot
-    int16_t pad;
-    int64_t k;          // constant (rhs / operand b / divisor), already wrapped to `type`
+    uint8_t code;       // PRED: type*8 + cmp (+64: rhs is a slot); EXPR: type*8 + ExprOp (+64: b is a slot)
+    uint8_t ta, tb;     // EXPR operand slot types (converted into the result type)
+    uint32_t a, b, dst; // encoded locations (kLocScratch | offset)
+    int64_t k;          // constant (rhs / operand b / divisor), already wrapped to the op type
 };
 
 struct ChainProg {
@@ -66,16 +66,22 @@ struct ChainProg {
     const void *in_ptr[kMaxSlots];      // scan kernel: global column base of each input slot
     DevOp ops[kMaxOps];
     int16_t out_slot[kMaxOut];
+    uint32_t out_loc[kMaxOut];          // encoded smem location of each output column
+    uint8_t out_w[kMaxOut];             // byte width of each output column
     void *out_ptr[kMaxOut];
     int64_t out_capacity;
     // aggregate terminal (is_agg): group code g = sum code_c * stride_c
     int32_t is_agg;
     int32_t ngc;
     int16_t gslot[kMaxGroupCols];
+    uint32_t g_loc[kMaxGroupCols];
+    uint8_t g_type[kMaxGroupCols];
     int32_t gdomain[kMaxGroupCols];
     int32_t D;                          // product of domains
     int32_t nagg;                       // number of SUM accumulators (count is implicit, index 0)
     int16_t agg_slot[kMaxAggs];
+    uint32_t agg_loc[kMaxAggs];
+    uint8_t agg_type[kMaxAggs];
     uint8_t agg_unsigned[kMaxAggs];     // 1: u64 sum (unsigned partials)
     int64_t flush_rows;                 // rows a thread may add before its int64 partials can overflow
     uint32_t stage_bytes;               // bytes of one stage (all input slots, aligned)
@@ -87,6 +93,7 @@ struct TileLaunch {
     int64_t n;                 // rows (scan) or join outputs (expand), if n_ptr == nullptr
     const int64_t *n_ptr;      // device row count written by an earlier kernel (else nullptr)
     int32_t stages;
+    uint32_t out_bytes;        // scan kernel: bytes of the compacted-tile ring
     int32_t use_tma;           // input slots may be bulk-copied (16B-aligned bases)
     uint32_t epoch;            // look-back epoch tag (1..65535)
     uint64_t *status;          // look-back status words, >= ntiles
@@ -94,6 +101,9 @@ struct TileLaunch {
     int64_t *n_dev;            // output row count
     unsigned long long *agg_acc;   // global 128-bit accumulators: D * (nagg+1) * 2 u64
     int32_t *err;              // [0] domain errors
+    int32_t dbg;               // diagnostics: 1 = skip look-back (offset = tile * T, uncompacted),
+                               // 2 = stream tiles only, 4 = per-tile phase timestamps into dbg_ts
+    uint64_t *dbg_ts;          // 6 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start)
 };
 
 // Join expansion inputs (run records written by k_join_runs).

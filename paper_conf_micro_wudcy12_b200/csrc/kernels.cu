@@ -22,13 +22,6 @@ namespace rw {
 
 static __host__ __device__ inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-template <int ITEMS>
-struct CtlSmem {
-    uint64_t mbar[kMaxStages];
-    int64_t tile_id[kMaxStages];
-    EmitSmem<ITEMS> es;
-};
-
 __device__ inline void cta_exit_reset(uint32_t *ctrs)
 {
     __syncthreads();
@@ -43,118 +36,393 @@ __device__ inline void cta_exit_reset(uint32_t *ctrs)
 }
 
 // ===========================================================================
-// Fused scan chain.  Tiles of T = 256 * ITEMS rows are staged into smem by TMA
-// bulk copies (one cp.async.bulk per live column, completion on an mbarrier),
-// L.stages tiles in flight per CTA; thread 0 is the producer and refills a stage
-// as soon as every thread has finished with it.
+// Fused scan chain, warp-specialised (kThreads compute threads + 3 warps):
+//   producer warp  : claims tiles in order (global atomic) and stages each live
+//                    column of the tile into smem with one TMA bulk copy
+//                    (cp.async.bulk -> full[s]), S input stages deep;
+//   compute warps  : run the fused micro-op program on the tile, ballot-compact,
+//                    block-scan, publish the tile aggregate for the look-back at
+//                    once, then scatter the survivors (tile-local order) into a
+//                    byte-granular smem ring and release the input stage;
+//   4 writer warps : round-robin over compacted tiles: decoupled look-back for
+//                    the tile's global offset, coalesced copy of its columns to
+//                    HBM, release of its ring bytes (in tile order).
+// Phase timing (scripts/phases.py) showed the offset of a tile resolves ~4 us
+// after its aggregate (waiting for straggling predecessors); a compacted tile
+// only holds its actual bytes (~6 KB at 25 % survival instead of a 24 KB
+// worst-case slot) while it waits, so enough tiles stay in flight per SM.
 // ===========================================================================
+constexpr int kWriterWarps = 4;
+constexpr int kScanThreads = kThreads + 32 * (kWriterWarps + 1);
+constexpr int kRingSlots = 16;          // compacted tiles awaiting their offset, per CTA
+constexpr uint32_t kComputeBar = 1;     // named barrier of the compute warps
+
+struct InCtl {
+    uint64_t full, empty;
+    int64_t tile;
+};
+struct BlkCtl {
+    uint64_t aggr, oempty;
+    int64_t tile;
+    uint32_t total;
+    uint32_t roff;                       // byte offset of the block in the ring
+    uint32_t used;                       // ring bytes consumed (block + skipped tail)
+    uint32_t pad;
+};
+template <int ITEMS>
+struct ScanCtl {
+    InCtl in[kMaxStages];
+    BlkCtl blk[kRingSlots];
+    uint32_t cnt[ITEMS * kWarps];
+    uint32_t total;
+    uint32_t roff;
+    volatile uint32_t tail;              // ring bytes released by the writers (monotone, wraps)
+    uint32_t head;                       // ring bytes reserved by the compute warps (monotone, wraps)
+    uint32_t hpos;                       // next write position in [0, R)
+};
+
+__device__ __forceinline__ uint32_t al16(uint32_t x) { return (x + 15u) & ~15u; }
+
+template <typename T>
+__device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t base, uint32_t total, int64_t cap,
+                                               int q, int nq)
+{
+    const int64_t lim = cap - base;
+    const uint32_t m = (int64_t)total < lim ? total : (lim > 0 ? (uint32_t)lim : 0u);
+    T *d = dst + base;
+    uint32_t j = q;
+    for (; j + 3 * nq < m; j += 4 * nq) {
+        const T a = src[j], b = src[j + nq], c = src[j + 2 * nq], e = src[j + 3 * nq];
+        d[j] = a;
+        d[j + nq] = b;
+        d[j + 2 * nq] = c;
+        d[j + 3 * nq] = e;
+    }
+    for (; j < m; j += nq)
+        d[j] = src[j];
+}
+
 template <int ITEMS, bool AGG>
-__global__ void __launch_bounds__(kThreads) k_scan_chain(const __grid_constant__ ChainProg P,
-                                                         const __grid_constant__ TileLaunch L)
+__global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_constant__ ChainProg P,
+                                                             const __grid_constant__ TileLaunch L)
 {
     constexpr int T = kThreads * ITEMS;
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    CtlSmem<ITEMS> *ctl = (CtlSmem<ITEMS> *)smem_raw;
-    char *stages = (char *)smem_raw + align_up(sizeof(CtlSmem<ITEMS>), 128);
-    char *scratch = stages + (size_t)L.stages * P.stage_bytes;
-    unsigned long long *part = (unsigned long long *)(scratch + P.scratch_bytes);
+    const int S = L.stages;
+    const uint32_t R = L.out_bytes;      // ring bytes (multiple of 128)
+    ScanCtl<ITEMS> *ctl = (ScanCtl<ITEMS> *)smem_raw;
+    char *stages = (char *)smem_raw + align_up(sizeof(ScanCtl<ITEMS>), 128);
+    char *scratch = stages + (size_t)S * P.stage_bytes;
+    char *ring = scratch + P.scratch_bytes;
+    unsigned long long *part = (unsigned long long *)(ring + (AGG ? 0 : R));
     const int NA = P.nagg + 1;
     unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * kThreads : 0);
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
+    const bool emit = !AGG && !(L.dbg & 2);
 
     if (tid == 0) {
-        for (int s = 0; s < L.stages; s++)
-            mbar_init(&ctl->mbar[s], 1);
+        for (int s = 0; s < S; s++) {
+            mbar_init(&ctl->in[s].full, 1);
+            mbar_init(&ctl->in[s].empty, 1);
+        }
+        for (int j = 0; j < kRingSlots; j++) {
+            mbar_init(&ctl->blk[j].aggr, 1);
+            mbar_init(&ctl->blk[j].oempty, 1);
+        }
+        ctl->tail = 0;
+        ctl->head = 0;
+        ctl->hpos = 0;
         fence_mbar_init();
     }
     if (AGG) {
-        for (int q = tid; q < P.D * NA * kThreads; q += kThreads)
+        for (int q = tid; q < P.D * NA * kThreads; q += blockDim.x)
             part[q] = 0;
-        for (int q = tid; q < P.D * NA * 2; q += kThreads)
+        for (int q = tid; q < P.D * NA * 2; q += blockDim.x)
             cta_acc[q] = 0;
     }
     __syncthreads();
 
-    uint32_t tx_bytes = 0;
-    for (int i = 0; i < P.nin; i++)
-        tx_bytes += (uint32_t)T * type_width(P.slot[i].type);
-    const uint64_t policy = policy_evict_first();
-
-    auto refill = [&](int s) {
-        int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
-        ctl->tile_id[s] = t;
-        if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
-            char *st = stages + (size_t)s * P.stage_bytes;
-            fence_proxy_async_smem();
-            mbar_arrive_expect_tx(&ctl->mbar[s], tx_bytes);
-            for (int i = 0; i < P.nin; i++) {
-                const int w = type_width(P.slot[i].type);
-                bulk_g2s(st + P.slot[i].off, (const char *)P.in_ptr[i] + (size_t)t * T * w, (uint32_t)T * w,
-                         &ctl->mbar[s], policy);
-            }
-        } else {
-            mbar_arrive(&ctl->mbar[s]);
-        }
-    };
-
-    if (tid == 0)
-        for (int s = 0; s < L.stages; s++)
-            refill(s);
-
-    int64_t since_flush = 0;
-    for (int64_t it = 0;; ++it) {
-        const int s = (int)(it % L.stages);
-        const uint32_t parity = (uint32_t)((it / L.stages) & 1);
-        mbar_wait(&ctl->mbar[s], parity);
-        const int64_t t = ctl->tile_id[s];
-        if (t >= ntiles)
-            break;
-        char *st = stages + (size_t)s * P.stage_bytes;
-        const int64_t row0 = t * T;
-        const int rows = (int)min((int64_t)T, n - row0);
-        if (!(L.use_tma && rows == T)) {
-            // ragged last tile or unaligned column bases: plain coalesced loads
-            for (int i = 0; i < P.nin; i++) {
-                const int w = type_width(P.slot[i].type);
-                char *dst = st + P.slot[i].off;
-                const char *src = (const char *)P.in_ptr[i] + (size_t)row0 * w;
-                if (w == 4) {
-                    for (int r = tid; r < rows; r += kThreads)
-                        ((uint32_t *)dst)[r] = ((const uint32_t *)src)[r];
-                } else if (w == 8) {
-                    for (int r = tid; r < rows; r += kThreads)
-                        ((uint64_t *)dst)[r] = ((const uint64_t *)src)[r];
+    if (warp == kWarps + kWriterWarps) {
+        // ---------------- producer warp ----------------
+        if (lane == 0) {
+            uint32_t tx_bytes = 0;
+            for (int i = 0; i < P.nin; i++)
+                tx_bytes += (uint32_t)T * type_width(P.slot[i].type);
+            const uint64_t policy = policy_evict_first();
+            int s = 0;
+            uint32_t eph = 1;                                // parity of the previous use
+            for (int64_t i = 0;; ++i) {
+                if (i >= S)
+                    mbar_wait_sleep(&ctl->in[s].empty, eph);
+                const int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
+                ctl->in[s].tile = t;
+                if ((L.dbg & 4) && t < ntiles)
+                    L.dbg_ts[6 * t + 0] = globaltimer();
+                if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
+                    char *st = stages + (size_t)s * P.stage_bytes;
+                    fence_proxy_async_smem();
+                    mbar_arrive_expect_tx(&ctl->in[s].full, tx_bytes);
+                    for (int c = 0; c < P.nin; c++) {
+                        const int w = type_width(P.slot[c].type);
+                        bulk_g2s(st + P.slot[c].off, (const char *)P.in_ptr[c] + (size_t)t * T * w,
+                                 (uint32_t)T * w, &ctl->in[s].full, policy);
+                    }
                 } else {
-                    for (int r = tid; r < rows; r += kThreads)
-                        dst[r] = src[r];
+                    mbar_arrive(&ctl->in[s].full);
+                }
+                if (t >= ntiles)
+                    break;
+                if (++s == S) {
+                    s = 0;
+                    eph ^= 1;
                 }
             }
-            __syncthreads();
         }
-        uint32_t mask = 0;
+    } else if (warp >= kWarps) {
+        // ---------------- writer warps: look-back + compacted store ----------------
+        // Writer w owns ring slots i = w (mod kWriterWarps): the look-backs and copies
+        // of consecutive tiles proceed concurrently; ring bytes are released in order.
+        const int wi = warp - kWarps;
+        if (emit) {
+            for (int64_t i = wi;; i += kWriterWarps) {
+                const int j = (int)(i % kRingSlots);
+                mbar_wait_sleep(&ctl->blk[j].aggr, (uint32_t)((i / kRingSlots) & 1));
+                const int64_t t = ctl->blk[j].tile;
+                if (t >= ntiles)
+                    break;
+                const uint32_t total = ctl->blk[j].total;
+                if ((L.dbg & 4) && lane == 0)
+                    L.dbg_ts[6 * t + 5] = globaltimer();
+                const int64_t excl = (L.dbg & 1) ? t * T
+                                                  : (int64_t)lookback_warp(L.status, t, total, L.epoch, /*aggregate_published=*/true);
+                if (lane == 0) {
+                    if (L.dbg & 4)
+                        L.dbg_ts[6 * t + 3] = globaltimer();
+                    if (t == ntiles - 1)
+                        *L.n_dev = excl + (int64_t)total;
+                }
+                const char *blk = ring + ctl->blk[j].roff;
+                uint32_t coff = 0;
+                for (int c = 0; c < P.nout; c++) {
+                    const int w = P.out_w[c];
+                    const char *src = blk + coff;
+                    coff += al16(total * w);
+                    switch (w) {
+                    case 1: group_copy_out<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, P.out_capacity, lane, 32); break;
+                    case 4: group_copy_out<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, P.out_capacity, lane, 32); break;
+                    default: group_copy_out<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, P.out_capacity, lane, 32); break;
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    if (L.dbg & 4)
+                        L.dbg_ts[6 * t + 4] = globaltimer();
+                    if (i > 0)   // release ring bytes in tile order
+                        mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1));
+                    __threadfence_block();
+                    ctl->tail = ctl->tail + ctl->blk[j].used;
+                    mbar_arrive(&ctl->blk[j].oempty);
+                }
+                __syncwarp();
+            }
+        }
+    } else {
+        // ---------------- compute warps ----------------
+        int64_t since_flush = 0;
+        int s = 0;
+        uint32_t fph = 0;
+        for (int64_t i = 0;; ++i) {
+            if (i > 0 && ++s == S) {
+                s = 0;
+                fph ^= 1;
+            }
+            mbar_wait(&ctl->in[s].full, fph);
+            const int64_t t = ctl->in[s].tile;
+            const int j = (int)(i % kRingSlots);
+            if (t >= ntiles) {
+                if (emit && tid == 0) {
+                    // one sentinel per writer warp (consecutive slots)
+                    for (int64_t u = i; u < i + kWriterWarps; ++u) {
+                        const int ju = (int)(u % kRingSlots);
+                        if (u >= kRingSlots)
+                            mbar_wait(&ctl->blk[ju].oempty, (uint32_t)(((u / kRingSlots) - 1) & 1));
+                        ctl->blk[ju].tile = ntiles;
+                        mbar_arrive(&ctl->blk[ju].aggr);
+                    }
+                }
+                break;
+            }
+            char *st = stages + (size_t)s * P.stage_bytes;
+            const int64_t row0 = t * T;
+            const int rows = (int)min((int64_t)T, n - row0);
+            if ((L.dbg & 4) && tid == 0)
+                L.dbg_ts[6 * t + 1] = globaltimer();
+            if (L.dbg & 2) {   // diagnostics: stream the tiles only (TMA pipeline ceiling)
+                bar_sync(kComputeBar, kThreads);
+                if (tid == 0)
+                    mbar_arrive(&ctl->in[s].empty);
+                continue;
+            }
+            if (!(L.use_tma && rows == T)) {
+                // ragged last tile or unaligned column bases: plain coalesced loads
+                for (int c = 0; c < P.nin; c++) {
+                    const int w = type_width(P.slot[c].type);
+                    char *dst = st + P.slot[c].off;
+                    const char *src = (const char *)P.in_ptr[c] + (size_t)row0 * w;
+                    if (w == 4) {
+                        for (int r = tid; r < rows; r += kThreads)
+                            ((uint32_t *)dst)[r] = ((const uint32_t *)src)[r];
+                    } else if (w == 8) {
+                        for (int r = tid; r < rows; r += kThreads)
+                            ((uint64_t *)dst)[r] = ((const uint64_t *)src)[r];
+                    } else {
+                        for (int r = tid; r < rows; r += kThreads)
+                            dst[r] = src[r];
+                    }
+                }
+                bar_sync(kComputeBar, kThreads);
+            }
+            uint32_t mask = (1u << ITEMS) - 1u;
+            if (rows < T) {
+                mask = 0;
 #pragma unroll
-        for (int k = 0; k < ITEMS; k++)
-            if (k * kThreads + tid < rows)
-                mask |= 1u << k;
-        mask = run_ops<ITEMS>(P, st, scratch, mask);
+                for (int k = 0; k < ITEMS; k++)
+                    if (k * kThreads + tid < rows)
+                        mask |= 1u << k;
+            }
+            mask = run_ops<ITEMS>(P, st, scratch, mask);
+            if (AGG) {
+                agg_tile<ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
+                bar_sync(kComputeBar, kThreads);
+                if (tid == 0)
+                    mbar_arrive(&ctl->in[s].empty);
+                continue;
+            }
+            uint32_t bal[ITEMS];
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
+                if (lane == 0)
+                    ctl->cnt[k * kWarps + warp] = __popc(bal[k]);
+            }
+            bar_sync(kComputeBar, kThreads);
+            if (warp == 0) {
+                constexpr int NV = ITEMS * kWarps;
+                constexpr int PER = (NV + 31) / 32;
+                uint32_t v[PER];
+                uint32_t sum = 0;
+#pragma unroll
+                for (int qq = 0; qq < PER; qq++) {
+                    const int idx = lane * PER + qq;
+                    v[qq] = idx < NV ? ctl->cnt[idx] : 0;
+                    sum += v[qq];
+                }
+                uint32_t inc = sum;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+                    if (lane >= o)
+                        inc += y;
+                }
+                uint32_t run = inc - sum;
+#pragma unroll
+                for (int qq = 0; qq < PER; qq++) {
+                    const int idx = lane * PER + qq;
+                    if (idx < NV)
+                        ctl->cnt[idx] = run;
+                    run += v[qq];
+                }
+                const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+                if (lane == 31) {
+                    // publish the tile aggregate before anything can block this CTA
+                    if (t > 0 && !(L.dbg & 1))
+                        st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
+                    if (L.dbg & 4)
+                        L.dbg_ts[6 * t + 2] = globaltimer();
+                }
+                if (lane == 0) {
+                    // reserve ring bytes for the compacted tile (blocks never wrap)
+                    uint32_t need = 0;
+                    for (int c = 0; c < P.nout; c++)
+                        need += al16(total * P.out_w[c]);
+                    const uint32_t head = ctl->head;
+                    uint32_t pos = ctl->hpos;
+                    uint32_t used = need;
+                    bool drain = false;
+                    if (pos + need > R) {           // blocks never wrap: skip the tail [pos, R)
+                        used += R - pos;
+                        pos = 0;
+                        if (used > R) {             // cannot fit behind live blocks: wait for an empty ring
+                            used = need;
+                            drain = true;
+                        }
+                    }
+                    ctl->hpos = pos + need == R ? 0 : pos + need;
+                    if (i >= kRingSlots)
+                        mbar_wait(&ctl->blk[j].oempty, (uint32_t)(((i / kRingSlots) - 1) & 1));
+                    uint32_t backoff = 32;
+                    while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
+                        __nanosleep(backoff);
+                        backoff = backoff < 512 ? backoff * 2 : 512;
+                    }
+                    ctl->head = head + used;
+                    ctl->roff = pos;
+                    ctl->total = total;
+                    ctl->blk[j].used = used;
+                }
+            }
+            bar_sync(kComputeBar, kThreads);
+            const uint32_t total = ctl->total;
+            char *blk = ring + ctl->roff;
+            const uint32_t lt = lanemask_lt();
+            uint32_t pos[ITEMS];
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++)
+                pos[k] = ctl->cnt[k * kWarps + warp] + __popc(bal[k] & lt);
+            uint32_t coff = 0;
+            for (int c = 0; c < P.nout; c++) {
+                const int w = P.out_w[c];
+                const char *src = loc_ptr(P.out_loc[c], st, scratch);
+                char *dst = blk + coff;
+                coff += al16(total * w);
+                switch (w) {
+                case 1:
+#pragma unroll
+                    for (int k = 0; k < ITEMS; k++)
+                        if ((mask >> k) & 1u) ((uint8_t *)dst)[pos[k]] = ((const uint8_t *)src)[k * kThreads + tid];
+                    break;
+                case 4:
+#pragma unroll
+                    for (int k = 0; k < ITEMS; k++)
+                        if ((mask >> k) & 1u) ((uint32_t *)dst)[pos[k]] = ((const uint32_t *)src)[k * kThreads + tid];
+                    break;
+                default:
+#pragma unroll
+                    for (int k = 0; k < ITEMS; k++)
+                        if ((mask >> k) & 1u) ((uint64_t *)dst)[pos[k]] = ((const uint64_t *)src)[k * kThreads + tid];
+                    break;
+                }
+            }
+            bar_sync(kComputeBar, kThreads);
+            if (tid == 0) {
+                mbar_arrive(&ctl->in[s].empty);          // input tile and scratch are free
+                ctl->blk[j].tile = t;
+                ctl->blk[j].total = total;
+                ctl->blk[j].roff = (uint32_t)(blk - ring);
+                mbar_arrive(&ctl->blk[j].aggr);
+            }
+        }
         if (AGG)
-            agg_tile<ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
-        else
-            emit_tile<ITEMS>(P, st, scratch, mask, t, ntiles, L, &ctl->es);
-        __syncthreads();
-        if (tid == 0)
-            refill(s);
+            agg_flush(P, part, cta_acc);
     }
-
+    __syncthreads();
     if (AGG) {
-        agg_flush(P, part, cta_acc);
-        __syncthreads();
-        for (int q = tid; q < P.D * NA; q += kThreads) {
-            unsigned long long lo = cta_acc[2 * q], hi = cta_acc[2 * q + 1];
+        for (int qq = tid; qq < P.D * NA; qq += blockDim.x) {
+            const unsigned long long lo = cta_acc[2 * qq], hi = cta_acc[2 * qq + 1];
             if (lo | hi)
-                atomic_add128(&L.agg_acc[2 * q], &L.agg_acc[2 * q + 1], lo, hi);
+                atomic_add128(&L.agg_acc[2 * qq], &L.agg_acc[2 * qq + 1], lo, hi);
         }
     } else if (ntiles == 0 && blockIdx.x == 0 && tid == 0) {
         *L.n_dev = 0;
@@ -601,7 +869,7 @@ __global__ void __launch_bounds__(kThreads) k_join_expand(const __grid_constant_
 // ===========================================================================
 // Host launchers
 // ===========================================================================
-size_t scan_ctl_bytes() { return align_up(sizeof(CtlSmem<kScanItems>), 128); }   // >= CtlSmem<4>
+size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<kScanItems>), 128); }   // >= ITEMS 4
 size_t join_ctl_bytes() { return align_up(sizeof(JoinCtl), 128); }
 size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
 int scan_tile() { return kThreads * kScanItems; }
@@ -613,11 +881,11 @@ size_t join_runs_smem(int key_type)
 }
 
 template <typename F>
-static int occ(F f, size_t smem)
+static int occ(F f, size_t smem, int threads = kThreads)
 {
     int n = 0;
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, kThreads, smem) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, threads, smem) != cudaSuccess)
         return 0;
     return n;
 }
@@ -625,8 +893,8 @@ static int occ(F f, size_t smem)
 int chain_occupancy(int which, int items, size_t smem)
 {
     switch (which) {
-    case 0: return items == 4 ? occ(k_scan_chain<4, false>, smem) : occ(k_scan_chain<8, false>, smem);
-    case 1: return items == 4 ? occ(k_scan_chain<4, true>, smem) : occ(k_scan_chain<8, true>, smem);
+    case 0: return items == 4 ? occ(k_scan_chain<4, false>, smem, kScanThreads) : occ(k_scan_chain<8, false>, smem, kScanThreads);
+    case 1: return items == 4 ? occ(k_scan_chain<4, true>, smem, kScanThreads) : occ(k_scan_chain<8, true>, smem, kScanThreads);
     case 2: return occ(k_join_expand, smem);
     default: return occ(k_join_runs<uint64_t>, smem);
     }
@@ -636,7 +904,7 @@ template <int ITEMS, bool AGG>
 static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
     cudaFuncSetAttribute(k_scan_chain<ITEMS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_chain<ITEMS, AGG><<<grid, kThreads, smem, s>>>(P, L);
+    k_scan_chain<ITEMS, AGG><<<grid, kScanThreads, smem, s>>>(P, L);
     return cudaGetLastError();
 }
 

@@ -45,11 +45,37 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
         "{\n"
         ".reg .pred p;\n"
         "RW_WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
         "@!p bra RW_WAIT_%=;\n"
         "}\n" ::"r"(smem_u32(bar)),
-        "r"(parity)
+        "r"(parity), "r"(1000000u)   // suspend-time hint (ns): sleep until the phase flips
         : "memory");
+}
+
+__device__ __forceinline__ bool mbar_try(uint64_t *bar, uint32_t parity)
+{
+    uint32_t ok;
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        "selp.u32 %0, 1, 0, p;\n"
+        "}\n"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+// wait with exponential nanosleep backoff: for warps off the critical path
+// (producer, writers) so their polling does not steal issue slots
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity)
+{
+    uint32_t ns = 64;
+    while (!mbar_try(bar, parity)) {
+        __nanosleep(ns);
+        ns = ns < 2048 ? ns * 2 : 2048;
+    }
 }
 
 // 1-D bulk copy global -> shared, completion signalled on `bar` (complete_tx).
@@ -82,6 +108,19 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
 __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
 {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t globaltimer()
+{
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// named barrier among `n` threads (n a multiple of 32); id 0 is __syncthreads
+__device__ __forceinline__ void bar_sync(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt()

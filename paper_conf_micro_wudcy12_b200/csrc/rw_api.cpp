@@ -90,6 +90,9 @@ struct Lowered {
     ChainProg P;
     std::vector<int> in_src;      // input slot i <- source column in_src[i]
     int items = 8, stages = 2, ctas = 1;
+    int ring = 0;                 // scan kernel: output ring entries
+    uint32_t out_bytes = 0;       // bytes of one output ring entry
+    std::vector<uint32_t> out_off;
     size_t smem = 0;
     bool agg = false;
     AggFinal F;
@@ -387,6 +390,13 @@ int classify_edge(const rw_plan *p, int prod, int cons)
 // ---------------------------------------------------------------------------
 // Lowering of one group to a ChainProg
 // ---------------------------------------------------------------------------
+// host form of a micro-op (slot ids); encoded into DevOp locations after layout
+struct HOp {
+    uint8_t kind, op, type, b_is_slot;
+    int16_t dst, a, b, pad;
+    int64_t k;
+};
+
 struct SlotB {
     int type;
     bool input;
@@ -405,7 +415,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     std::memset(&L.P, 0, sizeof(L.P));
     std::memset(&L.F, 0, sizeof(L.F));
     std::vector<SlotB> slots;
-    std::vector<DevOp> ops;
+    std::vector<HOp> ops;
     std::vector<int> src_slot(src_types.size(), -1);
     auto get_src = [&](int c) {
         if (src_slot[c] < 0) {
@@ -422,7 +432,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     for (size_t c = 0; c < cur.size(); c++)
         cur[c] = -1 - (int)c;
     auto resolve = [&](int v) { return v >= 0 ? v : get_src(-1 - v); };
-    auto push = [&](const DevOp &o) {
+    auto push = [&](const HOp &o) {
         if ((int)ops.size() >= kMaxOps)
             raise(RW_E_UNSUPPORTED, "fused group exceeds the micro-op budget");
         ops.push_back(o);
@@ -432,7 +442,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         const Node &nd = p->nodes[nid];
         if (nd.kind == N_SELECT) {
             for (const rw_pred &a : nd.preds) {
-                DevOp o{};
+                HOp o{};
                 o.kind = K_PRED;
                 o.op = (uint8_t)a.op;
                 o.a = (int16_t)resolve(cur[a.col]);
@@ -463,7 +473,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                         vslot[i] = s;
                     } else {
                         int d = new_slot(x.type);
-                        DevOp o{};
+                        HOp o{};
                         o.kind = K_EXPR; o.op = E_COPY; o.type = (uint8_t)x.type;
                         o.dst = (int16_t)d; o.a = (int16_t)s; o.b = -1;
                         push(o);
@@ -499,7 +509,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                         return;
                     }
                     int d = new_slot(t);
-                    DevOp o{};
+                    HOp o{};
                     o.kind = K_EXPR; o.op = E_DIVC; o.type = (uint8_t)t;
                     o.dst = (int16_t)d; o.a = (int16_t)vslot[x.a]; o.b = -1;
                     o.k = (int64_t)wrap_to(t, x.k);
@@ -513,7 +523,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                     return;
                 }
                 int d = new_slot(t);
-                DevOp o{};
+                HOp o{};
                 o.kind = K_EXPR; o.type = (uint8_t)t; o.dst = (int16_t)d; o.b = -1;
                 const uint8_t base = x.op == RW_ADD ? E_ADD : x.op == RW_SUB ? E_SUB : E_MUL;
                 if (isconst[x.b]) {
@@ -532,7 +542,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 ev(r);
                 if (isconst[r]) {
                     int d = new_slot(e[r].type);
-                    DevOp o{};
+                    HOp o{};
                     o.kind = K_EXPR; o.op = E_CONST; o.type = (uint8_t)e[r].type;
                     o.dst = (int16_t)d; o.a = -1; o.b = -1; o.k = (int64_t)vconst[r];
                     push(o);
@@ -604,7 +614,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
 
     // liveness
     for (size_t i = 0; i < ops.size(); i++) {
-        const DevOp &o = ops[i];
+        const HOp &o = ops[i];
         if (o.a >= 0) slots[o.a].last_use = std::max(slots[o.a].last_use, (int)i);
         if (o.b_is_slot && o.b >= 0) slots[o.b].last_use = std::max(slots[o.b].last_use, (int)i);
     }
@@ -656,12 +666,11 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     L.in_src.clear();
     for (int i = 0; i < nin; i++)
         L.in_src.push_back(slots[order[i]].src);
-    for (size_t i = 0; i < ops.size(); i++) {
-        DevOp o = ops[i];
+    std::vector<HOp> rops(ops);
+    for (HOp &o : rops) {
         if (o.a >= 0) o.a = (int16_t)remap[o.a];
         if (o.b_is_slot && o.b >= 0) o.b = (int16_t)remap[o.b];
         if (o.dst >= 0) o.dst = (int16_t)remap[o.dst];
-        P.ops[i] = o;
     }
     if (L.agg) {
         for (int c = 0; c < P.ngc; c++) P.gslot[c] = (int16_t)remap[P.gslot[c]];
@@ -693,6 +702,36 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             const SlotB &sb = slots[order[i]];
             P.slot[i].off = sb.region >= 0 ? roff[sb.region] : 0;
         }
+        // resolve every slot reference to an encoded smem location
+        auto loc = [&](int sl) -> uint32_t {
+            if (sl < 0) return 0;
+            return (P.slot[sl].is_input ? 0u : kLocScratch) | P.slot[sl].off;
+        };
+        for (size_t i = 0; i < rops.size(); i++) {
+            const HOp &h = rops[i];
+            DevOp d{};
+            d.kind = h.kind;
+            d.code = (uint8_t)(h.type * 8 + h.op + (h.b_is_slot ? 64 : 0));
+            d.ta = h.a >= 0 ? P.slot[h.a].type : (uint8_t)h.type;
+            d.tb = (h.b_is_slot && h.b >= 0) ? P.slot[h.b].type : (uint8_t)h.type;
+            d.a = loc(h.a);
+            d.b = h.b_is_slot ? loc(h.b) : 0;
+            d.dst = h.dst >= 0 ? loc(h.dst) : 0;
+            d.k = h.k;
+            P.ops[i] = d;
+        }
+        for (int c = 0; c < P.nout; c++) {
+            P.out_loc[c] = loc(P.out_slot[c]);
+            P.out_w[c] = (uint8_t)type_width(P.slot[P.out_slot[c]].type);
+        }
+        for (int c = 0; c < P.ngc; c++) {
+            P.g_loc[c] = loc(P.gslot[c]);
+            P.g_type[c] = P.slot[P.gslot[c]].type;
+        }
+        for (int q = 0; q < P.nagg; q++) {
+            P.agg_loc[q] = loc(P.agg_slot[q]);
+            P.agg_type[q] = P.slot[P.agg_slot[q]].type;
+        }
     };
     const size_t agg_bytes =
         L.agg ? (size_t)P.D * (P.nagg + 1) * kThreads * 8 + al128((size_t)P.D * (P.nagg + 1) * 16) : 0;
@@ -710,31 +749,53 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         L.ctas = std::max(1, chain_occupancy(2, kJoinItems, L.smem));
         return;
     }
+    // Scan kernel: S input stages (TMA ring), one scratch tile for computed
+    // columns, and a byte ring of R bytes holding compacted tiles until their
+    // global offset is resolved (resource budget, §4.3.3).
     const int want_stages = p->o.stages > 0 ? std::min(p->o.stages, kMaxStages) : 0;
-    double best = -1;
+    const size_t want_ring = p->o.reserved[0] > 0 ? (size_t)p->o.reserved[0] * 1024 : 0;
+    bool ok = false;
     for (int items : {8, 4}) {
         const int T = kThreads * items;
         layout(T);
-        for (int S = kMaxStages; S >= 1; S--) {
-            if (want_stages && S != want_stages) continue;
-            if (!want_stages && S > 4) continue;
-            size_t smem = scan_ctl_bytes() + (size_t)S * P.stage_bytes + P.scratch_bytes + agg_bytes;
-            if (smem > kSmemLimit) continue;
-            int occ = chain_occupancy(L.agg ? 1 : 0, items, smem);
-            if (occ <= 0) continue;
-            if (p->o.ctas_per_sm > 0) occ = std::min(occ, p->o.ctas_per_sm);
-            double inflight = (double)occ * S * std::max<uint32_t>(P.stage_bytes, 1);
-            double score = inflight + (items == 8 ? 1.0 : 0.0) + 0.01 * occ;
-            if (score > best) {
-                best = score;
+        size_t W = 0;                       // largest compacted tile (every row survives)
+        for (int c = 0; c < P.nout; c++)
+            W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+        const size_t base = scan_ctl_bytes() + P.scratch_bytes + agg_bytes;
+        const int occ_pref[2] = {2, 1};
+        for (int oi = 0; oi < 2 && !ok; oi++) {
+            int occ_t = occ_pref[oi];
+            if (p->o.ctas_per_sm > 0) {
+                if (oi > 0) break;
+                occ_t = p->o.ctas_per_sm;
+            }
+            const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
+            for (int S : {3, 2, 1, 4, 5, 6}) {
+                if (want_stages && S != want_stages) continue;
+                if (!want_stages && occ_t >= 2 && S > 2) continue;
+                if (base + (size_t)S * P.stage_bytes > per_cta) continue;
+                size_t Rb = 0;
+                if (!L.agg) {
+                    Rb = want_ring ? want_ring : (per_cta - base - (size_t)S * P.stage_bytes) / 128 * 128;
+                    if (Rb < W) continue;
+                }
+                const size_t smem = base + (size_t)S * P.stage_bytes + Rb;
+                if (smem > per_cta) continue;
+                int occ = chain_occupancy(L.agg ? 1 : 0, items, smem);
+                if (occ < occ_t) continue;
                 L.items = items;
                 L.stages = S;
+                L.ring = 0;
+                L.out_bytes = (uint32_t)Rb;
                 L.smem = smem;
-                L.ctas = occ;
+                L.ctas = occ_t;
+                ok = true;
+                break;
             }
         }
+        if (ok) break;
     }
-    if (best < 0)
+    if (!ok)
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
     layout(kThreads * L.items);
 }
@@ -870,6 +931,9 @@ void run_group(ExecCtx &X, int gi)
         TL.n = src.n_host >= 0 ? src.n_host : 0;
         TL.n_ptr = src.n_host >= 0 ? nullptr : src.n_dev;
         TL.stages = L.stages;
+        TL.dbg = p->o.reserved[1];
+        TL.dbg_ts = (uint64_t *)(((uint64_t)(uint32_t)p->o.reserved[3] << 32) | (uint32_t)p->o.reserved[2]);
+        TL.out_bytes = L.out_bytes;
         TL.use_tma = aligned ? 1 : 0;
         TL.epoch = next_epoch(p);
         TL.status = p->status;
@@ -1097,7 +1161,8 @@ std::string explain(rw_plan *p, int out_node)
             Lowered L;
             std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
             lower(p, g, st, L);
-            s << " | tile " << kThreads * L.items << " rows, stages " << L.stages << ", smem " << L.smem
+            s << " | tile " << kThreads * L.items << " rows, stages " << L.stages << ", out ring " << L.out_bytes << " B"
+              << ", smem " << L.smem
               << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
               << L.P.nops;
         } catch (const RwError &e) {

@@ -148,7 +148,8 @@ class Plan:
     plain-data spelling (see oracle/__init__.py docstring)."""
 
     def __init__(self, device: int = 0, stream=None, fuse: bool = True, zero_copy_project: bool = False,
-                 stages: int = 0, ctas_per_sm: int = 0, strict_overflow: bool = False):
+                 stages: int = 0, ctas_per_sm: int = 0, strict_overflow: bool = False, defer: int = 0,
+                 dbg: int = 0, dbg_ts: int = 0):
         import torch
         if stream is None:
             stream = torch.cuda.current_stream(device)
@@ -160,6 +161,10 @@ class Plan:
         o.zero_copy_project = 1 if zero_copy_project else 0
         o.stages, o.ctas_per_sm = stages, ctas_per_sm
         o.strict_overflow = 1 if strict_overflow else 0
+        o.reserved[0] = defer              # scan kernel store delay in tiles (0 = auto)
+        o.reserved[1] = dbg                # diagnostics only (1: no look-back, 2: stream only, 4: timestamps)
+        o.reserved[2] = ctypes.c_int32(dbg_ts & 0xffffffff).value
+        o.reserved[3] = ctypes.c_int32((dbg_ts >> 32) & 0xffffffff).value
         self.device = device
         h = ctypes.c_void_p()
         check(lib().rw_plan_create(ctypes.byref(h), ctypes.byref(o)))

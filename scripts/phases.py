@@ -1,0 +1,32 @@
+"""Diagnostic: per-tile phase timestamps of the C2 scan kernel (dbg=4)."""
+import sys, os, json
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import workloads
+from tests.planspec import build_gpu_plan
+
+def main(stages, ctas, ring, rows=1 << 29):
+    spec = workloads.c2_spec()
+    ins = workloads.c2_inputs(rows, 0, "cuda:0")
+    T = 2048
+    nt = (rows + T - 1) // T
+    ts = torch.zeros(nt * 6, dtype=torch.int64, device="cuda:0")
+    plan, ids = build_gpu_plan(spec, stages=stages, ctas_per_sm=ctas, defer=ring, dbg=4, dbg_ts=ts.data_ptr())
+    outs = [torch.empty(rows, dtype=torch.int32, device="cuda:0") for _ in range(3)]
+    nd = torch.zeros(1, dtype=torch.int64, device="cuda:0")
+    for _ in range(3):
+        plan.execute([(rows, ins["R"])], ids["s2"], outs, rows, n_dev=nd)
+    torch.cuda.synchronize()
+    a = ts.view(nt, 6).double()
+    t0 = a[:, 0].min()
+    d = {"load(claim->data)": a[:, 1] - a[:, 0], "eval(data->agg)": a[:, 2] - a[:, 1],
+         "writer queue(agg->wstart)": a[:, 5] - a[:, 2], "lookback(wstart->offset)": a[:, 3] - a[:, 5], "store(offset->stored)": a[:, 4] - a[:, 3],
+         "total(claim->stored)": a[:, 4] - a[:, 0]}
+    res = {"cfg": [stages, ctas, ring], "kernel_us": float((a[:, 4].max() - t0) / 1e3)}
+    for k, v in d.items():
+        q = torch.quantile(v[: min(nt, 1 << 24)] / 1e3, torch.tensor([0.1, 0.5, 0.9, 0.99], dtype=torch.float64, device=v.device))
+        res[k] = [round(float(x), 2) for x in q]
+    print(json.dumps(res))
+
+if __name__ == "__main__":
+    main(*[int(x) for x in sys.argv[1:4]])

@@ -160,7 +160,7 @@ def test_random_chains_against_oracle():
 def test_capacity_error_reports_required_rows():
     import torch
     from paper_conf_micro_wudcy12_b200 import rw
-    spec = workloads.c1_spec(1.0, 1.0)
+    spec = workloads.c1_spec(0.9999, 0.9999)
     ins = workloads.c1_inputs(5000, device=DEV, cfg=0x87)
     plan, ids = build_gpu_plan(spec)
     outs = [torch.empty(100, dtype=torch.int32, device=DEV) for _ in range(2)]
