@@ -2,7 +2,7 @@
 // (SELECT atoms, PROJECT / arithmetic), warp-ballot compaction, block scan,
 // decoupled look-back, compacted store, and the group-by aggregate terminal.
 //
-// Tile layout: T = kThreads * ITEMS rows; thread `tid` owns rows k*kThreads+tid
+// Tile layout: T = NT * ITEMS rows; thread `tid` owns rows k*NT+tid
 // (k < ITEMS), so every smem slot access and every global store of a warp is
 // over 32 consecutive rows.  The per-row predicate result is one bit of the
 // register `mask` (§5.1.1: filters AND-ed into `match`).
@@ -147,7 +147,7 @@ __device__ __forceinline__ bool cmpv(T x, T y)
 }
 
 // SELECT atom over the tile: clears bits of rows failing `a CMP b` (reading A4).
-template <int ITEMS, typename T, int CMP, bool BSLOT>
+template <int NT, int ITEMS, typename T, int CMP, bool BSLOT>
 __device__ __forceinline__ uint32_t pred_loop(const char *a, const char *b, T k, uint32_t mask)
 {
     const int tid = threadIdx.x;
@@ -156,31 +156,31 @@ __device__ __forceinline__ uint32_t pred_loop(const char *a, const char *b, T k,
     uint32_t keep = 0;
 #pragma unroll
     for (int i = 0; i < ITEMS; i++) {
-        const T x = pa[i * kThreads + tid];
-        const T y = BSLOT ? pb[i * kThreads + tid] : k;
+        const T x = pa[i * NT + tid];
+        const T y = BSLOT ? pb[i * NT + tid] : k;
         keep |= (uint32_t)cmpv<T, CMP>(x, y) << i;
     }
     return mask & keep;
 }
 
 #define RW_PRED_CASES(TT, TCODE)                                                                        \
-    case TCODE * 8 + C_LT: return pred_loop<ITEMS, TT, C_LT, false>(a, b, (TT)o.k, mask);           \
-    case TCODE * 8 + C_LE: return pred_loop<ITEMS, TT, C_LE, false>(a, b, (TT)o.k, mask);           \
-    case TCODE * 8 + C_GT: return pred_loop<ITEMS, TT, C_GT, false>(a, b, (TT)o.k, mask);           \
-    case TCODE * 8 + C_GE: return pred_loop<ITEMS, TT, C_GE, false>(a, b, (TT)o.k, mask);           \
-    case TCODE * 8 + C_EQ: return pred_loop<ITEMS, TT, C_EQ, false>(a, b, (TT)o.k, mask);           \
-    case TCODE * 8 + C_NE: return pred_loop<ITEMS, TT, C_NE, false>(a, b, (TT)o.k, mask);           \
-    case 64 + TCODE * 8 + C_LT: return pred_loop<ITEMS, TT, C_LT, true>(a, b, (TT)0, mask);         \
-    case 64 + TCODE * 8 + C_LE: return pred_loop<ITEMS, TT, C_LE, true>(a, b, (TT)0, mask);         \
-    case 64 + TCODE * 8 + C_GT: return pred_loop<ITEMS, TT, C_GT, true>(a, b, (TT)0, mask);         \
-    case 64 + TCODE * 8 + C_GE: return pred_loop<ITEMS, TT, C_GE, true>(a, b, (TT)0, mask);         \
-    case 64 + TCODE * 8 + C_EQ: return pred_loop<ITEMS, TT, C_EQ, true>(a, b, (TT)0, mask);         \
-    case 64 + TCODE * 8 + C_NE: return pred_loop<ITEMS, TT, C_NE, true>(a, b, (TT)0, mask);
+    case TCODE * 8 + C_LT: return pred_loop<NT, ITEMS, TT, C_LT, false>(a, b, (TT)k, mask);             \
+    case TCODE * 8 + C_LE: return pred_loop<NT, ITEMS, TT, C_LE, false>(a, b, (TT)k, mask);             \
+    case TCODE * 8 + C_GT: return pred_loop<NT, ITEMS, TT, C_GT, false>(a, b, (TT)k, mask);             \
+    case TCODE * 8 + C_GE: return pred_loop<NT, ITEMS, TT, C_GE, false>(a, b, (TT)k, mask);             \
+    case TCODE * 8 + C_EQ: return pred_loop<NT, ITEMS, TT, C_EQ, false>(a, b, (TT)k, mask);             \
+    case TCODE * 8 + C_NE: return pred_loop<NT, ITEMS, TT, C_NE, false>(a, b, (TT)k, mask);             \
+    case 64 + TCODE * 8 + C_LT: return pred_loop<NT, ITEMS, TT, C_LT, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_LE: return pred_loop<NT, ITEMS, TT, C_LE, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_GT: return pred_loop<NT, ITEMS, TT, C_GT, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_GE: return pred_loop<NT, ITEMS, TT, C_GE, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_EQ: return pred_loop<NT, ITEMS, TT, C_EQ, true>(a, b, (TT)0, mask);         \
+    case 64 + TCODE * 8 + C_NE: return pred_loop<NT, ITEMS, TT, C_NE, true>(a, b, (TT)0, mask);
 
-template <int ITEMS>
-__device__ __noinline__ uint32_t run_pred(const DevOp &o, const char *a, const char *b, uint32_t mask)
+template <int NT, int ITEMS>
+__device__ __noinline__ uint32_t run_pred(uint32_t code, int64_t k, const char *a, const char *b, uint32_t mask)
 {
-    switch (o.code) {
+    switch (code) {
         RW_PRED_CASES(int32_t, T_I32)
         RW_PRED_CASES(uint32_t, T_U32)
         RW_PRED_CASES(int64_t, T_I64)
@@ -210,7 +210,7 @@ __device__ __forceinline__ T ev(T a, T b)
 
 // dst[r] = a[r] OP (b[r] | k) over the tile.  Operands stored in another type are
 // converted into T (mod 2^w); same-type operands are loaded directly.
-template <int ITEMS, typename T, int OP, bool BSLOT>
+template <int NT, int ITEMS, typename T, int OP, bool BSLOT>
 __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, const char *b, int tb, T k)
 {
     const int tid = threadIdx.x;
@@ -223,7 +223,7 @@ __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, cons
     if (sa && (!BSLOT || sb)) {
 #pragma unroll
         for (int i = 0; i < ITEMS; i++) {
-            const int r = i * kThreads + tid;
+            const int r = i * NT + tid;
             const T x = (OP == E_CONST) ? (T)0 : ld_as<T>(a, r);
             const T y = BSLOT ? ld_as<T>(b, r) : k;
             ((T *)dst)[r] = ev<T, OP>(x, y);
@@ -231,7 +231,7 @@ __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, cons
     } else {
 #pragma unroll
         for (int i = 0; i < ITEMS; i++) {
-            const int r = i * kThreads + tid;
+            const int r = i * NT + tid;
             const T x = (OP == E_CONST) ? (T)0 : (T)ld_ext(a, ta, r);
             const T y = BSLOT ? (T)ld_ext(b, tb, r) : k;
             ((T *)dst)[r] = ev<T, OP>(x, y);
@@ -240,21 +240,21 @@ __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, cons
 }
 
 #define RW_EXPR_CASES(TT, TCODE)                                                                                  \
-    case TCODE * 8 + E_COPY: expr_loop<ITEMS, TT, E_COPY, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
-    case TCODE * 8 + E_CONST: expr_loop<ITEMS, TT, E_CONST, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;     \
-    case TCODE * 8 + E_ADD: expr_loop<ITEMS, TT, E_ADD, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
-    case TCODE * 8 + E_SUB: expr_loop<ITEMS, TT, E_SUB, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
-    case TCODE * 8 + E_MUL: expr_loop<ITEMS, TT, E_MUL, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;         \
-    case TCODE * 8 + E_DIVC: expr_loop<ITEMS, TT, E_DIVC, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
-    case TCODE * 8 + E_RSUB: expr_loop<ITEMS, TT, E_RSUB, false>(dst, a, o.ta, b, o.tb, (TT)o.k); return;       \
-    case 64 + TCODE * 8 + E_ADD: expr_loop<ITEMS, TT, E_ADD, true>(dst, a, o.ta, b, o.tb, (TT)0); return;       \
-    case 64 + TCODE * 8 + E_SUB: expr_loop<ITEMS, TT, E_SUB, true>(dst, a, o.ta, b, o.tb, (TT)0); return;       \
-    case 64 + TCODE * 8 + E_MUL: expr_loop<ITEMS, TT, E_MUL, true>(dst, a, o.ta, b, o.tb, (TT)0); return;
+    case TCODE * 8 + E_COPY: expr_loop<NT, ITEMS, TT, E_COPY, false>(dst, a, ta, b, tb, (TT)k); return;       \
+    case TCODE * 8 + E_CONST: expr_loop<NT, ITEMS, TT, E_CONST, false>(dst, a, ta, b, tb, (TT)k); return;     \
+    case TCODE * 8 + E_ADD: expr_loop<NT, ITEMS, TT, E_ADD, false>(dst, a, ta, b, tb, (TT)k); return;         \
+    case TCODE * 8 + E_SUB: expr_loop<NT, ITEMS, TT, E_SUB, false>(dst, a, ta, b, tb, (TT)k); return;         \
+    case TCODE * 8 + E_MUL: expr_loop<NT, ITEMS, TT, E_MUL, false>(dst, a, ta, b, tb, (TT)k); return;         \
+    case TCODE * 8 + E_DIVC: expr_loop<NT, ITEMS, TT, E_DIVC, false>(dst, a, ta, b, tb, (TT)k); return;       \
+    case TCODE * 8 + E_RSUB: expr_loop<NT, ITEMS, TT, E_RSUB, false>(dst, a, ta, b, tb, (TT)k); return;       \
+    case 64 + TCODE * 8 + E_ADD: expr_loop<NT, ITEMS, TT, E_ADD, true>(dst, a, ta, b, tb, (TT)0); return;       \
+    case 64 + TCODE * 8 + E_SUB: expr_loop<NT, ITEMS, TT, E_SUB, true>(dst, a, ta, b, tb, (TT)0); return;       \
+    case 64 + TCODE * 8 + E_MUL: expr_loop<NT, ITEMS, TT, E_MUL, true>(dst, a, ta, b, tb, (TT)0); return;
 
-template <int ITEMS>
-__device__ __noinline__ void run_expr(const DevOp &o, char *dst, const char *a, const char *b)
+template <int NT, int ITEMS>
+__device__ __noinline__ void run_expr(uint32_t code, int ta, int tb, int64_t k, char *dst, const char *a, const char *b)
 {
-    switch (o.code) {
+    switch (code) {
         RW_EXPR_CASES(int32_t, T_I32)
         RW_EXPR_CASES(uint32_t, T_U32)
         RW_EXPR_CASES(int64_t, T_I64)
@@ -264,18 +264,21 @@ __device__ __noinline__ void run_expr(const DevOp &o, char *dst, const char *a, 
 
 // Run the fused program over one tile (§4.3.1: SELECT / PROJECT in order,
 // in the same thread, no synchronisation between thread-dependent operators).
-template <int ITEMS>
+template <int NT, int ITEMS>
 __device__ __forceinline__ uint32_t run_ops(const ChainProg &P, const char *stage, char *scratch, uint32_t mask)
 {
 #pragma unroll 1
     for (int i = 0; i < P.nops; i++) {
-        const DevOp &o = P.ops[i];
-        const char *a = loc_ptr(o.a, stage, scratch);
-        const char *b = loc_ptr(o.b, stage, scratch);
-        if (o.kind == K_PRED)
-            mask = run_pred<ITEMS>(o, a, b, mask);
+        // fields are read once from the constant bank and passed by value (a reference
+        // into kernel-parameter space would turn every field access into a generic load)
+        const uint32_t kind = P.ops[i].kind, code = P.ops[i].code;
+        const int64_t k = P.ops[i].k;
+        const char *a = loc_ptr(P.ops[i].a, stage, scratch);
+        const char *b = loc_ptr(P.ops[i].b, stage, scratch);
+        if (kind == K_PRED)
+            mask = run_pred<NT, ITEMS>(code, k, a, b, mask);
         else
-            run_expr<ITEMS>(o, (char *)loc_ptr(o.dst, stage, scratch), a, b);
+            run_expr<NT, ITEMS>(code, P.ops[i].ta, P.ops[i].tb, k, (char *)loc_ptr(P.ops[i].dst, stage, scratch), a, b);
     }
     return mask;
 }
@@ -381,24 +384,25 @@ __device__ __forceinline__ void atomic_add128(unsigned long long *lo, unsigned l
         atomicAdd(hi, h);
 }
 
+template <int NT>
 __device__ inline void agg_flush(const ChainProg &P, unsigned long long *part, unsigned long long *cta_acc)
 {
     const int tid = threadIdx.x;
     const int NA = P.nagg + 1;
     const int n = P.D * NA;
     for (int q = 0; q < n; q++) {
-        unsigned long long v = part[q * kThreads + tid];
+        unsigned long long v = part[q * NT + tid];
         if (v) {
             const int a = q % NA;
             const bool uns = a > 0 && P.agg_unsigned[a - 1];
             unsigned long long hi = (!uns && (long long)v < 0) ? ~0ull : 0ull;
             atomic_add128(&cta_acc[2 * q], &cta_acc[2 * q + 1], v, hi);
-            part[q * kThreads + tid] = 0;
+            part[q * NT + tid] = 0;
         }
     }
 }
 
-template <int ITEMS>
+template <int NT, int ITEMS>
 __device__ inline void agg_tile(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
                                 unsigned long long *part, unsigned long long *cta_acc, int64_t &since_flush,
                                 int32_t *err)
@@ -409,7 +413,7 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
     for (int k = 0; k < ITEMS; k++) {
         if (!((mask >> k) & 1u))
             continue;
-        const int r = k * kThreads + tid;
+        const int r = k * NT + tid;
         int g = 0;
         bool ok = true;
         for (int c = 0; c < P.ngc; c++) {
@@ -423,12 +427,12 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
             atomicAdd(err, 1);
             continue;
         }
-        unsigned long long *pg = part + (size_t)g * NA * kThreads + tid;
+        unsigned long long *pg = part + (size_t)g * NA * NT + tid;
         pg[0] += 1ull;
         for (int a = 0; a < P.nagg; a++)
-            pg[(a + 1) * kThreads] += ld_ext(loc_ptr(P.agg_loc[a], stage, scratch), P.agg_type[a], r);
+            pg[(a + 1) * NT] += ld_ext(loc_ptr(P.agg_loc[a], stage, scratch), P.agg_type[a], r);
         if (++since_flush >= P.flush_rows) {
-            agg_flush(P, part, cta_acc);
+            agg_flush<NT>(P, part, cta_acc);
             since_flush = 0;
         }
     }

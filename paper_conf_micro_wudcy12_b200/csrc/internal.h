@@ -103,7 +103,7 @@ struct TileLaunch {
     int32_t *err;              // [0] domain errors
     int32_t dbg;               // diagnostics: 1 = skip look-back (offset = tile * T, uncompacted),
                                // 2 = stream tiles only, 4 = per-tile phase timestamps into dbg_ts
-    uint64_t *dbg_ts;          // 6 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start)
+    uint64_t *dbg_ts;          // 8 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots)
 };
 
 // Join expansion inputs (run records written by k_join_runs).

@@ -53,7 +53,7 @@ __device__ inline void cta_exit_reset(uint32_t *ctrs)
 // worst-case slot) while it waits, so enough tiles stay in flight per SM.
 // ===========================================================================
 constexpr int kWriterWarps = 4;
-constexpr int kScanThreads = kThreads + 32 * (kWriterWarps + 1);
+constexpr int kAuxThreads = 32 * (kWriterWarps + 1);      // writer warps + producer warp
 constexpr int kRingSlots = 16;          // compacted tiles awaiting their offset, per CTA
 constexpr uint32_t kComputeBar = 1;     // named barrier of the compute warps
 
@@ -69,11 +69,11 @@ struct BlkCtl {
     uint32_t used;                       // ring bytes consumed (block + skipped tail)
     uint32_t pad;
 };
-template <int ITEMS>
+template <int NT, int ITEMS>
 struct ScanCtl {
     InCtl in[kMaxStages];
     BlkCtl blk[kRingSlots];
-    uint32_t cnt[ITEMS * kWarps];
+    uint32_t cnt[ITEMS * NT / 32];
     uint32_t total;
     uint32_t roff;
     volatile uint32_t tail;              // ring bytes released by the writers (monotone, wraps)
@@ -102,21 +102,22 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
         d[j] = src[j];
 }
 
-template <int ITEMS, bool AGG>
-__global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_constant__ ChainProg P,
-                                                             const __grid_constant__ TileLaunch L)
+template <int NT, int ITEMS, bool AGG>
+__global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid_constant__ ChainProg P,
+                                                                                  const __grid_constant__ TileLaunch L)
 {
-    constexpr int T = kThreads * ITEMS;
+    constexpr int T = NT * ITEMS;
+    constexpr int NW = NT / 32;             // compute warps
     extern __shared__ __align__(128) unsigned char smem_raw[];
     const int S = L.stages;
     const uint32_t R = L.out_bytes;      // ring bytes (multiple of 128)
-    ScanCtl<ITEMS> *ctl = (ScanCtl<ITEMS> *)smem_raw;
-    char *stages = (char *)smem_raw + align_up(sizeof(ScanCtl<ITEMS>), 128);
+    ScanCtl<NT, ITEMS> *ctl = (ScanCtl<NT, ITEMS> *)smem_raw;
+    char *stages = (char *)smem_raw + align_up(sizeof(ScanCtl<NT, ITEMS>), 128);
     char *scratch = stages + (size_t)S * P.stage_bytes;
     char *ring = scratch + P.scratch_bytes;
     unsigned long long *part = (unsigned long long *)(ring + (AGG ? 0 : R));
     const int NA = P.nagg + 1;
-    unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * kThreads : 0);
+    unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * NT : 0);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
@@ -137,14 +138,14 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
         fence_mbar_init();
     }
     if (AGG) {
-        for (int q = tid; q < P.D * NA * kThreads; q += blockDim.x)
+        for (int q = tid; q < P.D * NA * NT; q += blockDim.x)
             part[q] = 0;
         for (int q = tid; q < P.D * NA * 2; q += blockDim.x)
             cta_acc[q] = 0;
     }
     __syncthreads();
 
-    if (warp == kWarps + kWriterWarps) {
+    if (warp == NW + kWriterWarps) {
         // ---------------- producer warp ----------------
         if (lane == 0) {
             uint32_t tx_bytes = 0;
@@ -159,7 +160,7 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                 const int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
-                    L.dbg_ts[6 * t + 0] = globaltimer();
+                    L.dbg_ts[8 * t + 0] = globaltimer();
                 if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
                     char *st = stages + (size_t)s * P.stage_bytes;
                     fence_proxy_async_smem();
@@ -180,11 +181,11 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                 }
             }
         }
-    } else if (warp >= kWarps) {
+    } else if (warp >= NW) {
         // ---------------- writer warps: look-back + compacted store ----------------
         // Writer w owns ring slots i = w (mod kWriterWarps): the look-backs and copies
         // of consecutive tiles proceed concurrently; ring bytes are released in order.
-        const int wi = warp - kWarps;
+        const int wi = warp - NW;
         if (emit) {
             for (int64_t i = wi;; i += kWriterWarps) {
                 const int j = (int)(i % kRingSlots);
@@ -194,12 +195,12 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                     break;
                 const uint32_t total = ctl->blk[j].total;
                 if ((L.dbg & 4) && lane == 0)
-                    L.dbg_ts[6 * t + 5] = globaltimer();
+                    L.dbg_ts[8 * t + 5] = globaltimer();
                 const int64_t excl = (L.dbg & 1) ? t * T
                                                   : (int64_t)lookback_warp(L.status, t, total, L.epoch, /*aggregate_published=*/true);
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[6 * t + 3] = globaltimer();
+                        L.dbg_ts[8 * t + 3] = globaltimer();
                     if (t == ntiles - 1)
                         *L.n_dev = excl + (int64_t)total;
                 }
@@ -218,7 +219,7 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                 __syncwarp();
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[6 * t + 4] = globaltimer();
+                        L.dbg_ts[8 * t + 4] = globaltimer();
                     if (i > 0)   // release ring bytes in tile order
                         mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1));
                     __threadfence_block();
@@ -238,7 +239,10 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                 s = 0;
                 fph ^= 1;
             }
-            mbar_wait(&ctl->in[s].full, fph);
+            if (L.dbg & 8)
+                mbar_wait_spin(&ctl->in[s].full, fph);
+            else
+                mbar_wait(&ctl->in[s].full, fph);
             const int64_t t = ctl->in[s].tile;
             const int j = (int)(i % kRingSlots);
             if (t >= ntiles) {
@@ -258,9 +262,9 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
             const int64_t row0 = t * T;
             const int rows = (int)min((int64_t)T, n - row0);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[6 * t + 1] = globaltimer();
+                L.dbg_ts[8 * t + 1] = globaltimer();
             if (L.dbg & 2) {   // diagnostics: stream the tiles only (TMA pipeline ceiling)
-                bar_sync(kComputeBar, kThreads);
+                bar_sync(kComputeBar, NT);
                 if (tid == 0)
                     mbar_arrive(&ctl->in[s].empty);
                 continue;
@@ -272,30 +276,32 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                     char *dst = st + P.slot[c].off;
                     const char *src = (const char *)P.in_ptr[c] + (size_t)row0 * w;
                     if (w == 4) {
-                        for (int r = tid; r < rows; r += kThreads)
+                        for (int r = tid; r < rows; r += NT)
                             ((uint32_t *)dst)[r] = ((const uint32_t *)src)[r];
                     } else if (w == 8) {
-                        for (int r = tid; r < rows; r += kThreads)
+                        for (int r = tid; r < rows; r += NT)
                             ((uint64_t *)dst)[r] = ((const uint64_t *)src)[r];
                     } else {
-                        for (int r = tid; r < rows; r += kThreads)
+                        for (int r = tid; r < rows; r += NT)
                             dst[r] = src[r];
                     }
                 }
-                bar_sync(kComputeBar, kThreads);
+                bar_sync(kComputeBar, NT);
             }
             uint32_t mask = (1u << ITEMS) - 1u;
             if (rows < T) {
                 mask = 0;
 #pragma unroll
                 for (int k = 0; k < ITEMS; k++)
-                    if (k * kThreads + tid < rows)
+                    if (k * NT + tid < rows)
                         mask |= 1u << k;
             }
-            mask = run_ops<ITEMS>(P, st, scratch, mask);
+            mask = run_ops<NT, ITEMS>(P, st, scratch, mask);
+            if ((L.dbg & 4) && tid == 0)
+                L.dbg_ts[8 * t + 6] = globaltimer();
             if (AGG) {
-                agg_tile<ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
-                bar_sync(kComputeBar, kThreads);
+                agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
+                bar_sync(kComputeBar, NT);
                 if (tid == 0)
                     mbar_arrive(&ctl->in[s].empty);
                 continue;
@@ -305,11 +311,17 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
             for (int k = 0; k < ITEMS; k++) {
                 bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
                 if (lane == 0)
-                    ctl->cnt[k * kWarps + warp] = __popc(bal[k]);
+                    ctl->cnt[k * NW + warp] = __popc(bal[k]);
             }
-            bar_sync(kComputeBar, kThreads);
-            if (warp == 0) {
-                constexpr int NV = ITEMS * kWarps;
+            bar_sync(kComputeBar, NT);
+            if ((L.dbg & 4) && tid == 0)
+                L.dbg_ts[8 * t + 7] = globaltimer();
+            // every warp scans the ITEMS x NW survivor counts itself (no wait on a
+            // single scanning warp); warp 0 also publishes the aggregate and reserves ring bytes
+            uint32_t pre[ITEMS];
+            uint32_t total;
+            {
+                constexpr int NV = ITEMS * NW;
                 constexpr int PER = (NV + 31) / 32;
                 uint32_t v[PER];
                 uint32_t sum = 0;
@@ -326,21 +338,28 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                     if (lane >= o)
                         inc += y;
                 }
-                uint32_t run = inc - sum;
+                total = __shfl_sync(0xffffffffu, inc, 31);
+                // exclusive prefix of entry idx = (inc - sum) of its owner lane + preceding v's
+                const uint32_t base = inc - sum;
 #pragma unroll
-                for (int qq = 0; qq < PER; qq++) {
-                    const int idx = lane * PER + qq;
-                    if (idx < NV)
-                        ctl->cnt[idx] = run;
-                    run += v[qq];
+                for (int k = 0; k < ITEMS; k++) {
+                    const int idx = k * NW + warp;
+                    const int owner = idx / PER, off = idx % PER;
+                    uint32_t part = 0;
+#pragma unroll
+                    for (int qq = 0; qq < PER; qq++)
+                        if (qq < off) part += v[qq];
+                    const uint32_t b0 = __shfl_sync(0xffffffffu, base + part, owner);
+                    pre[k] = b0;
                 }
-                const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+            }
+            if (warp == 0) {
                 if (lane == 31) {
                     // publish the tile aggregate before anything can block this CTA
                     if (t > 0 && !(L.dbg & 1))
                         st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
                     if (L.dbg & 4)
-                        L.dbg_ts[6 * t + 2] = globaltimer();
+                        L.dbg_ts[8 * t + 2] = globaltimer();
                 }
                 if (lane == 0) {
                     // reserve ring bytes for the compacted tile (blocks never wrap)
@@ -369,18 +388,16 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                     }
                     ctl->head = head + used;
                     ctl->roff = pos;
-                    ctl->total = total;
                     ctl->blk[j].used = used;
                 }
             }
-            bar_sync(kComputeBar, kThreads);
-            const uint32_t total = ctl->total;
-            char *blk = ring + ctl->roff;
             const uint32_t lt = lanemask_lt();
             uint32_t pos[ITEMS];
 #pragma unroll
             for (int k = 0; k < ITEMS; k++)
-                pos[k] = ctl->cnt[k * kWarps + warp] + __popc(bal[k] & lt);
+                pos[k] = pre[k] + __popc(bal[k] & lt);
+            bar_sync(kComputeBar, NT);      // ring position known
+            char *blk = ring + ctl->roff;
             uint32_t coff = 0;
             for (int c = 0; c < P.nout; c++) {
                 const int w = P.out_w[c];
@@ -391,21 +408,21 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
                 case 1:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint8_t *)dst)[pos[k]] = ((const uint8_t *)src)[k * kThreads + tid];
+                        if ((mask >> k) & 1u) ((uint8_t *)dst)[pos[k]] = ((const uint8_t *)src)[k * NT + tid];
                     break;
                 case 4:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint32_t *)dst)[pos[k]] = ((const uint32_t *)src)[k * kThreads + tid];
+                        if ((mask >> k) & 1u) ((uint32_t *)dst)[pos[k]] = ((const uint32_t *)src)[k * NT + tid];
                     break;
                 default:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint64_t *)dst)[pos[k]] = ((const uint64_t *)src)[k * kThreads + tid];
+                        if ((mask >> k) & 1u) ((uint64_t *)dst)[pos[k]] = ((const uint64_t *)src)[k * NT + tid];
                     break;
                 }
             }
-            bar_sync(kComputeBar, kThreads);
+            bar_sync(kComputeBar, NT);
             if (tid == 0) {
                 mbar_arrive(&ctl->in[s].empty);          // input tile and scratch are free
                 ctl->blk[j].tile = t;
@@ -415,7 +432,7 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_chain(const __grid_consta
             }
         }
         if (AGG)
-            agg_flush(P, part, cta_acc);
+            agg_flush<NT>(P, part, cta_acc);
     }
     __syncthreads();
     if (AGG) {
@@ -857,7 +874,7 @@ __global__ void __launch_bounds__(kThreads) k_join_expand(const __grid_constant_
         for (int k = 0; k < kJoinItems; k++)
             if (k * kThreads + tid < rows)
                 mask |= 1u << k;
-        mask = run_ops<kJoinItems>(P, tilebuf, scratch, mask);
+        mask = run_ops<kThreads, kJoinItems>(P, tilebuf, scratch, mask);
         emit_tile<kJoinItems>(P, tilebuf, scratch, mask, t, ntiles, L, &ctl->es);
         __syncthreads();
     }
@@ -869,7 +886,7 @@ __global__ void __launch_bounds__(kThreads) k_join_expand(const __grid_constant_
 // ===========================================================================
 // Host launchers
 // ===========================================================================
-size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<kScanItems>), 128); }   // >= ITEMS 4
+size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<256, 8>), 128); }   // >= every (NT, ITEMS) with NT*ITEMS <= 2048
 size_t join_ctl_bytes() { return align_up(sizeof(JoinCtl), 128); }
 size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
 int scan_tile() { return kThreads * kScanItems; }
@@ -890,30 +907,36 @@ static int occ(F f, size_t smem, int threads = kThreads)
     return n;
 }
 
-int chain_occupancy(int which, int items, size_t smem)
+int chain_occupancy(int which, int nt, int items, size_t smem)
 {
     switch (which) {
-    case 0: return items == 4 ? occ(k_scan_chain<4, false>, smem, kScanThreads) : occ(k_scan_chain<8, false>, smem, kScanThreads);
-    case 1: return items == 4 ? occ(k_scan_chain<4, true>, smem, kScanThreads) : occ(k_scan_chain<8, true>, smem, kScanThreads);
+    case 0:
+        if (nt == 512) return occ(k_scan_chain<512, 4, false>, smem, 512 + kAuxThreads);
+        return items == 4 ? occ(k_scan_chain<256, 4, false>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, false>, smem, 256 + kAuxThreads);
+    case 1: return items == 4 ? occ(k_scan_chain<256, 4, true>, smem, 256 + kAuxThreads)
+                              : occ(k_scan_chain<256, 8, true>, smem, 256 + kAuxThreads);
     case 2: return occ(k_join_expand, smem);
     default: return occ(k_join_runs<uint64_t>, smem);
     }
 }
 
-template <int ITEMS, bool AGG>
+template <int NT, int ITEMS, bool AGG>
 static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
-    cudaFuncSetAttribute(k_scan_chain<ITEMS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_chain<ITEMS, AGG><<<grid, kScanThreads, smem, s>>>(P, L);
+    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_scan_chain<NT, ITEMS, AGG><<<grid, NT + kAuxThreads, smem, s>>>(P, L);
     return cudaGetLastError();
 }
 
-cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int items, size_t smem, int grid,
-                              cudaStream_t s)
+cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem,
+                              int grid, cudaStream_t s)
 {
-    if (items == 4)
-        return agg ? sc<4, true>(P, L, smem, grid, s) : sc<4, false>(P, L, smem, grid, s);
-    return agg ? sc<8, true>(P, L, smem, grid, s) : sc<8, false>(P, L, smem, grid, s);
+    if (agg)
+        return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
+    if (nt == 512)
+        return sc<512, 4, false>(P, L, smem, grid, s);
+    return items == 4 ? sc<256, 4, false>(P, L, smem, grid, s) : sc<256, 8, false>(P, L, smem, grid, s);
 }
 
 cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s)

@@ -90,6 +90,8 @@ struct Lowered {
     ChainProg P;
     std::vector<int> in_src;      // input slot i <- source column in_src[i]
     int items = 8, stages = 2, ctas = 1;
+    int tile = 2048;              // rows per tile
+    int nt = 256;                 // compute threads per CTA
     int ring = 0;                 // scan kernel: output ring entries
     uint32_t out_bytes = 0;       // bytes of one output ring entry
     std::vector<uint32_t> out_off;
@@ -742,11 +744,12 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         const int T = join_expand_tile();
         layout(T);
         L.items = kJoinItems;
+        L.tile = T;
         L.stages = 1;
         L.smem = join_ctl_bytes() + join_run_cache_bytes() + P.stage_bytes + P.scratch_bytes;
         if (L.smem > kSmemLimit)
             raise(RW_E_UNSUPPORTED, "join group exceeds the shared-memory budget");
-        L.ctas = std::max(1, chain_occupancy(2, kJoinItems, L.smem));
+        L.ctas = std::max(1, chain_occupancy(2, kThreads, kJoinItems, L.smem));
         return;
     }
     // Scan kernel: S input stages (TMA ring), one scratch tile for computed
@@ -755,8 +758,17 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     const int want_stages = p->o.stages > 0 ? std::min(p->o.stages, kMaxStages) : 0;
     const size_t want_ring = p->o.reserved[0] > 0 ? (size_t)p->o.reserved[0] * 1024 : 0;
     bool ok = false;
-    for (int items : {8, 4}) {
-        const int T = kThreads * items;
+    // kernel variants (compute threads NT x rows per thread): 256 x 8 (2048-row tiles),
+    // 256 x 4 (1024-row tiles, wide rows); 512 x 4 on request (opts.reserved[4] == 2)
+    struct Var { int nt, items; };
+    std::vector<Var> vars;
+    if (!L.agg && p->o.reserved[4] == 2) vars.push_back({512, 4});
+    vars.push_back({256, 8});
+    vars.push_back({256, 4});
+    for (size_t ii = 0; ii < vars.size(); ii++) {
+        const int items = vars[ii].items;
+        const int nt = vars[ii].nt;
+        const int T = nt * items;
         layout(T);
         size_t W = 0;                       // largest compacted tile (every row survives)
         for (int c = 0; c < P.nout; c++)
@@ -781,9 +793,11 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 }
                 const size_t smem = base + (size_t)S * P.stage_bytes + Rb;
                 if (smem > per_cta) continue;
-                int occ = chain_occupancy(L.agg ? 1 : 0, items, smem);
+                int occ = chain_occupancy(L.agg ? 1 : 0, nt, items, smem);
                 if (occ < occ_t) continue;
                 L.items = items;
+                L.nt = nt;
+                L.tile = T;
                 L.stages = S;
                 L.ring = 0;
                 L.out_bytes = (uint32_t)Rb;
@@ -797,7 +811,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     }
     if (!ok)
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
-    layout(kThreads * L.items);
+    layout(L.tile);
 }
 
 // ---------------------------------------------------------------------------
@@ -916,7 +930,7 @@ void run_group(ExecCtx &X, int gi)
         Rel src = rel_of(X, g.source);
         Lowered L;
         lower(p, g, src.types, L);
-        const int T = kThreads * L.items;
+        const int T = L.tile;
         int64_t cap_out = L.agg ? p->nodes[g.agg].D : src.cap;
         make_output(X, gi, outn.types, cap_out, o, outp, capacity, n_dev);
         bool aligned = true;
@@ -946,7 +960,7 @@ void run_group(ExecCtx &X, int gi)
             unsigned long long *acc = agg_buffer(p, g.agg, words);
             TL.agg_acc = acc;
             TL.n_dev = n_dev;
-            cuda_check(scan_chain_launch(L.P, TL, true, L.items, L.smem, grid, p->stream), "k_scan_chain<agg>");
+            cuda_check(scan_chain_launch(L.P, TL, true, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain<agg>");
             p->launches++;
             L.F.acc = acc;
             L.F.acc_w = acc;
@@ -962,7 +976,7 @@ void run_group(ExecCtx &X, int gi)
                 L.P.out_ptr[c] = outp[c];
             L.P.out_capacity = capacity;
             TL.n_dev = n_dev;
-            cuda_check(scan_chain_launch(L.P, TL, false, L.items, L.smem, grid, p->stream), "k_scan_chain");
+            cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
             p->launches++;
         }
     } else {
@@ -994,7 +1008,7 @@ void run_group(ExecCtx &X, int gi)
         J.ctrs = p->ctrs;
         J.totals = p->jtot;
         const size_t smem1 = join_runs_smem(kt);
-        const int occ1 = std::max(1, chain_occupancy(3, 8, smem1));
+        const int occ1 = std::max(1, chain_occupancy(3, kThreads, 8, smem1));
         const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
         cuda_check(join_runs_launch(J, kt, smem1, grid1, p->stream), "k_join_runs");
         p->launches++;
@@ -1161,7 +1175,7 @@ std::string explain(rw_plan *p, int out_node)
             Lowered L;
             std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
             lower(p, g, st, L);
-            s << " | tile " << kThreads * L.items << " rows, stages " << L.stages << ", out ring " << L.out_bytes << " B"
+            s << " | tile " << L.tile << " rows (" << L.items << "/thread), stages " << L.stages << ", out ring " << L.out_bytes << " B"
               << ", smem " << L.smem
               << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
               << L.P.nops;
