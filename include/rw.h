@@ -198,13 +198,27 @@ const char *rw_last_error(void);
 rw_status rw_split_by_splitters(const void *keys_dev, int64_t n, int32_t key_type, const void *splitters_dev,
                                 int32_t nsplit, int64_t *bounds_dev, void *cuda_stream);
 
-/* Merge nrun key-sorted runs (concatenated in `cols`, run r = rows [run_off[r],
- * run_off[r+1]) of every column, run_off host array of nrun+1 entries) into one
- * sequence sorted by (key column 0, then run index, then row) written to out_cols.
- * Equal keys keep run order, so merging per-rank slices in rank order reproduces
- * a stable global order. */
+/* Merge nrun runs, each sorted lexicographically over all ncols columns (<= 8), that
+ * lie concatenated in `cols` (run r = rows [run_off[r], run_off[r+1]) of every column;
+ * run_off is a HOST array of nrun+1 entries) into one sequence sorted the same way,
+ * written to out_cols (device, run_off[nrun] - run_off[0] rows).  Equal tuples keep run
+ * order.  Pairwise merge-path tree (ceil(log2 nrun) passes); temporaries come from
+ * cudaMallocAsync on the given stream. */
 rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t ncols, const int64_t *run_off,
                         int32_t nrun, void *const *out_cols, void *cuda_stream);
+
+/* Aggregate combine across row shards: an aggregate result is
+ * exported as D * L dense int64 words (per group: a presence word, then per aggregate
+ * 1 word for COUNT or four 32-bit limbs of the 128-bit two's complement SUM), so that a
+ * plain int64 SUM all-reduce over <= 2^31 ranks is exact; import recombines the limbs
+ * (sum_k limb_k * 2^32k mod 2^128) and emits the groups present on any rank, ascending.
+ * rw_plan_agg_limbs gives D * L.  export: cols = the node's local result columns on
+ * device, row count from n_dev (device) or n_host; limbs_dev is overwritten.  Both are
+ * enqueued on the plan's stream; import synchronises when out->n_dev is NULL. */
+rw_status rw_plan_agg_limbs(const rw_plan *plan, int32_t agg_node, int64_t *nlimbs);
+rw_status rw_plan_agg_export(rw_plan *plan, int32_t agg_node, const void *const *cols, const int64_t *n_dev,
+                             int64_t n_host, int64_t *limbs_dev);
+rw_status rw_plan_agg_import(rw_plan *plan, int32_t agg_node, const int64_t *limbs_dev, rw_relation_out *out);
 
 #ifdef __cplusplus
 }

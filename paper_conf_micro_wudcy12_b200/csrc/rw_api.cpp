@@ -12,6 +12,7 @@
 #include <string>
 #include <vector>
 
+#include "dist_kernels.h"
 #include "kernels.h"
 #include "plan.h"
 
@@ -1625,17 +1626,172 @@ int64_t rw_plan_last_launches(const rw_plan *p) { return p ? p->launches : -1; }
 rw_status rw_split_by_splitters(const void *keys_dev, int64_t n, int32_t key_type, const void *splitters_dev,
                                 int32_t nsplit, int64_t *bounds_dev, void *cuda_stream)
 {
-    g_err = "rw_split_by_splitters: not built yet";
-    (void)keys_dev; (void)n; (void)key_type; (void)splitters_dev; (void)nsplit; (void)bounds_dev; (void)cuda_stream;
-    return RW_E_UNSUPPORTED;
+    RW_TRY
+    if (n < 0 || nsplit < 0 || (n > 0 && !keys_dev) || (nsplit > 0 && (!splitters_dev || !bounds_dev)))
+        raise(RW_E_ARG, "bad split arguments");
+    check_type(key_type);
+    cuda_check(split_bounds_launch(keys_dev, n, key_type, splitters_dev, nsplit, bounds_dev,
+                                   (cudaStream_t)cuda_stream),
+               "k_split_bounds");
+    return RW_OK;
+    RW_CATCH
 }
 
 rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t ncols, const int64_t *run_off,
                         int32_t nrun, void *const *out_cols, void *cuda_stream)
 {
-    g_err = "rw_merge_runs: not built yet";
-    (void)cols; (void)types; (void)ncols; (void)run_off; (void)nrun; (void)out_cols; (void)cuda_stream;
-    return RW_E_UNSUPPORTED;
+    RW_TRY
+    if (ncols < 1 || ncols > kMaxMergeCols || nrun < 0 || !cols || !types || !run_off || !out_cols)
+        raise(RW_E_ARG, "bad merge arguments");
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    MergeTypes T{};
+    for (int c = 0; c < ncols; c++) {
+        check_type(types[c]);
+        T.t[c] = (uint8_t)types[c];
+    }
+    struct Run {
+        MergeCols c;
+        int64_t n;
+        bool temp;
+    };
+    std::vector<Run> runs;
+    for (int r = 0; r < nrun; r++) {
+        if (run_off[r + 1] < run_off[r])
+            raise(RW_E_ARG, "run offsets must be non-decreasing");
+        Run x{};
+        x.n = run_off[r + 1] - run_off[r];
+        for (int c = 0; c < ncols; c++)
+            x.c.col[c] = (const char *)cols[c] + (size_t)run_off[r] * type_width(types[c]);
+        runs.push_back(x);
+    }
+    const int64_t total = nrun ? run_off[nrun] - run_off[0] : 0;
+    std::vector<void *> temps;
+    auto release = [&]() {
+        for (void *t : temps)
+            cudaFreeAsync(t, st);
+    };
+    try {
+        if (runs.size() <= 1) {
+            for (int c = 0; c < ncols && total > 0; c++)
+                cuda_check(cudaMemcpyAsync(out_cols[c], runs[0].c.col[c], (size_t)total * type_width(types[c]),
+                                           cudaMemcpyDeviceToDevice, st),
+                           "copy run");
+        }
+        // pairwise merge tree; the last round writes the caller's columns
+        while (runs.size() > 1) {
+            std::vector<Run> next;
+            const bool last = runs.size() == 2;
+            for (size_t r = 0; r + 1 < runs.size(); r += 2) {
+                Run m{};
+                m.n = runs[r].n + runs[r + 1].n;
+                MergeOut O{};
+                for (int c = 0; c < ncols; c++) {
+                    if (last) {
+                        O.col[c] = out_cols[c];
+                    } else {
+                        void *p = nullptr;
+                        cuda_check(cudaMallocAsync(&p, (size_t)std::max<int64_t>(m.n, 1) * type_width(types[c]), st),
+                                   "cudaMallocAsync");
+                        temps.push_back(p);
+                        O.col[c] = p;
+                    }
+                    m.c.col[c] = O.col[c];
+                }
+                cuda_check(merge2_launch(runs[r].c, runs[r].n, runs[r + 1].c, runs[r + 1].n, O, ncols, T, st),
+                           "k_merge2");
+                next.push_back(m);
+            }
+            if (runs.size() % 2)
+                next.push_back(runs.back());
+            runs.swap(next);
+        }
+    } catch (...) {
+        release();
+        throw;
+    }
+    release();
+    return RW_OK;
+    RW_CATCH
+}
+
+static AggXfer agg_xfer(const rw_plan *p, int32_t agg_node)
+{
+    const Node &a = node_at(p, agg_node);
+    if (a.kind != N_AGG)
+        raise(RW_E_ARG, "node is not an aggregate");
+    AggXfer X{};
+    X.ngc = (int)a.gcols.size();
+    for (int c = 0; c < X.ngc; c++) {
+        X.gdomain[c] = a.gdomain[c];
+        X.gtype[c] = (uint8_t)a.types[c];
+    }
+    X.nreq = (int)a.aggs.size();
+    int L = 1;
+    for (int q = 0; q < X.nreq; q++) {
+        X.is_sum[q] = a.aggs[q].op == RW_SUM;
+        L += X.is_sum[q] ? 4 : 1;
+    }
+    X.D = a.D;
+    X.L = L;
+    return X;
+}
+
+rw_status rw_plan_agg_limbs(const rw_plan *p, int32_t agg_node, int64_t *nlimbs)
+{
+    RW_TRY
+    if (!p || !nlimbs)
+        raise(RW_E_ARG, "null argument");
+    AggXfer X = agg_xfer(p, agg_node);
+    *nlimbs = (int64_t)X.D * X.L;
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_agg_export(rw_plan *p, int32_t agg_node, const void *const *cols, const int64_t *n_dev,
+                             int64_t n_host, int64_t *limbs_dev)
+{
+    RW_TRY
+    if (!p || !cols || !limbs_dev)
+        raise(RW_E_ARG, "null argument");
+    AggXfer X = agg_xfer(p, agg_node);
+    const int ncols = (int)p->nodes[agg_node].types.size();
+    for (int c = 0; c < ncols; c++)
+        X.col[c] = cols[c];
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    cuda_check(cudaMemsetAsync(limbs_dev, 0, (size_t)X.D * X.L * 8, p->stream), "memset limbs");
+    cuda_check(agg_export_launch(X, n_dev, n_host, limbs_dev, p->stream), "k_agg_export");
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_agg_import(rw_plan *p, int32_t agg_node, const int64_t *limbs_dev, rw_relation_out *out)
+{
+    RW_TRY
+    if (!p || !limbs_dev || !out || !out->cols)
+        raise(RW_E_ARG, "null argument");
+    AggXfer X = agg_xfer(p, agg_node);
+    const int ncols = (int)p->nodes[agg_node].types.size();
+    OutPtrs O{};
+    for (int c = 0; c < ncols; c++)
+        O.col[c] = out->cols[c];
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    int64_t *nd = out->n_dev ? out->n_dev : p->cnt;
+    if (!nd) {
+        p->cnt_cap = 8;
+        p->cnt = (int64_t *)dev_alloc(p, 64);
+        nd = p->cnt;
+    }
+    cuda_check(agg_import_launch(X, limbs_dev, O, out->capacity, nd, p->stream), "k_agg_import");
+    out->n = -1;
+    if (!out->n_dev) {
+        cuda_check(cudaMemcpyAsync(p->jtot_host + 2, nd, 8, cudaMemcpyDeviceToHost, p->stream), "copy n");
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+        out->n = p->jtot_host[2];
+        if (out->n > out->capacity)
+            raise(RW_E_CAPACITY, "aggregate output needs " + std::to_string(out->n) + " rows");
+    }
+    return RW_OK;
+    RW_CATCH
 }
 
 }  // extern "C"

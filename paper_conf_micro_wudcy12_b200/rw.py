@@ -62,7 +62,8 @@ class rw_relation_out(ctypes.Structure):
 EXPORTS = ["rw_plan_create", "rw_plan_destroy", "rw_plan_add_input", "rw_plan_add_select",
            "rw_plan_add_project", "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema",
            "rw_plan_execute", "rw_plan_execute_host", "rw_plan_explain", "rw_plan_last_launches",
-           "rw_status_str", "rw_last_error", "rw_split_by_splitters", "rw_merge_runs"]
+           "rw_status_str", "rw_last_error", "rw_split_by_splitters", "rw_merge_runs",
+           "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]
 
 _lib = None
 
@@ -96,9 +97,13 @@ def lib():
     L.rw_last_error.restype = ctypes.c_char_p
     L.rw_split_by_splitters.argtypes = [vp, i64, i32, vp, i32, vp, vp]
     L.rw_merge_runs.argtypes = [P(vp), P(i32), i32, P(i64), i32, P(vp), vp]
+    L.rw_plan_agg_limbs.argtypes = [vp, i32, P(i64)]
+    L.rw_plan_agg_export.argtypes = [vp, i32, P(vp), vp, i64, vp]
+    L.rw_plan_agg_import.argtypes = [vp, i32, vp, P(rw_relation_out)]
     for f in ["rw_plan_create", "rw_plan_add_input", "rw_plan_add_select", "rw_plan_add_project",
               "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema", "rw_plan_execute",
-              "rw_plan_execute_host", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs"]:
+              "rw_plan_execute_host", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs",
+              "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]:
         getattr(L, f).restype = i32
     _lib = L
     return L
@@ -264,6 +269,29 @@ class Plan:
         buf = ctypes.create_string_buffer(1 << 16)
         check(lib().rw_plan_explain(self.h, out_node, buf, len(buf)))
         return buf.value.decode()
+
+    # -- aggregate combine across row shards -------------------------------
+    def agg_limbs(self, node: int) -> int:
+        n = ctypes.c_int64()
+        check(lib().rw_plan_agg_limbs(self.h, node, ctypes.byref(n)))
+        return n.value
+
+    def agg_export(self, node: int, cols, n_dev=None, n_host: int = 0, limbs=None):
+        """Local aggregate result -> dense int64 limbs (device tensor, returned)."""
+        import torch
+        if limbs is None:
+            limbs = torch.empty(self.agg_limbs(node), dtype=torch.int64, device=f"cuda:{self.device}")
+        c = (ctypes.c_void_p * len(cols))(*[_ptr(x) for x in cols])
+        check(lib().rw_plan_agg_export(self.h, node, c, ctypes.c_void_p(_ptr(n_dev)) if n_dev is not None else None,
+                                       int(n_host), ctypes.c_void_p(_ptr(limbs))))
+        return limbs
+
+    def agg_import(self, node: int, limbs, out_cols, capacity: int, n_dev=None):
+        oc = (ctypes.c_void_p * max(1, len(out_cols)))(*[_ptr(x) for x in out_cols])
+        out = rw_relation_out(ctypes.cast(oc, ctypes.POINTER(ctypes.c_void_p)), int(capacity),
+                              ctypes.c_void_p(_ptr(n_dev)) if n_dev is not None else None, -1)
+        check(lib().rw_plan_agg_import(self.h, node, ctypes.c_void_p(_ptr(limbs)), ctypes.byref(out)))
+        return None if n_dev is not None else out.n
 
     def last_launches(self) -> int:
         return int(lib().rw_plan_last_launches(self.h))
