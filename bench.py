@@ -34,6 +34,7 @@ CONFIGS = {
     "c2": dict(name="C2: SELECT->PROJECT->SELECT over 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
     "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
+    "c5": dict(name="C5: JOIN->JOIN->SELECT over three relations, 2^27 rows each per GPU (2^30 at 8 GPUs), key-range sharded", rows=1 << 27),
 }
 
 
@@ -72,6 +73,9 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
         return workloads.c3_spec(), workloads.c3_inputs(rows, device=device)
     if cfg == "c4":
         return workloads.c4_spec(), workloads.c4_inputs(rows, start, device)
+    if cfg == "c5":
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        return workloads.c5_spec(), workloads.c5_inputs(rows, key_space=rows * world, start=start, device=device)
     raise ValueError(cfg)
 
 
@@ -177,7 +181,7 @@ def run_reference(args):
         return 0
     cfg = args.config
     rows = args.rows or CONFIGS[cfg]["rows"]
-    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23}[cfg]
+    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21}[cfg]
     import oracle
     oracle.build()
     vals = []
@@ -224,6 +228,8 @@ def main():
     in_bytes = workloads.input_bytes(spec, nrows)
     stream = torch.cuda.current_stream()
 
+    dtn = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
+
     def make(fuse):
         plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse, stages=args.stages,
                                    ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg)
@@ -231,32 +237,71 @@ def main():
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
         if cfg == "c3":
             cap = 400_000_000 if rows == workloads.C3_ROWS else 8 * rows + 1024
-        dt = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
-        outs = [torch.empty(cap, dtype=dt[t], device=dev) for t in out_types]
+        if cfg == "c5":
+            cap = 2 * max(nrows.values()) + 4096
+        outs = [torch.empty(cap, dtype=dtn[t], device=dev) for t in out_types]
         return plan, ids, outs, cap, out_types
 
     inputs = [(nrows[k], ins[k]) for k in spec["inputs"]]
     n_dev = torch.zeros(1, dtype=torch.int64, device=dev)
+    from paper_conf_micro_wudcy12_b200 import dist as rdist
 
-    def timed(plan, ids, outs, cap, steps, warmup):
+    def make_step(plan, ids, outs, cap):
+        node = ids[spec["out"]]
+        if cfg == "c4" and world > 1:
+            # local fused Q1, exact limb export, one NCCL all-reduce, import
+            limbs = torch.empty(plan.agg_limbs(node), dtype=torch.int64, device=dev)
+            loc = [torch.empty(6, dtype=o.dtype, device=dev) for o in outs]
+            loc_n = torch.zeros(1, dtype=torch.int64, device=dev)
+
+            def step():
+                plan.execute(inputs, node, loc, 6, n_dev=loc_n)
+                plan.agg_export(node, loc, n_dev=loc_n, limbs=limbs)
+                pg.all_reduce(limbs, op=pg.ReduceOp.SUM)
+                plan.agg_import(node, limbs, outs, cap, n_dev=n_dev)
+                return plan.last_launches() + 2
+            return step
+        if cfg == "c5" and world > 1:
+            schema = {k: v["types"] for k, v in spec["inputs"].items()}
+            backend = rdist.GpuBackend(local)
+
+            def step():
+                mine = rdist.exchange_all(backend, ins, schema, world)
+                loc_in = [(int(mine[k][0].numel()), mine[k]) for k in spec["inputs"]]
+                plan.execute(loc_in, node, outs, cap, n_dev=n_dev)
+                return plan.last_launches() + 3 * (2 + (world - 1).bit_length())
+            return step
+
+        def step():
+            plan.execute(inputs, node, outs, cap, n_dev=n_dev)
+            return plan.last_launches()
+        return step
+
+    # inputs smaller than 4x L2 (C1): flush L2 between timed steps by writing 512 MB,
+    # outside each step's event pair
+    flush_buf = torch.empty(512 << 20, dtype=torch.uint8, device=dev) if in_bytes < (512 << 20) else None
+
+    def timed(step, steps, warmup):
         for _ in range(warmup):
-            plan.execute(inputs, ids[spec["out"]], outs, cap, n_dev=n_dev)
+            step()
         torch.cuda.synchronize()
         if pg:
             pg.barrier()
         torch.cuda.synchronize()
-        evs = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1)]
+        ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
         launches = 0
         sampler = ClockSampler(local)
         with sampler:
-            evs[0].record(stream)
             for i in range(steps):
-                plan.execute(inputs, ids[spec["out"]], outs, cap, n_dev=n_dev)
-                launches += plan.last_launches()
-                evs[i + 1].record(stream)
+                if flush_buf is not None:
+                    flush_buf.zero_()
+                ev0[i].record(stream)
+                launches += step()
+                ev1[i].record(stream)
             torch.cuda.synchronize()
-        per = [evs[i].elapsed_time(evs[i + 1]) for i in range(steps)]
-        total_ms = evs[0].elapsed_time(evs[-1])
+        per = [ev0[i].elapsed_time(ev1[i]) for i in range(steps)]
+        total_ms = sum(per)
         if pg:
             t = torch.tensor([total_ms], device=dev)
             pg.all_reduce(t, op=pg.ReduceOp.MAX)
@@ -264,29 +309,34 @@ def main():
         return total_ms, per, launches, sampler.result()
 
     plan, ids, outs, cap, out_types = make(True)
-    total_ms, per, launches, clocks = timed(plan, ids, outs, cap, args.steps, args.warmup)
+    total_ms, per, launches, clocks = timed(make_step(plan, ids, outs, cap), args.steps, args.warmup)
     n_out = int(n_dev.item())
     ms_step = total_ms / args.steps
     value = n_in * world / (total_ms / 1e3 / args.steps)
 
-    # roofline of the dominant kernel (the fused chain kernel is the whole step for C1/C2;
-    # for C4 the finalize kernel is ~µs; for C3 the expansion kernel dominates)
+    # roofline of the dominant kernel.  C1/C2: the fused k_scan_chain is the whole step;
+    # C4: k_scan_chain<agg> (k_agg_finalize is a 1-CTA epilogue of a few us); C3/C5: the
+    # join pair (k_join_runs + k_join_expand), algorithmic bytes = inputs + output.
     out_w = sum(W[t] for t in out_types)
     alg_bytes = in_bytes + n_out * out_w
     peak, peak_src = measured_peak()
     kern_ms = statistics.mean(per)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    kname = {"c3": "k_join_runs + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand"}.get(cfg, "k_scan_chain")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": ncu_traffic(cfg), "kernel": "k_scan_chain" if cfg != "c3" else "join (k_join_runs+k_join_expand)",
+                "traffic": ncu_traffic(cfg), "kernel": kname,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
-                "note": "achieved = (input bytes + compacted output bytes) / CUDA-event time per step"}
+                "note": "achieved = (input bytes + compacted output bytes) / CUDA-event time per step; "
+                        "peak = measured copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"}
 
+    par = {"c5": f"key-range shard x{world} (all_to_all)", "c4": f"row-shard x{world} + limb all-reduce"}
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else "i32",
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5") else "i32"),
             "data": "synthetic (rwgen seeded SplitMix64 generators, generated on device)",
             "config": {"workload": CONFIGS[cfg]["name"], "rows_per_gpu": nrows, "output_rows_per_gpu": n_out,
-                       "parallelism": f"row-shard x{world}", "l2": "inputs larger than L2 (no flush needed)",
+                       "parallelism": par.get(cfg, f"row-shard x{world}"),
+                       "l2": "inputs larger than L2 (no flush needed)" if in_bytes > (1 << 28) else "L2 flushed before every step",
                        "fused": True},
             "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
 
@@ -294,11 +344,12 @@ def main():
         del outs
         torch.cuda.empty_cache()
         uplan, uids, uouts, ucap, _ = make(False)
-        ut, uper, ul, _ = timed(uplan, uids, uouts, ucap, max(3, args.steps // 4), 2)
-        uv = n_in * world / (ut / 1e3 / max(3, args.steps // 4))
-        line["unfused"] = {"value": uv, "ms_per_step": ut / max(3, args.steps // 4), "gpu_launches_per_step":
-                           ul / max(3, args.steps // 4), "speedup_fused_vs_unfused": value / uv,
-                           "roofline_frac_same_numerator": alg_bytes / (ut / max(3, args.steps // 4) / 1e3) / 1e9 / peak}
+        us = max(3, args.steps // 4)
+        ut, uper, ul, _ = timed(make_step(uplan, uids, uouts, ucap), us, 2)
+        uv = n_in * world / (ut / 1e3 / us)
+        line["unfused"] = {"value": uv, "ms_per_step": ut / us, "gpu_launches_per_step": ul / us,
+                           "speedup_fused_vs_unfused": value / uv,
+                           "roofline_frac_same_numerator": alg_bytes / (ut / us / 1e3) / 1e9 / peak}
         del uouts, uplan
         torch.cuda.empty_cache()
 
@@ -332,7 +383,7 @@ def main():
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:
-        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24}[cfg]
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22}[cfg]
         v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
         line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
                                 "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}
