@@ -402,10 +402,12 @@ __device__ inline void agg_flush(const ChainProg &P, unsigned long long *part, u
     }
 }
 
+// Per-row reference path (used when the partials must be flushed more often than
+// every ITEMS rows, i.e. without declared value bounds).
 template <int NT, int ITEMS>
-__device__ inline void agg_tile(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
-                                unsigned long long *part, unsigned long long *cta_acc, int64_t &since_flush,
-                                int32_t *err)
+__device__ inline void agg_tile_rowwise(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
+                                        unsigned long long *part, unsigned long long *cta_acc, int64_t &since_flush,
+                                        int32_t *err)
 {
     const int tid = threadIdx.x;
     const int NA = P.nagg + 1;
@@ -435,6 +437,117 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
             agg_flush<NT>(P, part, cta_acc);
             since_flush = 0;
         }
+    }
+}
+
+constexpr int kAggUnroll = 8;
+
+// Tile-wise aggregate terminal: group codes of the thread's ITEMS rows computed
+// column by column (type switch hoisted out of the row loop), then each aggregate
+// column added into the thread-private partials; the aggregate loop is unrolled so
+// the independent read-modify-write chains of different aggregates overlap.
+template <int NT, int ITEMS>
+__device__ inline void agg_tile(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
+                                unsigned long long *part, unsigned long long *cta_acc, int64_t &since_flush,
+                                int32_t *err)
+{
+    if (P.flush_rows < ITEMS || P.nagg > kAggUnroll) {
+        agg_tile_rowwise<NT, ITEMS>(P, stage, scratch, mask, part, cta_acc, since_flush, err);
+        return;
+    }
+    const int tid = threadIdx.x;
+    const int NA = P.nagg + 1;
+    uint32_t g[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++)
+        g[k] = 0;
+    uint32_t ok = mask;
+    for (int c = 0; c < P.ngc; c++) {
+        const char *b = loc_ptr(P.g_loc[c], stage, scratch);
+        const uint32_t dom = (uint32_t)P.gdomain[c];
+        switch (P.g_type[c]) {
+        case T_U8:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint8_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        case T_I32:
+        case T_U32:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint32_t *)b)[k * NT + tid];   // negative i32 -> huge
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        default:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint64_t v = ((const uint64_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + (uint32_t)v;
+            }
+            break;
+        }
+    }
+    if (ok != mask)
+        atomicAdd(err, __popc(mask & ~ok));
+    const int rows = __popc(ok);
+    if (since_flush + rows > P.flush_rows) {
+        agg_flush<NT>(P, part, cta_acc);
+        since_flush = 0;
+    }
+    since_flush += rows;
+    const uint32_t stride = (uint32_t)NA * NT;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++)
+        if ((ok >> k) & 1u)
+            part[g[k] * stride + tid] += 1ull;
+#pragma unroll
+    for (int a = 0; a < kAggUnroll; a++) {
+        if (a < P.nagg) {
+            const char *b = loc_ptr(P.agg_loc[a], stage, scratch);
+            unsigned long long *pa = part + (a + 1) * NT + tid;
+            const int t = P.agg_type[a];
+            if (t == T_I64 || t == T_U64) {
+#pragma unroll
+                for (int k = 0; k < ITEMS; k++)
+                    if ((ok >> k) & 1u)
+                        pa[g[k] * stride] += ((const uint64_t *)b)[k * NT + tid];
+            } else {
+#pragma unroll
+                for (int k = 0; k < ITEMS; k++)
+                    if ((ok >> k) & 1u)
+                        pa[g[k] * stride] += ld_ext(b, t, k * NT + tid);
+            }
+        }
+    }
+}
+
+// End-of-kernel combine of the thread-private partials: one thread per (group,
+// aggregate) slot sums the NT partials exactly in 128 bits (no shared atomics, whose
+// 64-bit form is a CAS loop on sm_100), then adds the slot into cta_acc.
+template <int NT>
+__device__ inline void agg_combine(const ChainProg &P, unsigned long long *part, unsigned long long *cta_acc,
+                                   int nthreads)
+{
+    const int NA = P.nagg + 1;
+    for (int q = threadIdx.x; q < P.D * NA; q += nthreads) {
+        const int a = q % NA;
+        const bool uns = a > 0 && P.agg_unsigned[a - 1];
+        unsigned long long lo = cta_acc[2 * q], hi = cta_acc[2 * q + 1];
+        for (int t = 0; t < NT; t++) {
+            const unsigned long long v = part[q * NT + t];
+            const unsigned long long vh = (!uns && (long long)v < 0) ? ~0ull : 0ull;
+            const unsigned long long nlo = lo + v;
+            hi += vh + (nlo < lo ? 1ull : 0ull);
+            lo = nlo;
+        }
+        cta_acc[2 * q] = lo;
+        cta_acc[2 * q + 1] = hi;
     }
 }
 

@@ -94,6 +94,7 @@ struct TileLaunch {
     const int64_t *n_ptr;      // device row count written by an earlier kernel (else nullptr)
     int32_t stages;
     uint32_t out_bytes;        // scan kernel: bytes of the compacted-tile ring
+    int32_t direct;            // scan kernel: no SELECT in the group, rows stored at their offsets
     int32_t use_tma;           // input slots may be bulk-copied (16B-aligned bases)
     uint32_t epoch;            // look-back epoch tag (1..65535)
     uint64_t *status;          // look-back status words, >= ntiles

@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
-    const bool emit = !AGG && !(L.dbg & 2);
+    const bool emit = !AGG && !(L.dbg & 2) && !L.direct;
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) {
@@ -301,6 +301,37 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                 L.dbg_ts[8 * t + 6] = globaltimer();
             if (AGG) {
                 agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
+                if ((L.dbg & 4) && tid == 0)
+                    L.dbg_ts[8 * t + 2] = globaltimer();
+                bar_sync(kComputeBar, NT);
+                if (tid == 0)
+                    mbar_arrive(&ctl->in[s].empty);
+                continue;
+            }
+            if (L.direct) {
+                // every row survives: coalesced stores at the rows' own offsets
+                const int64_t lim64 = min((int64_t)rows, P.out_capacity - row0);
+                const int lim = (int)(lim64 > 0 ? lim64 : 0);
+                for (int c = 0; c < P.nout; c++) {
+                    const char *src = loc_ptr(P.out_loc[c], st, scratch);
+                    switch (P.out_w[c]) {
+                    case 1:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if (k * NT + tid < lim) ((uint8_t *)P.out_ptr[c])[row0 + k * NT + tid] = ((const uint8_t *)src)[k * NT + tid];
+                        break;
+                    case 4:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if (k * NT + tid < lim) ((uint32_t *)P.out_ptr[c])[row0 + k * NT + tid] = ((const uint32_t *)src)[k * NT + tid];
+                        break;
+                    default:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if (k * NT + tid < lim) ((uint64_t *)P.out_ptr[c])[row0 + k * NT + tid] = ((const uint64_t *)src)[k * NT + tid];
+                        break;
+                    }
+                }
                 bar_sync(kComputeBar, NT);
                 if (tid == 0)
                     mbar_arrive(&ctl->in[s].empty);
@@ -431,18 +462,18 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                 mbar_arrive(&ctl->blk[j].aggr);
             }
         }
-        if (AGG)
-            agg_flush<NT>(P, part, cta_acc);
     }
     __syncthreads();
     if (AGG) {
+        agg_combine<NT>(P, part, cta_acc, blockDim.x);
+        __syncthreads();
         for (int qq = tid; qq < P.D * NA; qq += blockDim.x) {
             const unsigned long long lo = cta_acc[2 * qq], hi = cta_acc[2 * qq + 1];
             if (lo | hi)
                 atomic_add128(&L.agg_acc[2 * qq], &L.agg_acc[2 * qq + 1], lo, hi);
         }
-    } else if (ntiles == 0 && blockIdx.x == 0 && tid == 0) {
-        *L.n_dev = 0;
+    } else if ((ntiles == 0 || L.direct) && blockIdx.x == 0 && tid == 0) {
+        *L.n_dev = L.direct ? n : 0;
     }
     cta_exit_reset(L.ctrs);
 }
@@ -914,8 +945,10 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         if (nt == 512) return occ(k_scan_chain<512, 4, false>, smem, 512 + kAuxThreads);
         return items == 4 ? occ(k_scan_chain<256, 4, false>, smem, 256 + kAuxThreads)
                           : occ(k_scan_chain<256, 8, false>, smem, 256 + kAuxThreads);
-    case 1: return items == 4 ? occ(k_scan_chain<256, 4, true>, smem, 256 + kAuxThreads)
-                              : occ(k_scan_chain<256, 8, true>, smem, 256 + kAuxThreads);
+    case 1:
+        if (nt == 128) return occ(k_scan_chain<128, 16, true>, smem, 128 + kAuxThreads);
+        return items == 4 ? occ(k_scan_chain<256, 4, true>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, true>, smem, 256 + kAuxThreads);
     case 2: return occ(k_join_expand, smem);
     default: return occ(k_join_runs<uint64_t>, smem);
     }
@@ -932,8 +965,11 @@ static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int 
 cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem,
                               int grid, cudaStream_t s)
 {
-    if (agg)
+    if (agg) {
+        if (nt == 128)
+            return sc<128, 16, true>(P, L, smem, grid, s);
         return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
+    }
     if (nt == 512)
         return sc<512, 4, false>(P, L, smem, grid, s);
     return items == 4 ? sc<256, 4, false>(P, L, smem, grid, s) : sc<256, 8, false>(P, L, smem, grid, s);

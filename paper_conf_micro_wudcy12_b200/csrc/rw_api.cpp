@@ -93,6 +93,7 @@ struct Lowered {
     int items = 8, stages = 2, ctas = 1;
     int tile = 2048;              // rows per tile
     int nt = 256;                 // compute threads per CTA
+    bool direct = false;          // no SELECT: outputs written at their row offsets
     int ring = 0;                 // scan kernel: output ring entries
     uint32_t out_bytes = 0;       // bytes of one output ring entry
     std::vector<uint32_t> out_off;
@@ -736,8 +737,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             P.agg_type[q] = P.slot[P.agg_slot[q]].type;
         }
     };
-    const size_t agg_bytes =
-        L.agg ? (size_t)P.D * (P.nagg + 1) * kThreads * 8 + al128((size_t)P.D * (P.nagg + 1) * 16) : 0;
+    auto agg_bytes_for = [&](int nt) -> size_t {
+        return L.agg ? (size_t)P.D * (P.nagg + 1) * nt * 8 + al128((size_t)P.D * (P.nagg + 1) * 16) : 0;
+    };
     if (L.agg && (size_t)P.D * (P.nagg + 1) > (size_t)kMaxAggSlots)
         raise(RW_E_UNSUPPORTED, "aggregate needs more than 4096 accumulators");
 
@@ -759,11 +761,18 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     const int want_stages = p->o.stages > 0 ? std::min(p->o.stages, kMaxStages) : 0;
     const size_t want_ring = p->o.reserved[0] > 0 ? (size_t)p->o.reserved[0] * 1024 : 0;
     bool ok = false;
+    double best_score = -1;
+    bool direct = !L.agg;
+    for (const HOp &h : ops)
+        if (h.kind == K_PRED)
+            direct = false;
+    L.direct = direct;
     // kernel variants (compute threads NT x rows per thread): 256 x 8 (2048-row tiles),
     // 256 x 4 (1024-row tiles, wide rows); 512 x 4 on request (opts.reserved[4] == 2)
     struct Var { int nt, items; };
     std::vector<Var> vars;
     if (!L.agg && p->o.reserved[4] == 2) vars.push_back({512, 4});
+    if (L.agg && p->o.reserved[4] != 1) vars.push_back({128, 16});   // halves the thread-private partials
     vars.push_back({256, 8});
     vars.push_back({256, 4});
     for (size_t ii = 0; ii < vars.size(); ii++) {
@@ -774,41 +783,61 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         size_t W = 0;                       // largest compacted tile (every row survives)
         for (int c = 0; c < P.nout; c++)
             W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+        const size_t agg_bytes = agg_bytes_for(nt);
         const size_t base = scan_ctl_bytes() + P.scratch_bytes + agg_bytes;
-        const int occ_pref[2] = {2, 1};
-        for (int oi = 0; oi < 2 && !ok; oi++) {
-            int occ_t = occ_pref[oi];
-            if (p->o.ctas_per_sm > 0) {
-                if (oi > 0) break;
-                occ_t = p->o.ctas_per_sm;
-            }
+        // Candidate (CTAs/SM, input stages, ring bytes) for this variant:
+        //  - aggregate: maximise input bytes in flight per SM (no ring);
+        //  - no SELECT in the group (every row survives): outputs go straight to their
+        //    row offsets, no ring;
+        //  - otherwise 2 CTAs/SM x 2 stages when the ring still holds >= 1.9 worst-case
+        //    compacted tiles (latency hiding of the compute warps measured best), else
+        //    1 CTA/SM with the deepest stage count whose ring holds >= 2.5 tiles.
+        struct Cand { int occ, S; size_t Rb, smem; double score; };
+        std::vector<Cand> cands;
+        for (int occ_t : {2, 1}) {
+            if (p->o.ctas_per_sm > 0 && occ_t != p->o.ctas_per_sm) continue;
             const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
-            for (int S : {3, 2, 1, 4, 5, 6}) {
+            for (int S = 1; S <= 6; S++) {
                 if (want_stages && S != want_stages) continue;
-                if (!want_stages && occ_t >= 2 && S > 2) continue;
                 if (base + (size_t)S * P.stage_bytes > per_cta) continue;
                 size_t Rb = 0;
-                if (!L.agg) {
+                if (!L.agg && !direct) {
                     Rb = want_ring ? want_ring : (per_cta - base - (size_t)S * P.stage_bytes) / 128 * 128;
                     if (Rb < W) continue;
                 }
                 const size_t smem = base + (size_t)S * P.stage_bytes + Rb;
                 if (smem > per_cta) continue;
-                int occ = chain_occupancy(L.agg ? 1 : 0, nt, items, smem);
-                if (occ < occ_t) continue;
+                if (chain_occupancy(L.agg ? 1 : 0, nt, items, smem) < occ_t) continue;
+                double inflight = std::min<double>((double)occ_t * S * P.stage_bytes, 192.0 * 1024);
+                double score;
+                if (L.agg || direct) {
+                    score = inflight + (occ_t == 2 ? 1024.0 : 0) + S;
+                } else {
+                    const double q = (double)Rb / (double)W;
+                    const bool ok2 = occ_t == 2 && q >= 1.9 && S == 2;
+                    const bool ok1 = occ_t == 1 && q >= 2.5;
+                    score = (ok2 ? 1e9 : 0) + (ok1 ? 1e8 : 0) + inflight + q * 1024.0;
+                }
+                cands.push_back({occ_t, S, Rb, smem, score});
+            }
+        }
+        // best candidate over all variants (a 2048-row tile with one stage loses to a
+        // 1024-row tile with three when the row is wide, e.g. Q1's 38 B + partials)
+        for (const Cand &c : cands) {
+            const double sc = c.score + (T == 2048 ? 512.0 : 0.0);
+            if (!ok || sc > best_score) {
+                best_score = sc;
                 L.items = items;
                 L.nt = nt;
                 L.tile = T;
-                L.stages = S;
+                L.stages = c.S;
                 L.ring = 0;
-                L.out_bytes = (uint32_t)Rb;
-                L.smem = smem;
-                L.ctas = occ_t;
+                L.out_bytes = (uint32_t)c.Rb;
+                L.smem = c.smem;
+                L.ctas = c.occ;
                 ok = true;
-                break;
             }
         }
-        if (ok) break;
     }
     if (!ok)
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
@@ -949,6 +978,7 @@ void run_group(ExecCtx &X, int gi)
         TL.dbg = p->o.reserved[1];
         TL.dbg_ts = (uint64_t *)(((uint64_t)(uint32_t)p->o.reserved[3] << 32) | (uint32_t)p->o.reserved[2]);
         TL.out_bytes = L.out_bytes;
+        TL.direct = L.direct ? 1 : 0;
         TL.use_tma = aligned ? 1 : 0;
         TL.epoch = next_epoch(p);
         TL.status = p->status;
@@ -1180,6 +1210,9 @@ std::string explain(rw_plan *p, int out_node)
               << ", smem " << L.smem
               << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
               << L.P.nops;
+            if (L.agg)
+                s << ", groups " << L.P.D << ", sums " << L.P.nagg << ", partial flush every " << L.P.flush_rows
+                  << " rows";
         } catch (const RwError &e) {
             s << " | not lowerable: " << e.msg;
         }

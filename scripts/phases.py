@@ -5,28 +5,42 @@ import torch
 import workloads
 from tests.planspec import build_gpu_plan
 
-def main(stages, ctas, ring, extra=0, rows=1 << 29):
-    spec = workloads.c2_spec()
-    ins = workloads.c2_inputs(rows, 0, "cuda:0")
-    T = 2048
+def main(stages, ctas, ring, extra=0, cfg="c2"):
+    if cfg == "c4":
+        rows = 600_000_000
+        spec = workloads.c4_spec()
+        ins = workloads.c4_inputs(rows, 0, "cuda:0")
+    else:
+        rows = 1 << 29
+        spec = workloads.c2_spec()
+        ins = workloads.c2_inputs(rows, 0, "cuda:0")
+    T = 1024 if cfg == "c4" else 2048
     nt = (rows + T - 1) // T
     ts = torch.zeros(nt * 8, dtype=torch.int64, device="cuda:0")
     plan, ids = build_gpu_plan(spec, stages=stages, ctas_per_sm=ctas, defer=ring, dbg=4 | extra, dbg_ts=ts.data_ptr())
-    outs = [torch.empty(rows, dtype=torch.int32, device="cuda:0") for _ in range(3)]
+    out_node = ids[spec["out"]]
+    types = plan.node_schema(out_node)
+    dt = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
+    cap = 6 if cfg == "c4" else rows
+    outs = [torch.empty(cap, dtype=dt[t], device="cuda:0") for t in types]
     nd = torch.zeros(1, dtype=torch.int64, device="cuda:0")
+    name = list(spec["inputs"])[0]
+    print(plan.explain(out_node))
     for _ in range(3):
-        plan.execute([(rows, ins["R"])], ids["s2"], outs, rows, n_dev=nd)
+        plan.execute([(rows, ins[name])], out_node, outs, cap, n_dev=nd)
     torch.cuda.synchronize()
     a = ts.view(nt, 8).double()
     t0 = a[:, 0].min()
     d = {"load(claim->data)": a[:, 1] - a[:, 0], "ops(data->ops)": a[:, 6] - a[:, 1], "ballot(ops->bar1)": a[:, 7] - a[:, 6], "scan(bar1->agg)": a[:, 2] - a[:, 7],
          "writer queue(agg->wstart)": a[:, 5] - a[:, 2], "lookback(wstart->offset)": a[:, 3] - a[:, 5], "store(offset->stored)": a[:, 4] - a[:, 3],
          "total(claim->stored)": a[:, 4] - a[:, 0]}
-    res = {"cfg": [stages, ctas, ring, extra], "kernel_us": float((a[:, 4].max() - t0) / 1e3)}
+    if cfg == "c4":
+        a[:, 3] = a[:, 2]; a[:, 4] = a[:, 2]; a[:, 5] = a[:, 2]; a[:, 7] = a[:, 6]
+    res = {"cfg": [stages, ctas, ring, extra, cfg], "kernel_us": float((a[:, 4].max() - t0) / 1e3)}
     for k, v in d.items():
         q = torch.quantile(v[: min(nt, 1 << 24)] / 1e3, torch.tensor([0.1, 0.5, 0.9, 0.99], dtype=torch.float64, device=v.device))
         res[k] = [round(float(x), 2) for x in q]
     print(json.dumps(res))
 
 if __name__ == "__main__":
-    main(*[int(x) for x in sys.argv[1:5]])
+    main(*[int(x) for x in sys.argv[1:5]], *sys.argv[5:6])

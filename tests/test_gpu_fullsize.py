@@ -1,0 +1,110 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(default plan options).  The oracle is run on chunks it finishes in seconds; offsets
+of a chunk inside the GPU output come from torch reductions (an implementation
+independent of librw), never from the CUDA path:
+
+* C2 (2^29 x 4 i32): first, last and two interior 2^22-row chunks compared element by
+  element (order included); total count vs a torch count of the predicate.
+* C4 (6e8 lineitem rows): the full aggregate equals the sum of per-chunk oracle
+  aggregates (exact additivity of integer sums), all 600M rows covered.
+* C3 (2 x 2^26 Zipf-0.5): |J| = sum_k mL(k) mR(k) via torch.unique; three key ranges
+  (including the hottest key) compared with the oracle join of the sub-relations.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from tests.planspec import NPT, assert_same, build_gpu_plan, run_oracle
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+DEV = "cuda:0"
+CH = 1 << 22
+
+
+def _host(cols, types, a, b):
+    return oracle.Relation(types, [c[a:b].cpu().numpy().view(NPT[t]) for c, t in zip(cols, types)])
+
+
+def test_c2_full_size_chunks():
+    import torch
+    n = workloads.C2_ROWS
+    spec = workloads.c2_spec()
+    ins = workloads.c2_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    outs = [torch.empty(n, dtype=torch.int32, device=DEV) for _ in range(3)]
+    m = plan.execute([(n, ins["R"])], ids["s2"], outs, n)
+    R = ins["R"]
+    keep = (R[1] < workloads.thr_i32(0.5)) & (R[3] < workloads.thr_i32(0.5))
+    assert m == int(keep.sum().item())
+    types = ["i32"] * 4
+    for a in [0, 123 * CH, 77 * CH + 5, n - CH]:
+        b = min(a + CH, n)
+        ref = run_oracle(spec, {"R": [c[a:b] for c in R]})
+        off = int(keep[:a].sum().item())
+        got = oracle.Relation(ref.types, [o[off:off + ref.n].cpu().numpy().view(np.int32) for o in outs])
+        assert_same(got, ref)
+
+
+def test_c4_full_size_additive():
+    import torch
+    n = workloads.C4_ROWS
+    spec = workloads.c4_spec()
+    ins = workloads.c4_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    got_cols, k = plan.run([(n, ins["lineitem"])], ids["g"], 6)
+    types = plan.node_schema(ids["g"])
+    got = {}
+    for i in range(k):
+        g = (int(got_cols[0][i]), int(got_cols[1][i]))
+        got[g] = [int(got_cols[2][i])] + [
+            (int(got_cols[4 + 2 * q][i].item()) << 64) + (int(got_cols[3 + 2 * q][i].item()) & ((1 << 64) - 1))
+            for q in range(5)]
+    ref = {}
+    big = 1 << 25
+    for a in range(0, n, big):
+        b = min(a + big, n)
+        part = run_oracle(spec, {"lineitem": [c[a:b] for c in ins["lineitem"]]})
+        for i in range(part.n):
+            g = (int(part.cols[0][i]), int(part.cols[1][i]))
+            row = [int(part.cols[2][i])] + [
+                int(part.cols[4 + 2 * q][i]) * (1 << 64) + int(part.cols[3 + 2 * q][i]) for q in range(5)]
+            acc = ref.setdefault(g, [0] * 6)
+            ref[g] = [x + y for x, y in zip(acc, row)]
+    assert sorted(got) == sorted(ref)
+    for g in ref:
+        assert got[g] == ref[g], g
+    assert sum(v[0] for v in ref.values()) > 0.98 * n      # ~98.6% of rows pass the date filter
+
+
+def test_c3_full_size_cardinality_and_key_ranges():
+    import torch
+    n = workloads.C3_ROWS
+    spec = workloads.c3_spec()
+    ins = workloads.c3_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    cap = 400_000_000
+    outs = [torch.empty(cap, dtype=torch.int32, device=DEV) for _ in range(2)]
+    m = plan.execute([(n, ins["L"]), (n, ins["R"])], ids["p"], outs, cap)
+    lk = ins["L"][0].to(torch.int64) & 0xFFFFFFFF
+    rk = ins["R"][0].to(torch.int64) & 0xFFFFFFFF
+    ku, cl = torch.unique_consecutive(lk, return_counts=True)
+    kv, cr = torch.unique_consecutive(rk, return_counts=True)
+    # |L join R| before the SELECT (property): join the plan without the select
+    common_l = torch.isin(ku, kv)
+    common_r = torch.isin(kv, ku)
+    total = int((cl[common_l] * cr[common_r]).sum().item())
+    assert total > 0 and m <= total
+    okey = outs[0][:m].to(torch.int64) & 0xFFFFFFFF
+    assert bool((okey[1:] >= okey[:-1]).all())
+    hot = int(ku[torch.argmax(cl * common_l)].item())
+    for lo, hi in [(0, 1 << 24), (hot, hot + 1), (3 << 30, (3 << 30) + (1 << 25))]:
+        lsel = (lk >= lo) & (lk < hi)
+        rsel = (rk >= lo) & (rk < hi)
+        sub = {"L": [c[lsel] for c in ins["L"]], "R": [c[rsel] for c in ins["R"]]}
+        ref = run_oracle(spec, sub)
+        a = int(torch.searchsorted(okey, torch.tensor([lo], device=DEV)).item())
+        got = oracle.Relation(ref.types, [o[a:a + ref.n].cpu().numpy().view(np.uint32) for o in outs])
+        assert_same(got, ref)
+        b = int(torch.searchsorted(okey, torch.tensor([hi], device=DEV)).item())
+        assert b - a == ref.n
