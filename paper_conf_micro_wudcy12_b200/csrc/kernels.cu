@@ -8,8 +8,9 @@
 //   k_join_runs<K>            merge-path partitioned sorted-key JOIN, phase 1:
 //                             matched key runs + output offsets (a7).
 //   k_tile_runs               first run of every expansion tile.
-//   k_join_expand             JOIN phase 2: output-balanced expansion fused with
-//                             the downstream SELECT / PROJECT chain (a8).
+//   k_scan_chain<..., JOIN>   JOIN phase 2: output-balanced expansion (join_fill)
+//                             fused with the downstream SELECT / PROJECT chain (a8),
+//                             same warp-specialised pipeline as the scan chain.
 //
 // Every persistent kernel claims tiles with a global atomic counter (so the
 // decoupled look-back always has forward progress) and the last CTA to leave
@@ -102,9 +103,94 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
         d[j] = src[j];
 }
 
-template <int NT, int ITEMS, bool AGG>
+// Join expansion into a tile (§8(a) a8): candidates [t*T, t*T + rows) of the
+// join output are mapped to (left row, right row) through the tile's run records
+// (cached in smem) and the live join columns are gathered into the tile's slots.
+// Thread `tid` expands candidates [tid*ITEMS, tid*ITEMS + ITEMS): one binary search,
+// then a forward walk; ITEMS odd makes the thread-contiguous smem writes conflict-free.
+template <int NT, int ITEMS>
+__device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_t t, int64_t ntiles, int rows,
+                                 char *st, char *rcache)
+{
+    constexpr int T = NT * ITEMS;
+    const int tid = threadIdx.x;
+    uint64_t *c_off = (uint64_t *)rcache;
+    uint32_t *c_s = (uint32_t *)(c_off + (T + 1));
+    uint32_t *c_lo = c_s + (T + 1);
+    uint32_t *c_lenR = c_lo + (T + 1);
+    const int64_t o0 = t * T;
+    const int64_t r0 = X.tile_run[t];
+    const int64_t r1 = (t + 1 < ntiles) ? X.tile_run[t + 1] : X.nruns - 1;
+    const int nr = (int)(r1 - r0 + 1);
+    for (int q = tid; q < nr; q += NT) {
+        c_off[q] = X.off[r0 + q];
+        c_s[q] = X.s[r0 + q];
+        c_lo[q] = X.lo[r0 + q];
+        c_lenR[q] = X.lenR[r0 + q];
+    }
+    bar_sync(kComputeBar, NT);
+    const int first = tid * ITEMS;
+    if (first < rows) {
+        uint32_t ii[ITEMS], jj[ITEMS];
+        const uint64_t o = (uint64_t)(o0 + first);
+        int lo = 0, hi = nr;
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (c_off[mid] <= o) lo = mid + 1;
+            else hi = mid;
+        }
+        int r = lo - 1;
+        // (i, j) of the first candidate by division, the rest by a carry walk
+        uint64_t d = o - c_off[r];
+        uint32_t lr = c_lenR[r];
+        uint32_t qi = (uint32_t)(d / lr), qj = (uint32_t)(d - (uint64_t)qi * lr);
+#pragma unroll
+        for (int k = 0; k < ITEMS; k++) {
+            ii[k] = jj[k] = 0;
+            if (first + k < rows) {
+                const uint64_t oo = o + k;
+                if (r + 1 < nr && c_off[r + 1] <= oo) {
+                    while (r + 1 < nr && c_off[r + 1] <= oo)
+                        r++;
+                    lr = c_lenR[r];
+                    d = oo - c_off[r];
+                    qi = (uint32_t)(d / lr);
+                    qj = (uint32_t)(d - (uint64_t)qi * lr);
+                }
+                ii[k] = c_s[r] + qi;
+                jj[k] = c_lo[r] + qj;
+                if (++qj == lr) {
+                    qj = 0;
+                    ++qi;
+                }
+            }
+        }
+        for (int c = 0; c < X.ncols; c++) {
+            char *dst = st + P.slot[X.dst_slot[c]].off;
+            const int w = type_width(P.slot[X.dst_slot[c]].type);
+            const char *src = (const char *)X.src[c];
+            const bool right = X.from_right[c];
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                if (first + k < rows) {
+                    const size_t row = right ? jj[k] : ii[k];
+                    if (w == 4)
+                        ((uint32_t *)dst)[first + k] = ((const uint32_t *)src)[row];
+                    else if (w == 8)
+                        ((uint64_t *)dst)[first + k] = ((const uint64_t *)src)[row];
+                    else
+                        ((uint8_t *)dst)[first + k] = ((const uint8_t *)src)[row];
+                }
+            }
+        }
+    }
+    bar_sync(kComputeBar, NT);
+}
+
+template <int NT, int ITEMS, bool AGG, bool JOIN>
 __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid_constant__ ChainProg P,
-                                                                                  const __grid_constant__ TileLaunch L)
+                                                                     const __grid_constant__ TileLaunch L,
+                                                                     const __grid_constant__ JoinExpand X)
 {
     constexpr int T = NT * ITEMS;
     constexpr int NW = NT / 32;             // compute warps
@@ -118,6 +204,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     unsigned long long *part = (unsigned long long *)(ring + (AGG ? 0 : R));
     const int NA = P.nagg + 1;
     unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * NT : 0);
+    char *rcache = ring + (JOIN ? R : 0);   // join: run-record cache for the current tile
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
@@ -161,7 +248,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
                     L.dbg_ts[8 * t + 0] = globaltimer();
-                if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
+                if (!JOIN && t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
                     char *st = stages + (size_t)s * P.stage_bytes;
                     fence_proxy_async_smem();
                     mbar_arrive_expect_tx(&ctl->in[s].full, tx_bytes);
@@ -269,7 +356,9 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                     mbar_arrive(&ctl->in[s].empty);
                 continue;
             }
-            if (!(L.use_tma && rows == T)) {
+            if (JOIN) {
+                join_fill<NT, ITEMS>(P, X, t, ntiles, rows, st, rcache);
+            } else if (!(L.use_tma && rows == T)) {
                 // ragged last tile or unaligned column bases: plain coalesced loads
                 for (int c = 0; c < P.nin; c++) {
                     const int w = type_width(P.slot[c].type);
@@ -559,6 +648,7 @@ __global__ void __launch_bounds__(kThreads) k_agg_finalize(const __grid_constant
 // ===========================================================================
 constexpr int kRunItems = 8;
 constexpr int kRunT = kThreads * kRunItems;
+constexpr int kRunExt = 512;     // extra L / R elements staged past the partition end
 
 template <typename K>
 __device__ __forceinline__ int64_t merge_path(const K *L, int64_t nl, const K *R, int64_t nr, int64_t d)
@@ -674,14 +764,25 @@ __device__ inline void block_scan_u64(uint64_t (&v)[ITEMS], uint64_t *wtot /* IT
         v[k] += wtot[k * kWarps + warp];
 }
 
+// merge-path split of every partition boundary d = p * kRunT (p = 0..nparts)
 template <typename K>
-__global__ void __launch_bounds__(kThreads) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
+__global__ void k_merge_splits(const __grid_constant__ JoinRunsLaunch J)
+{
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p > J.nparts)
+        return;
+    const int64_t d = min(p * kRunT, J.nl + J.nr);
+    J.split[p] = merge_path((const K *)J.lkey, J.nl, (const K *)J.rkey, J.nr, d);
+}
+
+template <typename K>
+__global__ void __launch_bounds__(kThreads, 3) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
 {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     uint64_t *wtot = (uint64_t *)smem_raw;                        // kRunItems*kWarps + 1
-    K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT
-    K *sR = sL + kRunT;                                           // kRunT
-    __shared__ int64_t sh_part, sh_i0, sh_i1, sh_base_runs, sh_base_outs;
+    K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT + kRunExt
+    K *sR = sL + kRunT + kRunExt;                                 // kRunT + kRunExt
+    __shared__ int64_t sh_part, sh_base_runs, sh_base_outs;
     const K *L = (const K *)J.lkey;
     const K *R = (const K *)J.rkey;
     const int tid = threadIdx.x;
@@ -695,16 +796,15 @@ __global__ void __launch_bounds__(kThreads) k_join_runs(const __grid_constant__ 
         if (p >= J.nparts)
             break;
         const int64_t d0 = p * kRunT, d1 = min(d0 + kRunT, ntot);
-        if (tid == 0)
-            sh_i0 = merge_path(L, J.nl, R, J.nr, d0);
-        if (tid == 32)
-            sh_i1 = merge_path(L, J.nl, R, J.nr, d1);
-        __syncthreads();
-        const int64_t i0 = sh_i0, i1 = sh_i1, j0 = d0 - i0, j1 = d1 - i1;
-        const int nL = (int)(i1 - i0), nR = (int)(j1 - j0);
-        for (int q = tid; q < nL; q += kThreads)
+        // partition splits were found by k_merge_splits (one thread per diagonal)
+        const int64_t i0 = J.split[p], i1 = J.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
+        const int nL = (int)(i1 - i0);
+        // stage the partition plus kRunExt elements beyond it: runs cut by the partition
+        // boundary are then resolved in smem; only longer runs gallop through HBM
+        const int nLe = (int)(min(i1 + kRunExt, J.nl) - i0), nRe = (int)(min(j1 + kRunExt, J.nr) - j0);
+        for (int q = tid; q < nLe; q += kThreads)
             sL[q] = L[i0 + q];
-        for (int q = tid; q < nR; q += kThreads)
+        for (int q = tid; q < nRe; q += kThreads)
             sR[q] = R[j0 + q];
         __syncthreads();
 
@@ -722,16 +822,16 @@ __global__ void __launch_bounds__(kThreads) k_join_runs(const __grid_constant__ 
                 const int64_t gi = i0 + li;
                 const bool start = gi == 0 || (li > 0 ? sL[li - 1] != key : L[gi - 1] != key);
                 if (start) {
-                    const int lo_l = lower_bound_smem(sR, nR, key);
-                    const int hi_l = upper_bound_smem(sR, nR, key);
+                    const int lo_l = lower_bound_smem(sR, nRe, key);
+                    const int hi_l = upper_bound_smem(sR, nRe, key);
                     int64_t hi = j0 + hi_l;
-                    if (hi_l == nR)
+                    if (hi_l == nRe)
                         hi = gallop_upper(R, hi, J.nr, key);
                     const int64_t lo = j0 + lo_l;
                     if (hi > lo) {
-                        const int e_l = li + upper_bound_smem(sL + li, nL - li, key);
+                        const int e_l = li + upper_bound_smem(sL + li, nLe - li, key);
                         int64_t iend = i0 + e_l;
-                        if (e_l == nL)
+                        if (e_l == nLe)
                             iend = gallop_upper(L, iend, J.nl, key);
                         emitted |= 1u << k;
                         idx[k] = 1;
@@ -746,16 +846,20 @@ __global__ void __launch_bounds__(kThreads) k_join_runs(const __grid_constant__ 
         uint64_t tot_runs, tot_outs;
         block_scan_u64<kRunItems>(idx, wtot, tot_runs);
         block_scan_u64<kRunItems>(cnt, wtot, tot_outs);
+        // the two look-backs (run count, output count) proceed in two warps at once
         if (tid < 32) {
             const uint64_t br = lookback_warp(J.status_runs, p, tot_runs, J.epoch_runs);
-            const uint64_t bo = lookback_warp(J.status_outs, p, tot_outs, J.epoch_outs);
             if (tid == 0) {
                 sh_base_runs = (int64_t)br;
-                sh_base_outs = (int64_t)bo;
-                if (p == J.nparts - 1) {
+                if (p == J.nparts - 1)
                     J.totals[0] = (int64_t)(br + tot_runs);
+            }
+        } else if (tid < 64) {
+            const uint64_t bo = lookback_warp(J.status_outs, p, tot_outs, J.epoch_outs);
+            if (tid == 32) {
+                sh_base_outs = (int64_t)bo;
+                if (p == J.nparts - 1)
                     J.totals[1] = (int64_t)(bo + tot_outs);
-                }
             }
         }
         __syncthreads();
@@ -799,133 +903,16 @@ __global__ void k_tile_runs(const uint64_t *off, int64_t nruns, int64_t ntiles, 
 }
 
 // ===========================================================================
-// JOIN phase 2 — output-balanced expansion.  Tile = 2304 consecutive join
-// candidates (so a hot key's lenL x lenR block is spread over many CTAs).  The
-// tile's run records are cached in smem; thread t expands candidates
-// [t*9, t*9+9) of the tile (one binary search, then a forward walk), gathers
-// the live join columns into smem slots, and the fused downstream chain runs on
-// the tile exactly as in the scan kernel (§4.3.2: JOIN inside the CTA,
-// then the consumer operators, then one compacted dump).
-// ===========================================================================
-struct JoinCtl {
-    int64_t tile;
-    EmitSmem<kJoinItems> es;
-};
-
-__global__ void __launch_bounds__(kThreads) k_join_expand(const __grid_constant__ ChainProg P,
-                                                          const __grid_constant__ TileLaunch L,
-                                                          const __grid_constant__ JoinExpand X)
-{
-    constexpr int T = kThreads * kJoinItems;
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    JoinCtl *ctl = (JoinCtl *)smem_raw;
-    uint64_t *c_off = (uint64_t *)(smem_raw + align_up(sizeof(JoinCtl), 128));   // T + 1
-    uint32_t *c_s = (uint32_t *)(c_off + (T + 1));
-    uint32_t *c_lo = c_s + (T + 1);
-    uint32_t *c_lenR = c_lo + (T + 1);
-    char *tilebuf = (char *)smem_raw + align_up(sizeof(JoinCtl), 128) + align_up((size_t)(T + 1) * 20, 128);
-    char *scratch = tilebuf + P.stage_bytes;
-    const int tid = threadIdx.x;
-    const int64_t ntiles = (L.n + T - 1) / T;
-
-    while (true) {
-        if (tid == 0)
-            ctl->tile = (int64_t)atomicAdd(&L.ctrs[0], 1u);
-        __syncthreads();
-        const int64_t t = ctl->tile;
-        if (t >= ntiles)
-            break;
-        const int64_t o0 = t * T;
-        const int rows = (int)min((int64_t)T, L.n - o0);
-        const int64_t r0 = X.tile_run[t];
-        const int64_t r1 = (t + 1 < ntiles) ? X.tile_run[t + 1] : X.nruns - 1;
-        const int nr = (int)(r1 - r0 + 1);
-        for (int q = tid; q < nr; q += kThreads) {
-            c_off[q] = X.off[r0 + q];
-            c_s[q] = X.s[r0 + q];
-            c_lo[q] = X.lo[r0 + q];
-            c_lenR[q] = X.lenR[r0 + q];
-        }
-        __syncthreads();
-
-        uint32_t ii[kJoinItems], jj[kJoinItems];
-        const int first = tid * kJoinItems;
-        if (first < rows) {
-            const uint64_t o = (uint64_t)(o0 + first);
-            int lo = 0, hi = nr;
-            while (lo < hi) {
-                int mid = (lo + hi) >> 1;
-                if (c_off[mid] <= o) lo = mid + 1;
-                else hi = mid;
-            }
-            int r = lo - 1;
-#pragma unroll
-            for (int k = 0; k < kJoinItems; k++) {
-                const uint64_t oo = o + k;
-                ii[k] = jj[k] = 0;
-                if (first + k < rows) {
-                    while (r + 1 < nr && c_off[r + 1] <= oo)
-                        r++;
-                    const uint64_t d = oo - c_off[r];
-                    const uint32_t lr = c_lenR[r];
-                    uint64_t qi, qj;
-                    if (d < 0xffffffffull) {
-                        qi = (uint32_t)d / lr;
-                        qj = (uint32_t)d - (uint32_t)qi * lr;
-                    } else {
-                        qi = d / lr;
-                        qj = d - qi * lr;
-                    }
-                    ii[k] = c_s[r] + (uint32_t)qi;
-                    jj[k] = c_lo[r] + (uint32_t)qj;
-                }
-            }
-            for (int c = 0; c < X.ncols; c++) {
-                char *dst = tilebuf + P.slot[X.dst_slot[c]].off;
-                const int w = type_width(P.slot[X.dst_slot[c]].type);
-                const char *src = (const char *)X.src[c];
-                const bool right = X.from_right[c];
-#pragma unroll
-                for (int k = 0; k < kJoinItems; k++) {
-                    if (first + k < rows) {
-                        const size_t row = right ? jj[k] : ii[k];
-                        if (w == 4)
-                            ((uint32_t *)dst)[first + k] = ((const uint32_t *)src)[row];
-                        else if (w == 8)
-                            ((uint64_t *)dst)[first + k] = ((const uint64_t *)src)[row];
-                        else
-                            ((uint8_t *)dst)[first + k] = ((const uint8_t *)src)[row];
-                    }
-                }
-            }
-        }
-        __syncthreads();
-        uint32_t mask = 0;
-#pragma unroll
-        for (int k = 0; k < kJoinItems; k++)
-            if (k * kThreads + tid < rows)
-                mask |= 1u << k;
-        mask = run_ops<kThreads, kJoinItems>(P, tilebuf, scratch, mask);
-        emit_tile<kJoinItems>(P, tilebuf, scratch, mask, t, ntiles, L, &ctl->es);
-        __syncthreads();
-    }
-    if (ntiles == 0 && blockIdx.x == 0 && tid == 0)
-        *L.n_dev = 0;
-    cta_exit_reset(L.ctrs);
-}
-
-// ===========================================================================
 // Host launchers
 // ===========================================================================
-size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<256, 8>), 128); }   // >= every (NT, ITEMS) with NT*ITEMS <= 2048
-size_t join_ctl_bytes() { return align_up(sizeof(JoinCtl), 128); }
+size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<256, 9>), 128); }   // >= every (NT, ITEMS) variant
 size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
 int scan_tile() { return kThreads * kScanItems; }
 int join_expand_tile() { return kThreads * kJoinItems; }
 
 size_t join_runs_smem(int key_type)
 {
-    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)kRunT * type_width(key_type);
+    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)(kRunT + kRunExt) * type_width(key_type);
 }
 
 template <typename F>
@@ -942,14 +929,14 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
 {
     switch (which) {
     case 0:
-        if (nt == 512) return occ(k_scan_chain<512, 4, false>, smem, 512 + kAuxThreads);
-        return items == 4 ? occ(k_scan_chain<256, 4, false>, smem, 256 + kAuxThreads)
-                          : occ(k_scan_chain<256, 8, false>, smem, 256 + kAuxThreads);
+        if (nt == 512) return occ(k_scan_chain<512, 4, false, false>, smem, 512 + kAuxThreads);
+        return items == 4 ? occ(k_scan_chain<256, 4, false, false>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
     case 1:
-        if (nt == 128) return occ(k_scan_chain<128, 16, true>, smem, 128 + kAuxThreads);
-        return items == 4 ? occ(k_scan_chain<256, 4, true>, smem, 256 + kAuxThreads)
-                          : occ(k_scan_chain<256, 8, true>, smem, 256 + kAuxThreads);
-    case 2: return occ(k_join_expand, smem);
+        if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + kAuxThreads);
+        return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, true, false>, smem, 256 + kAuxThreads);
+    case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
     default: return occ(k_join_runs<uint64_t>, smem);
     }
 }
@@ -957,8 +944,18 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
 template <int NT, int ITEMS, bool AGG>
 static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
-    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_chain<NT, ITEMS, AGG><<<grid, NT + kAuxThreads, smem, s>>>(P, L);
+    JoinExpand X{};
+    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_scan_chain<NT, ITEMS, AGG, false><<<grid, NT + kAuxThreads, smem, s>>>(P, L, X);
+    return cudaGetLastError();
+}
+
+cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem, int grid,
+                              cudaStream_t s)
+{
+    cudaFuncSetAttribute(k_scan_chain<kThreads, kJoinItems, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+    k_scan_chain<kThreads, kJoinItems, false, true><<<grid, kThreads + kAuxThreads, smem, s>>>(P, L, X);
     return cudaGetLastError();
 }
 
@@ -984,6 +981,7 @@ cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s)
 template <typename K>
 static cudaError_t jr(const JoinRunsLaunch &J, size_t smem, int grid, cudaStream_t s)
 {
+    k_merge_splits<K><<<(unsigned)((J.nparts + 1 + 255) / 256), 256, 0, s>>>(J);
     cudaFuncSetAttribute(k_join_runs<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     k_join_runs<K><<<grid, kThreads, smem, s>>>(J);
     return cudaGetLastError();
@@ -1008,12 +1006,5 @@ cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles,
     return cudaGetLastError();
 }
 
-cudaError_t join_expand_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem,
-                               int grid, cudaStream_t s)
-{
-    cudaFuncSetAttribute(k_join_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_join_expand<<<grid, kThreads, smem, s>>>(P, L, X);
-    return cudaGetLastError();
-}
 
 }  // namespace rw

@@ -34,6 +34,7 @@ struct JoinRunsLaunch {
     uint32_t epoch_runs, epoch_outs;
     uint32_t *ctrs;
     int64_t *totals;                 // [0] runs, [1] join candidates
+    int64_t *split;                  // nparts + 1 merge-path splits (k_merge_splits)
 };
 
 struct JoinExpand {
@@ -48,7 +49,6 @@ struct JoinExpand {
 };
 
 size_t scan_ctl_bytes();
-size_t join_ctl_bytes();
 size_t join_run_cache_bytes();
 int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs
 cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem, int grid,
@@ -58,9 +58,9 @@ cudaError_t join_runs_launch(const JoinRunsLaunch &J, int key_type, size_t smem,
 size_t join_runs_smem(int key_type);
 cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run,
                              cudaStream_t s);
-cudaError_t join_expand_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem,
-                               int grid, cudaStream_t s);
 int join_expand_tile();
+cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem, int grid,
+                              cudaStream_t s);
 int scan_tile();
 
 }  // namespace rw

@@ -744,15 +744,36 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         raise(RW_E_UNSUPPORTED, "aggregate needs more than 4096 accumulators");
 
     if (g.kind == G_JOIN) {
+        // join expansion runs inside the warp-specialised chain kernel: one stage (the
+        // compute warps fill it themselves), the run-record cache, and the output ring
         const int T = join_expand_tile();
         layout(T);
-        L.items = kJoinItems;
-        L.tile = T;
-        L.stages = 1;
-        L.smem = join_ctl_bytes() + join_run_cache_bytes() + P.stage_bytes + P.scratch_bytes;
-        if (L.smem > kSmemLimit)
+        size_t W = 0;
+        for (int c = 0; c < P.nout; c++)
+            W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+        const size_t base = scan_ctl_bytes() + P.scratch_bytes + join_run_cache_bytes() + P.stage_bytes;
+        bool found = false;
+        for (int occ_t : {2, 1}) {
+            if (p->o.ctas_per_sm > 0 && occ_t != p->o.ctas_per_sm) continue;
+            const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
+            if (base + W > per_cta) continue;
+            size_t Rb = (per_cta - base) / 128 * 128;
+            if (p->o.reserved[0] > 0) Rb = std::min(Rb, (size_t)p->o.reserved[0] * 1024);
+            if (Rb < W || (occ_t == 2 && Rb < W * 19 / 10)) continue;
+            const size_t smem = base + Rb;
+            if (chain_occupancy(2, kThreads, kJoinItems, smem) < occ_t) continue;
+            L.items = kJoinItems;
+            L.nt = kThreads;
+            L.tile = T;
+            L.stages = 1;
+            L.out_bytes = (uint32_t)Rb;
+            L.smem = smem;
+            L.ctas = occ_t;
+            found = true;
+            break;
+        }
+        if (!found)
             raise(RW_E_UNSUPPORTED, "join group exceeds the shared-memory budget");
-        L.ctas = std::max(1, chain_occupancy(2, kThreads, kJoinItems, L.smem));
         return;
     }
     // Scan kernel: S input stages (TMA ring), one scratch tile for computed
@@ -1038,11 +1059,12 @@ void run_group(ExecCtx &X, int gi)
         J.epoch_outs = next_epoch(p);
         J.ctrs = p->ctrs;
         J.totals = p->jtot;
+        J.split = (int64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
         const size_t smem1 = join_runs_smem(kt);
         const int occ1 = std::max(1, chain_occupancy(3, kThreads, 8, smem1));
         const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
         cuda_check(join_runs_launch(J, kt, smem1, grid1, p->stream), "k_join_runs");
-        p->launches++;
+        p->launches += 2;
         cuda_check(cudaMemcpyAsync(p->jtot_host, p->jtot, 16, cudaMemcpyDeviceToHost, p->stream), "copy totals");
         cuda_check(cudaStreamSynchronize(p->stream), "sync after join runs");
         const int64_t nruns = p->jtot_host[0], total = p->jtot_host[1];
@@ -1088,8 +1110,10 @@ void run_group(ExecCtx &X, int gi)
         TL.ctrs = p->ctrs;
         TL.n_dev = n_dev;
         TL.err = p->err;
+        TL.out_bytes = L.out_bytes;
+        TL.dbg = p->o.reserved[1];
         const int grid2 = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (int64_t)p->sms * L.ctas));
-        cuda_check(join_expand_launch(L.P, TL, XJ, L.smem, grid2, p->stream), "k_join_expand");
+        cuda_check(join_chain_launch(L.P, TL, XJ, L.smem, grid2, p->stream), "k_scan_chain<join>");
         p->launches++;
     }
     X.rels[gi] = o;
@@ -1194,7 +1218,7 @@ std::string explain(rw_plan *p, int out_node)
     s << "groups:\n";
     for (size_t q = 0; q < G.groups.size(); q++) {
         const Group &g = G.groups[q];
-        s << "  group " << q << ": " << (g.kind == G_SCAN ? "k_scan_chain" : "k_join_runs+k_join_expand");
+        s << "  group " << q << ": " << (g.kind == G_SCAN ? "k_scan_chain" : "k_merge_splits+k_join_runs+k_tile_runs+k_scan_chain<join>");
         if (g.agg >= 0) s << "<agg>+k_agg_finalize";
         s << " nodes [";
         if (g.kind == G_SCAN) s << "src " << g.source;
