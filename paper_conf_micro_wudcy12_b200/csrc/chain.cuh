@@ -275,8 +275,18 @@ __device__ __forceinline__ uint32_t run_ops(const ChainProg &P, const char *stag
         const int64_t k = P.ops[i].k;
         const char *a = loc_ptr(P.ops[i].a, stage, scratch);
         const char *b = loc_ptr(P.ops[i].b, stage, scratch);
-        if (kind == K_PRED)
-            mask = run_pred<NT, ITEMS>(code, k, a, b, mask);
+        if (kind == K_PRED) {
+            // inline fast paths for the commonest atoms (32-bit column vs constant);
+            // everything else goes through the generic dispatch
+            if (code == T_I32 * 8 + C_LT)
+                mask = pred_loop<NT, ITEMS, int32_t, C_LT, false>(a, b, (int32_t)k, mask);
+            else if (code == T_U32 * 8 + C_LT)
+                mask = pred_loop<NT, ITEMS, uint32_t, C_LT, false>(a, b, (uint32_t)k, mask);
+            else if (code == T_I32 * 8 + C_LE)
+                mask = pred_loop<NT, ITEMS, int32_t, C_LE, false>(a, b, (int32_t)k, mask);
+            else
+                mask = run_pred<NT, ITEMS>(code, k, a, b, mask);
+        }
         else
             run_expr<NT, ITEMS>(code, P.ops[i].ta, P.ops[i].tb, k, (char *)loc_ptr(P.ops[i].dst, stage, scratch), a, b);
     }

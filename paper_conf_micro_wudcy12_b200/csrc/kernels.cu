@@ -74,7 +74,7 @@ template <int NT, int ITEMS>
 struct ScanCtl {
     InCtl in[kMaxStages];
     BlkCtl blk[kRingSlots];
-    uint32_t cnt[ITEMS * NT / 32];
+    uint32_t cnt[2][ITEMS * NT / 32];    // double-buffered: a warp may run one tile ahead
     uint32_t total;
     uint32_t roff;
     volatile uint32_t tail;              // ring bytes released by the writers (monotone, wraps)
@@ -213,10 +213,10 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     if (tid == 0) {
         for (int s = 0; s < S; s++) {
             mbar_init(&ctl->in[s].full, 1);
-            mbar_init(&ctl->in[s].empty, 1);
+            mbar_init(&ctl->in[s].empty, NW);          // one arrival per compute warp
         }
         for (int j = 0; j < kRingSlots; j++) {
-            mbar_init(&ctl->blk[j].aggr, 1);
+            mbar_init(&ctl->blk[j].aggr, NW);          // one arrival per compute warp
             mbar_init(&ctl->blk[j].oempty, 1);
         }
         ctl->tail = 0;
@@ -318,18 +318,21 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
         }
     } else {
         // ---------------- compute warps ----------------
+        // Every thread reads and writes only its own rows (k*NT + tid) of the stage and
+        // of the scratch tile, so warps run independently: the only CTA-wide barrier per
+        // tile is the one that makes the survivor counts visible.  The stage is released
+        // and the compacted block handed to the writers by per-warp mbarrier arrivals
+        // (count = NW); the ring reservation is replicated, deterministically, in every warp.
         int64_t since_flush = 0;
         int s = 0;
         uint32_t fph = 0;
+        uint32_t head = 0, hpos = 0;
         for (int64_t i = 0;; ++i) {
             if (i > 0 && ++s == S) {
                 s = 0;
                 fph ^= 1;
             }
-            if (L.dbg & 8)
-                mbar_wait_spin(&ctl->in[s].full, fph);
-            else
-                mbar_wait(&ctl->in[s].full, fph);
+            mbar_wait(&ctl->in[s].full, fph);
             const int64_t t = ctl->in[s].tile;
             const int j = (int)(i % kRingSlots);
             if (t >= ntiles) {
@@ -340,7 +343,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                         if (u >= kRingSlots)
                             mbar_wait(&ctl->blk[ju].oempty, (uint32_t)(((u / kRingSlots) - 1) & 1));
                         ctl->blk[ju].tile = ntiles;
-                        mbar_arrive(&ctl->blk[ju].aggr);
+                        mbar_arrive_cnt(&ctl->blk[ju].aggr, NW);
                     }
                 }
                 break;
@@ -350,16 +353,19 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
             const int rows = (int)min((int64_t)T, n - row0);
             if ((L.dbg & 4) && tid == 0)
                 L.dbg_ts[8 * t + 1] = globaltimer();
-            if (L.dbg & 2) {   // diagnostics: stream the tiles only (TMA pipeline ceiling)
-                bar_sync(kComputeBar, NT);
-                if (tid == 0)
+            auto release_stage = [&]() {
+                __syncwarp();
+                if (lane == 0)
                     mbar_arrive(&ctl->in[s].empty);
+            };
+            if (L.dbg & 2) {   // diagnostics: stream the tiles only (TMA pipeline ceiling)
+                release_stage();
                 continue;
             }
             if (JOIN) {
                 join_fill<NT, ITEMS>(P, X, t, ntiles, rows, st, rcache);
             } else if (!(L.use_tma && rows == T)) {
-                // ragged last tile or unaligned column bases: plain coalesced loads
+                // ragged last tile or unaligned column bases: each thread loads its own rows
                 for (int c = 0; c < P.nin; c++) {
                     const int w = type_width(P.slot[c].type);
                     char *dst = st + P.slot[c].off;
@@ -375,7 +381,6 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                             dst[r] = src[r];
                     }
                 }
-                bar_sync(kComputeBar, NT);
             }
             uint32_t mask = (1u << ITEMS) - 1u;
             if (rows < T) {
@@ -392,9 +397,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                 agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
                 if ((L.dbg & 4) && tid == 0)
                     L.dbg_ts[8 * t + 2] = globaltimer();
-                bar_sync(kComputeBar, NT);
-                if (tid == 0)
-                    mbar_arrive(&ctl->in[s].empty);
+                release_stage();
                 continue;
             }
             if (L.direct) {
@@ -421,23 +424,21 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                         break;
                     }
                 }
-                bar_sync(kComputeBar, NT);
-                if (tid == 0)
-                    mbar_arrive(&ctl->in[s].empty);
+                release_stage();
                 continue;
             }
+            uint32_t *cnt = ctl->cnt[i & 1];
             uint32_t bal[ITEMS];
 #pragma unroll
             for (int k = 0; k < ITEMS; k++) {
                 bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
                 if (lane == 0)
-                    ctl->cnt[k * NW + warp] = __popc(bal[k]);
+                    cnt[k * NW + warp] = __popc(bal[k]);
             }
             bar_sync(kComputeBar, NT);
             if ((L.dbg & 4) && tid == 0)
                 L.dbg_ts[8 * t + 7] = globaltimer();
-            // every warp scans the ITEMS x NW survivor counts itself (no wait on a
-            // single scanning warp); warp 0 also publishes the aggregate and reserves ring bytes
+            // every warp scans the ITEMS x NW survivor counts itself
             uint32_t pre[ITEMS];
             uint32_t total;
             {
@@ -448,7 +449,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
 #pragma unroll
                 for (int qq = 0; qq < PER; qq++) {
                     const int idx = lane * PER + qq;
-                    v[qq] = idx < NV ? ctl->cnt[idx] : 0;
+                    v[qq] = idx < NV ? cnt[idx] : 0;
                     sum += v[qq];
                 }
                 uint32_t inc = sum;
@@ -459,65 +460,58 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                         inc += y;
                 }
                 total = __shfl_sync(0xffffffffu, inc, 31);
-                // exclusive prefix of entry idx = (inc - sum) of its owner lane + preceding v's
                 const uint32_t base = inc - sum;
 #pragma unroll
                 for (int k = 0; k < ITEMS; k++) {
                     const int idx = k * NW + warp;
                     const int owner = idx / PER, off = idx % PER;
-                    uint32_t part = 0;
+                    uint32_t part_sum = 0;
 #pragma unroll
                     for (int qq = 0; qq < PER; qq++)
-                        if (qq < off) part += v[qq];
-                    const uint32_t b0 = __shfl_sync(0xffffffffu, base + part, owner);
-                    pre[k] = b0;
+                        if (qq < off) part_sum += v[qq];
+                    pre[k] = __shfl_sync(0xffffffffu, base + part_sum, owner);
                 }
             }
-            if (warp == 0) {
-                if (lane == 31) {
-                    // publish the tile aggregate before anything can block this CTA
-                    if (t > 0 && !(L.dbg & 1))
-                        st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
-                    if (L.dbg & 4)
-                        L.dbg_ts[8 * t + 2] = globaltimer();
-                }
-                if (lane == 0) {
-                    // reserve ring bytes for the compacted tile (blocks never wrap)
-                    uint32_t need = 0;
-                    for (int c = 0; c < P.nout; c++)
-                        need += al16(total * P.out_w[c]);
-                    const uint32_t head = ctl->head;
-                    uint32_t pos = ctl->hpos;
-                    uint32_t used = need;
-                    bool drain = false;
-                    if (pos + need > R) {           // blocks never wrap: skip the tail [pos, R)
-                        used += R - pos;
-                        pos = 0;
-                        if (used > R) {             // cannot fit behind live blocks: wait for an empty ring
-                            used = need;
-                            drain = true;
-                        }
-                    }
-                    ctl->hpos = pos + need == R ? 0 : pos + need;
-                    if (i >= kRingSlots)
-                        mbar_wait(&ctl->blk[j].oempty, (uint32_t)(((i / kRingSlots) - 1) & 1));
-                    uint32_t backoff = 32;
-                    while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
-                        __nanosleep(backoff);
-                        backoff = backoff < 512 ? backoff * 2 : 512;
-                    }
-                    ctl->head = head + used;
-                    ctl->roff = pos;
-                    ctl->blk[j].used = used;
+            if (warp == 0 && lane == 31) {
+                // publish the tile aggregate before anything can block this CTA
+                if (t > 0 && !(L.dbg & 1))
+                    st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
+                if (L.dbg & 4)
+                    L.dbg_ts[8 * t + 2] = globaltimer();
+            }
+            // ring bytes for the compacted tile (blocks never wrap); every warp computes
+            // the same reservation from the same (head, hpos, total)
+            uint32_t need = 0;
+            for (int c = 0; c < P.nout; c++)
+                need += al16(total * P.out_w[c]);
+            uint32_t pos = hpos;
+            uint32_t used = need;
+            bool drain = false;
+            if (pos + need > R) {           // skip the tail [pos, R)
+                used += R - pos;
+                pos = 0;
+                if (used > R) {             // cannot fit behind live blocks: wait for an empty ring
+                    used = need;
+                    drain = true;
                 }
             }
+            if (i >= kRingSlots)
+                mbar_wait(&ctl->blk[j].oempty, (uint32_t)(((i / kRingSlots) - 1) & 1));
+            {
+                uint32_t backoff = 32;
+                while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
+                    __nanosleep(backoff);
+                    backoff = backoff < 512 ? backoff * 2 : 512;
+                }
+            }
+            head += used;
+            hpos = pos + need == R ? 0 : pos + need;
+            char *blk = ring + pos;
             const uint32_t lt = lanemask_lt();
-            uint32_t pos[ITEMS];
+            uint32_t posk[ITEMS];
 #pragma unroll
             for (int k = 0; k < ITEMS; k++)
-                pos[k] = pre[k] + __popc(bal[k] & lt);
-            bar_sync(kComputeBar, NT);      // ring position known
-            char *blk = ring + ctl->roff;
+                posk[k] = pre[k] + __popc(bal[k] & lt);
             uint32_t coff = 0;
             for (int c = 0; c < P.nout; c++) {
                 const int w = P.out_w[c];
@@ -528,27 +522,30 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                 case 1:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint8_t *)dst)[pos[k]] = ((const uint8_t *)src)[k * NT + tid];
+                        if ((mask >> k) & 1u) ((uint8_t *)dst)[posk[k]] = ((const uint8_t *)src)[k * NT + tid];
                     break;
                 case 4:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint32_t *)dst)[pos[k]] = ((const uint32_t *)src)[k * NT + tid];
+                        if ((mask >> k) & 1u) ((uint32_t *)dst)[posk[k]] = ((const uint32_t *)src)[k * NT + tid];
                     break;
                 default:
 #pragma unroll
                     for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint64_t *)dst)[pos[k]] = ((const uint64_t *)src)[k * NT + tid];
+                        if ((mask >> k) & 1u) ((uint64_t *)dst)[posk[k]] = ((const uint64_t *)src)[k * NT + tid];
                     break;
                 }
             }
-            bar_sync(kComputeBar, NT);
-            if (tid == 0) {
-                mbar_arrive(&ctl->in[s].empty);          // input tile and scratch are free
-                ctl->blk[j].tile = t;
-                ctl->blk[j].total = total;
-                ctl->blk[j].roff = (uint32_t)(blk - ring);
-                mbar_arrive(&ctl->blk[j].aggr);
+            __syncwarp();
+            if (lane == 0) {
+                if (warp == 0) {
+                    ctl->blk[j].tile = t;
+                    ctl->blk[j].total = total;
+                    ctl->blk[j].roff = pos;
+                    ctl->blk[j].used = used;
+                }
+                mbar_arrive(&ctl->in[s].empty);          // this warp is done with the stage
+                mbar_arrive(&ctl->blk[j].aggr);          // and with the ring block
             }
         }
     }
@@ -775,115 +772,215 @@ __global__ void k_merge_splits(const __grid_constant__ JoinRunsLaunch J)
     J.split[p] = merge_path((const K *)J.lkey, J.nl, (const K *)J.rkey, J.nr, d);
 }
 
+// Two streaming passes (no look-back on the critical path): WRITE = false counts
+// the matched runs and join candidates of every partition; k_scan_parts turns the
+// counts into exclusive offsets; WRITE = true recomputes the partition (identical
+// arithmetic) and writes the run records at their offsets.  Phase timing showed the
+// single-pass version spent a third of its samples parked behind per-partition
+// look-backs.
+// first index in [start, n) of a sorted smem array with a[idx] > key (a[start-1] <= key)
 template <typename K>
-__global__ void __launch_bounds__(kThreads, 3) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
+__device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
+{
+    int lo = start, hi = n, step = 1;
+    while (true) {
+        const int probe = lo + step - 1;
+        if (probe >= n) { hi = n; break; }
+        if (a[probe] > key) { hi = probe; break; }
+        lo = probe + 1;
+        step <<= 1;
+    }
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (a[mid] <= key) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// Two streaming passes (no look-back on the critical path): WRITE = false counts
+// the matched runs and join candidates of every partition; k_scan_parts turns the
+// counts into exclusive offsets; WRITE = true recomputes the partition (identical
+// arithmetic) and writes the run records at their offsets.
+// Inside a partition thread t walks merged positions [8t, 8t+8) (L before R on equal
+// keys, P:196 binary-search partitioning, one diagonal search per thread): an L
+// element's R lower bound is the walk's R index; the R and L run ends are found by
+// galloping in smem (runs are short except for hot keys, which gallop on into HBM).
+template <typename K, bool WRITE>
+__global__ void __launch_bounds__(kThreads, 5) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
 {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    uint64_t *wtot = (uint64_t *)smem_raw;                        // kRunItems*kWarps + 1
+    uint64_t *wtot = (uint64_t *)smem_raw;                        // 2 * kWarps + 2
     K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT + kRunExt
     K *sR = sL + kRunT + kRunExt;                                 // kRunT + kRunExt
-    __shared__ int64_t sh_part, sh_base_runs, sh_base_outs;
     const K *L = (const K *)J.lkey;
     const K *R = (const K *)J.rkey;
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t ntot = J.nl + J.nr;
 
-    while (true) {
-        if (tid == 0)
-            sh_part = (int64_t)atomicAdd(&J.ctrs[0], 1u);
-        __syncthreads();
-        const int64_t p = sh_part;
-        if (p >= J.nparts)
-            break;
+    for (int64_t p = blockIdx.x; p < J.nparts; p += gridDim.x) {
         const int64_t d0 = p * kRunT, d1 = min(d0 + kRunT, ntot);
-        // partition splits were found by k_merge_splits (one thread per diagonal)
         const int64_t i0 = J.split[p], i1 = J.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
-        const int nL = (int)(i1 - i0);
-        // stage the partition plus kRunExt elements beyond it: runs cut by the partition
-        // boundary are then resolved in smem; only longer runs gallop through HBM
+        const int nL = (int)(i1 - i0), nR = (int)(j1 - j0), m = (int)(d1 - d0);
         const int nLe = (int)(min(i1 + kRunExt, J.nl) - i0), nRe = (int)(min(j1 + kRunExt, J.nr) - j0);
+        __syncthreads();
         for (int q = tid; q < nLe; q += kThreads)
             sL[q] = L[i0 + q];
         for (int q = tid; q < nRe; q += kThreads)
             sR[q] = R[j0 + q];
         __syncthreads();
 
-        uint64_t idx[kRunItems], cnt[kRunItems];
-        uint32_t rlenL[kRunItems], rlo[kRunItems], rlenR[kRunItems];
-        uint32_t emitted = 0;
-#pragma unroll
-        for (int k = 0; k < kRunItems; k++) {
-            const int li = k * kThreads + tid;
-            idx[k] = 0;
-            cnt[k] = 0;
-            rlenL[k] = rlo[k] = rlenR[k] = 0;
-            if (li < nL) {
+        // one walk over the thread's merged positions; `emit` writes the run records
+        // starting at (r, off) (second walk of the WRITE pass), else only counts
+        auto walk = [&](bool emit, int64_t r, uint64_t off, int &nrun, uint64_t &outs) {
+            nrun = 0;
+            outs = 0;
+            const int dt = tid * kRunItems;
+            if (dt >= m)
+                return;
+            int lo = dt > nR ? dt - nR : 0, hi = dt < nL ? dt : nL;
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (sL[mid] <= sR[dt - mid - 1]) lo = mid + 1;
+                else hi = mid;
+            }
+            int li = lo, rj = dt - lo;
+            const int end = min(dt + kRunItems, m);
+            for (int d = dt; d < end; d++) {
+                const bool takeL = rj >= nR || (li < nL && sL[li] <= sR[rj]);
+                if (!takeL) {
+                    rj++;
+                    continue;
+                }
                 const K key = sL[li];
                 const int64_t gi = i0 + li;
                 const bool start = gi == 0 || (li > 0 ? sL[li - 1] != key : L[gi - 1] != key);
-                if (start) {
-                    const int lo_l = lower_bound_smem(sR, nRe, key);
-                    const int hi_l = upper_bound_smem(sR, nRe, key);
-                    int64_t hi = j0 + hi_l;
-                    if (hi_l == nRe)
-                        hi = gallop_upper(R, hi, J.nr, key);
-                    const int64_t lo = j0 + lo_l;
-                    if (hi > lo) {
-                        const int e_l = li + upper_bound_smem(sL + li, nLe - li, key);
-                        int64_t iend = i0 + e_l;
-                        if (e_l == nLe)
-                            iend = gallop_upper(L, iend, J.nl, key);
-                        emitted |= 1u << k;
-                        idx[k] = 1;
-                        cnt[k] = (uint64_t)(iend - gi) * (uint64_t)(hi - lo);
-                        rlenL[k] = (uint32_t)(iend - gi);
-                        rlo[k] = (uint32_t)lo;
-                        rlenR[k] = (uint32_t)(hi - lo);
+                if (start && rj < nRe && sR[rj] == key) {
+                    // R elements with key < this key precede it in the merge: lower bound = rj
+                    const int e = gallop_smem(sR, rj + 1, nRe, key);
+                    int64_t rhi = j0 + e;
+                    if (e == nRe)
+                        rhi = gallop_upper(R, rhi, J.nr, key);
+                    const int64_t rlo64 = j0 + rj;
+                    const int el = gallop_smem(sL, li + 1, nLe, key);
+                    int64_t iend = i0 + el;
+                    if (el == nLe)
+                        iend = gallop_upper(L, iend, J.nl, key);
+                    const uint64_t c = (uint64_t)(iend - gi) * (uint64_t)(rhi - rlo64);
+                    if (emit && r < J.cap_runs) {
+                        J.s[r] = (uint32_t)gi;
+                        J.lenL[r] = (uint32_t)(iend - gi);
+                        J.lo[r] = (uint32_t)rlo64;
+                        J.lenR[r] = (uint32_t)(rhi - rlo64);
+                        J.off[r] = off;
                     }
+                    r++;
+                    off += c;
+                    outs += c;
+                    nrun++;
                 }
+                li++;
             }
-        }
-        uint64_t tot_runs, tot_outs;
-        block_scan_u64<kRunItems>(idx, wtot, tot_runs);
-        block_scan_u64<kRunItems>(cnt, wtot, tot_outs);
-        // the two look-backs (run count, output count) proceed in two warps at once
-        if (tid < 32) {
-            const uint64_t br = lookback_warp(J.status_runs, p, tot_runs, J.epoch_runs);
-            if (tid == 0) {
-                sh_base_runs = (int64_t)br;
-                if (p == J.nparts - 1)
-                    J.totals[0] = (int64_t)(br + tot_runs);
-            }
-        } else if (tid < 64) {
-            const uint64_t bo = lookback_warp(J.status_outs, p, tot_outs, J.epoch_outs);
-            if (tid == 32) {
-                sh_base_outs = (int64_t)bo;
-                if (p == J.nparts - 1)
-                    J.totals[1] = (int64_t)(bo + tot_outs);
-            }
-        }
-        __syncthreads();
-        const int64_t br = sh_base_runs, bo = sh_base_outs;
+        };
+        int nrun;
+        uint64_t outs;
+        walk(false, 0, 0, nrun, outs);
+        // block exclusive scan of (runs, outputs) over threads (thread order = merge order)
+        uint64_t ir = (uint64_t)nrun, io = outs;
 #pragma unroll
-        for (int k = 0; k < kRunItems; k++) {
-            if ((emitted >> k) & 1u) {
-                const int64_t r = br + (int64_t)idx[k];
-                if (r < J.cap_runs) {
-                    J.s[r] = (uint32_t)(i0 + k * kThreads + tid);
-                    J.lenL[r] = rlenL[k];
-                    J.lo[r] = rlo[k];
-                    J.lenR[r] = rlenR[k];
-                    J.off[r] = bo + cnt[k];
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t yr = __shfl_up_sync(0xffffffffu, ir, o), yo = __shfl_up_sync(0xffffffffu, io, o);
+            if (lane >= o) {
+                ir += yr;
+                io += yo;
+            }
+        }
+        if (lane == 31) {
+            wtot[warp] = ir;
+            wtot[kWarps + warp] = io;
+        }
+        __syncthreads();
+        uint64_t br = 0, bo = 0, tr = 0, to = 0;
+        for (int w = 0; w < kWarps; w++) {
+            if (w < warp) {
+                br += wtot[w];
+                bo += wtot[kWarps + w];
+            }
+            tr += wtot[w];
+            to += wtot[kWarps + w];
+        }
+        br += ir - (uint64_t)nrun;
+        bo += io - outs;
+        if (!WRITE) {
+            if (tid == 0) {
+                J.pruns[p] = tr;
+                J.pouts[p] = to;
+            }
+            continue;
+        }
+        int nr2;
+        uint64_t o2;
+        walk(true, (int64_t)J.pruns[p] + (int64_t)br, J.pouts[p] + bo, nr2, o2);
+    }
+}
+
+// exclusive scan of the per-partition counts (one CTA; nparts is ~ rows / 2048)
+__global__ void __launch_bounds__(1024) k_scan_parts(const __grid_constant__ JoinRunsLaunch J)
+{
+    __shared__ uint64_t wr[32], wo[32];
+    __shared__ uint64_t carry_r, carry_o;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0)
+        carry_r = carry_o = 0;
+    __syncthreads();
+    for (int64_t b0 = 0; b0 < J.nparts; b0 += 1024) {
+        const int64_t p = b0 + tid;
+        const uint64_t r = p < J.nparts ? J.pruns[p] : 0, o = p < J.nparts ? J.pouts[p] : 0;
+        uint64_t ir = r, io = o;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint64_t yr = __shfl_up_sync(0xffffffffu, ir, d), yo = __shfl_up_sync(0xffffffffu, io, d);
+            if (lane >= d) {
+                ir += yr;
+                io += yo;
+            }
+        }
+        if (lane == 31) {
+            wr[warp] = ir;
+            wo[warp] = io;
+        }
+        __syncthreads();
+        if (warp == 0) {
+            uint64_t xr = wr[lane], xo = wo[lane];
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint64_t yr = __shfl_up_sync(0xffffffffu, xr, d), yo = __shfl_up_sync(0xffffffffu, xo, d);
+                if (lane >= d) {
+                    xr += yr;
+                    xo += yo;
                 }
             }
+            wr[lane] = xr;
+            wo[lane] = xo;
+        }
+        __syncthreads();
+        const uint64_t er = carry_r + (warp ? wr[warp - 1] : 0) + ir - r;
+        const uint64_t eo = carry_o + (warp ? wo[warp - 1] : 0) + io - o;
+        if (p < J.nparts) {
+            J.pruns[p] = er;
+            J.pouts[p] = eo;
+        }
+        __syncthreads();
+        if (tid == 0) {
+            carry_r += wr[31];
+            carry_o += wo[31];
         }
         __syncthreads();
     }
-    if (J.nparts == 0 && blockIdx.x == 0 && tid == 0) {
-        J.totals[0] = 0;
-        J.totals[1] = 0;
+    if (tid == 0) {
+        J.totals[0] = (int64_t)carry_r;
+        J.totals[1] = (int64_t)carry_o;
     }
-    cta_exit_reset(J.ctrs);
 }
 
 // first run of every expansion tile: tile_run[t] = upper_bound(off, t*T) - 1
@@ -937,7 +1034,7 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + kAuxThreads)
                           : occ(k_scan_chain<256, 8, true, false>, smem, 256 + kAuxThreads);
     case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
-    default: return occ(k_join_runs<uint64_t>, smem);
+    default: return occ(k_join_runs<uint64_t, true>, smem);
     }
 }
 
@@ -982,8 +1079,15 @@ template <typename K>
 static cudaError_t jr(const JoinRunsLaunch &J, size_t smem, int grid, cudaStream_t s)
 {
     k_merge_splits<K><<<(unsigned)((J.nparts + 1 + 255) / 256), 256, 0, s>>>(J);
-    cudaFuncSetAttribute(k_join_runs<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_join_runs<K><<<grid, kThreads, smem, s>>>(J);
+    cudaFuncSetAttribute(k_join_runs<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_join_runs<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (J.nparts > 0) {
+        k_join_runs<K, false><<<grid, kThreads, smem, s>>>(J);
+        k_scan_parts<<<1, 1024, 0, s>>>(J);
+        k_join_runs<K, true><<<grid, kThreads, smem, s>>>(J);
+    } else {
+        k_scan_parts<<<1, 1024, 0, s>>>(J);
+    }
     return cudaGetLastError();
 }
 

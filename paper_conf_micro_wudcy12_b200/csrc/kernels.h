@@ -35,6 +35,7 @@ struct JoinRunsLaunch {
     uint32_t *ctrs;
     int64_t *totals;                 // [0] runs, [1] join candidates
     int64_t *split;                  // nparts + 1 merge-path splits (k_merge_splits)
+    uint64_t *pruns, *pouts;         // per-partition counts, then exclusive offsets
 };
 
 struct JoinExpand {

@@ -815,8 +815,8 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         //    1 CTA/SM with the deepest stage count whose ring holds >= 2.5 tiles.
         struct Cand { int occ, S; size_t Rb, smem; double score; };
         std::vector<Cand> cands;
-        for (int occ_t : {2, 1}) {
-            if (p->o.ctas_per_sm > 0 && occ_t != p->o.ctas_per_sm) continue;
+        for (int occ_t : {4, 3, 2, 1}) {
+            if (p->o.ctas_per_sm > 0 ? occ_t != p->o.ctas_per_sm : occ_t > 2) continue;
             const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
             for (int S = 1; S <= 6; S++) {
                 if (want_stages && S != want_stages) continue;
@@ -1060,11 +1060,13 @@ void run_group(ExecCtx &X, int gi)
         J.ctrs = p->ctrs;
         J.totals = p->jtot;
         J.split = (int64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
+        J.pruns = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
+        J.pouts = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
         const size_t smem1 = join_runs_smem(kt);
         const int occ1 = std::max(1, chain_occupancy(3, kThreads, 8, smem1));
         const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
         cuda_check(join_runs_launch(J, kt, smem1, grid1, p->stream), "k_join_runs");
-        p->launches += 2;
+        p->launches += 4;
         cuda_check(cudaMemcpyAsync(p->jtot_host, p->jtot, 16, cudaMemcpyDeviceToHost, p->stream), "copy totals");
         cuda_check(cudaStreamSynchronize(p->stream), "sync after join runs");
         const int64_t nruns = p->jtot_host[0], total = p->jtot_host[1];
