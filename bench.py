@@ -54,6 +54,9 @@ def parse():
     ap.add_argument("--ctas", type=int, default=0, help="CTAs per SM cap (0 = auto)")
     ap.add_argument("--defer", type=int, default=0, help="scan store delay in tiles (0 = auto)")
     ap.add_argument("--dbg", type=int, default=0, help="diagnostic ablations (not a bench value)")
+    ap.add_argument("--items", type=int, default=0, help="rows per thread of the scan tile (0 = auto)")
+    ap.add_argument("--variant", type=int, default=0, help="2 = 512x4, 3 = 512x8 compute threads x rows")
+    ap.add_argument("--gring", type=int, default=0, help="1 = compacted-tile ring in global memory (L2)")
     return ap.parse_args()
 
 
@@ -232,7 +235,7 @@ def main():
 
     def make(fuse):
         plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse, stages=args.stages,
-                                   ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg)
+                                   ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg, items=args.items, variant=args.variant, gring=args.gring)
         out_types = plan.node_schema(ids[spec["out"]])
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
         if cfg == "c3":

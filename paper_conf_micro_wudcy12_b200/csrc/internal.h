@@ -93,7 +93,8 @@ struct TileLaunch {
     int64_t n;                 // rows (scan) or join outputs (expand), if n_ptr == nullptr
     const int64_t *n_ptr;      // device row count written by an earlier kernel (else nullptr)
     int32_t stages;
-    uint32_t out_bytes;        // scan kernel: bytes of the compacted-tile ring
+    uint32_t out_bytes;        // scan kernel: bytes of the compacted-tile ring (per CTA)
+    char *gring;               // scan kernel: global ring, gridDim.x * out_bytes bytes (nullptr: in smem)
     int32_t direct;            // scan kernel: no SELECT in the group, rows stored at their offsets
     int32_t use_tma;           // input slots may be bulk-copied (16B-aligned bases)
     uint32_t epoch;            // look-back epoch tag (1..65535)

@@ -85,22 +85,29 @@ struct ScanCtl {
 __device__ __forceinline__ uint32_t al16(uint32_t x) { return (x + 15u) & ~15u; }
 
 template <typename T>
+__device__ __forceinline__ T ld_ring(const T *p, bool gring)
+{
+    return gring ? __ldcg(p) : *p;     // global ring: read through L2 (written by other warps)
+}
+
+template <typename T>
 __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t base, uint32_t total, int64_t cap,
-                                               int q, int nq)
+                                               int q, int nq, bool gring)
 {
     const int64_t lim = cap - base;
     const uint32_t m = (int64_t)total < lim ? total : (lim > 0 ? (uint32_t)lim : 0u);
     T *d = dst + base;
     uint32_t j = q;
     for (; j + 3 * nq < m; j += 4 * nq) {
-        const T a = src[j], b = src[j + nq], c = src[j + 2 * nq], e = src[j + 3 * nq];
+        const T a = ld_ring(src + j, gring), b = ld_ring(src + j + nq, gring), c = ld_ring(src + j + 2 * nq, gring),
+                e = ld_ring(src + j + 3 * nq, gring);
         d[j] = a;
         d[j + nq] = b;
         d[j + 2 * nq] = c;
         d[j + 3 * nq] = e;
     }
     for (; j < m; j += nq)
-        d[j] = src[j];
+        d[j] = ld_ring(src + j, gring);
 }
 
 // Join expansion into a tile (§8(a) a8): candidates [t*T, t*T + rows) of the
@@ -200,11 +207,16 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     ScanCtl<NT, ITEMS> *ctl = (ScanCtl<NT, ITEMS> *)smem_raw;
     char *stages = (char *)smem_raw + align_up(sizeof(ScanCtl<NT, ITEMS>), 128);
     char *scratch = stages + (size_t)S * P.stage_bytes;
-    char *ring = scratch + P.scratch_bytes;
-    unsigned long long *part = (unsigned long long *)(ring + (AGG ? 0 : R));
+    // compacted-tile ring: in smem, or (L.gring) a per-CTA slice of an L2-resident
+    // global buffer, which leaves the shared memory to more input stages
+    char *sm_ring = scratch + P.scratch_bytes;
+    const bool gring = L.gring != nullptr;
+    char *ring = gring ? L.gring + (size_t)blockIdx.x * R : sm_ring;
+    char *sm_after = sm_ring + ((AGG || gring) ? 0 : R);
+    unsigned long long *part = (unsigned long long *)sm_after;
     const int NA = P.nagg + 1;
     unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * NT : 0);
-    char *rcache = ring + (JOIN ? R : 0);   // join: run-record cache for the current tile
+    char *rcache = sm_after;                // join: run-record cache for the current tile
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
@@ -298,9 +310,9 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                     const char *src = blk + coff;
                     coff += al16(total * w);
                     switch (w) {
-                    case 1: group_copy_out<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, P.out_capacity, lane, 32); break;
-                    case 4: group_copy_out<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, P.out_capacity, lane, 32); break;
-                    default: group_copy_out<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, P.out_capacity, lane, 32); break;
+                    case 1: group_copy_out<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
+                    case 4: group_copy_out<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
+                    default: group_copy_out<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
                     }
                 }
                 __syncwarp();
@@ -538,6 +550,8 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
             }
             __syncwarp();
             if (lane == 0) {
+                if (gring)
+                    __threadfence_block();
                 if (warp == 0) {
                     ctl->blk[j].tile = t;
                     ctl->blk[j].total = total;
@@ -1002,7 +1016,7 @@ __global__ void k_tile_runs(const uint64_t *off, int64_t nruns, int64_t ntiles, 
 // ===========================================================================
 // Host launchers
 // ===========================================================================
-size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<256, 9>), 128); }   // >= every (NT, ITEMS) variant
+size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<512, 8>), 128); }   // >= every (NT, ITEMS) variant
 size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
 int scan_tile() { return kThreads * kScanItems; }
 int join_expand_tile() { return kThreads * kJoinItems; }
@@ -1026,9 +1040,14 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
 {
     switch (which) {
     case 0:
-        if (nt == 512) return occ(k_scan_chain<512, 4, false, false>, smem, 512 + kAuxThreads);
-        return items == 4 ? occ(k_scan_chain<256, 4, false, false>, smem, 256 + kAuxThreads)
-                          : occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
+        if (nt == 512) return items == 8 ? occ(k_scan_chain<512, 8, false, false>, smem, 512 + kAuxThreads)
+                                         : occ(k_scan_chain<512, 4, false, false>, smem, 512 + kAuxThreads);
+        switch (items) {
+        case 4: return occ(k_scan_chain<256, 4, false, false>, smem, 256 + kAuxThreads);
+        case 5: return occ(k_scan_chain<256, 5, false, false>, smem, 256 + kAuxThreads);
+        case 6: return occ(k_scan_chain<256, 6, false, false>, smem, 256 + kAuxThreads);
+        default: return occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
+        }
     case 1:
         if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + kAuxThreads);
         return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + kAuxThreads)
@@ -1065,8 +1084,13 @@ cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg,
         return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
     }
     if (nt == 512)
-        return sc<512, 4, false>(P, L, smem, grid, s);
-    return items == 4 ? sc<256, 4, false>(P, L, smem, grid, s) : sc<256, 8, false>(P, L, smem, grid, s);
+        return items == 8 ? sc<512, 8, false>(P, L, smem, grid, s) : sc<512, 4, false>(P, L, smem, grid, s);
+    switch (items) {
+    case 4: return sc<256, 4, false>(P, L, smem, grid, s);
+    case 5: return sc<256, 5, false>(P, L, smem, grid, s);
+    case 6: return sc<256, 6, false>(P, L, smem, grid, s);
+    default: return sc<256, 8, false>(P, L, smem, grid, s);
+    }
 }
 
 cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s)

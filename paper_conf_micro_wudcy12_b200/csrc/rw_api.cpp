@@ -93,6 +93,7 @@ struct Lowered {
     int items = 8, stages = 2, ctas = 1;
     int tile = 2048;              // rows per tile
     int nt = 256;                 // compute threads per CTA
+    uint32_t gring_bytes = 0;     // per-CTA global ring bytes (0: ring in smem)
     bool direct = false;          // no SELECT: outputs written at their row offsets
     int ring = 0;                 // scan kernel: output ring entries
     uint32_t out_bytes = 0;       // bytes of one output ring entry
@@ -117,6 +118,8 @@ struct rw_plan {
     int64_t *jtot = nullptr;      // join totals: 2 int64 per join group
     int64_t *jtot_host = nullptr; // pinned mirror
     int32_t *err = nullptr;       // [0] running domain errors, [1] last finalised
+    char *gring = nullptr;        // global compacted-tile rings (per CTA slices)
+    size_t gring_cap = 0;
     std::map<int, unsigned long long *> agg_acc;
     uint32_t epoch = 0;
     int64_t launches = 0;
@@ -783,6 +786,11 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     const size_t want_ring = p->o.reserved[0] > 0 ? (size_t)p->o.reserved[0] * 1024 : 0;
     bool ok = false;
     double best_score = -1;
+    // compacted-tile ring in global memory (L2-resident) instead of smem
+    // default on for compacting chains (measured: frees smem for a third input stage
+    // per CTA, C2 2.59 -> 2.29 ms); opts.reserved[6] == 2 keeps the ring in smem
+    const bool global_ring = !L.agg && p->o.reserved[6] != 2;
+    L.gring_bytes = 0;
     bool direct = !L.agg;
     for (const HOp &h : ops)
         if (h.kind == K_PRED)
@@ -792,10 +800,22 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     // 256 x 4 (1024-row tiles, wide rows); 512 x 4 on request (opts.reserved[4] == 2)
     struct Var { int nt, items; };
     std::vector<Var> vars;
+    const int force_items = p->o.reserved[5];              // diagnostics: force rows per thread
     if (!L.agg && p->o.reserved[4] == 2) vars.push_back({512, 4});
+    if (!L.agg && p->o.reserved[4] == 3) vars.push_back({512, 8});
     if (L.agg && p->o.reserved[4] != 1) vars.push_back({128, 16});   // halves the thread-private partials
     vars.push_back({256, 8});
+    if (!L.agg) {
+        vars.push_back({256, 6});
+        vars.push_back({256, 5});
+    }
     vars.push_back({256, 4});
+    if (force_items > 0) {
+        std::vector<Var> v2;
+        for (const Var &v : vars)
+            if (v.items == force_items) v2.push_back(v);
+        if (!v2.empty()) vars = v2;
+    }
     for (size_t ii = 0; ii < vars.size(); ii++) {
         const int items = vars[ii].items;
         const int nt = vars[ii].nt;
@@ -822,7 +842,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 if (want_stages && S != want_stages) continue;
                 if (base + (size_t)S * P.stage_bytes > per_cta) continue;
                 size_t Rb = 0;
-                if (!L.agg && !direct) {
+                if (!L.agg && !direct && !global_ring) {
                     Rb = want_ring ? want_ring : (per_cta - base - (size_t)S * P.stage_bytes) / 128 * 128;
                     if (Rb < W) continue;
                 }
@@ -831,13 +851,15 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 if (chain_occupancy(L.agg ? 1 : 0, nt, items, smem) < occ_t) continue;
                 double inflight = std::min<double>((double)occ_t * S * P.stage_bytes, 192.0 * 1024);
                 double score;
-                if (L.agg || direct) {
-                    score = inflight + (occ_t == 2 ? 1024.0 : 0) + S;
+                if (L.agg || direct || global_ring) {
+                    score = inflight + (occ_t == 2 ? 1024.0 : 0) + S + (double)T * 1e4 * (global_ring ? 1 : 0);
                 } else {
                     const double q = (double)Rb / (double)W;
-                    const bool ok2 = occ_t == 2 && q >= 1.9 && S == 2;
+                    const bool ok2 = occ_t == 2 && q >= 1.9 && S >= 2;
                     const bool ok1 = occ_t == 1 && q >= 2.5;
-                    score = (ok2 ? 1e9 : 0) + (ok1 ? 1e8 : 0) + inflight + q * 1024.0;
+                    // measured (scripts/sweep4.sh): per-tile overhead dominates, so the
+                    // largest tile wins before bytes in flight
+                    score = (ok2 ? 1e9 : 0) + (ok1 ? 1e8 : 0) + (double)T * 1e4 + inflight + q * 1024.0;
                 }
                 cands.push_back({occ_t, S, Rb, smem, score});
             }
@@ -863,6 +885,13 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     if (!ok)
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
     layout(L.tile);
+    if (global_ring && !L.direct) {
+        size_t W = 0;
+        for (int c = 0; c < P.nout; c++)
+            W += (((size_t)L.tile * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+        L.gring_bytes = (uint32_t)std::max<size_t>(128 * 1024, 4 * W);
+        L.out_bytes = L.gring_bytes;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -1000,12 +1029,21 @@ void run_group(ExecCtx &X, int gi)
         TL.dbg_ts = (uint64_t *)(((uint64_t)(uint32_t)p->o.reserved[3] << 32) | (uint32_t)p->o.reserved[2]);
         TL.out_bytes = L.out_bytes;
         TL.direct = L.direct ? 1 : 0;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(max_tiles, (int64_t)p->sms * L.ctas));
+        if (L.gring_bytes) {
+            const size_t need = (size_t)grid * L.gring_bytes;
+            if (need > p->gring_cap) {
+                if (p->gring) cudaFreeAsync(p->gring, p->stream);
+                p->gring = (char *)dev_alloc(p, need);
+                p->gring_cap = need;
+            }
+            TL.gring = p->gring;
+        }
         TL.use_tma = aligned ? 1 : 0;
         TL.epoch = next_epoch(p);
         TL.status = p->status;
         TL.ctrs = p->ctrs;
         TL.err = p->err;
-        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(max_tiles, (int64_t)p->sms * L.ctas));
         if (L.agg) {
             const Node &an = p->nodes[g.agg];
             const size_t words = (size_t)an.D * (L.P.nagg + 1) * 2;
@@ -1351,6 +1389,7 @@ void rw_plan_destroy(rw_plan *p)
     if (p->cnt) cudaFree(p->cnt);
     if (p->jtot) cudaFree(p->jtot);
     if (p->err) cudaFree(p->err);
+    if (p->gring) cudaFree(p->gring);
     if (p->jtot_host) cudaFreeHost(p->jtot_host);
     delete p;
 }

@@ -154,7 +154,8 @@ class Plan:
 
     def __init__(self, device: int = 0, stream=None, fuse: bool = True, zero_copy_project: bool = False,
                  stages: int = 0, ctas_per_sm: int = 0, strict_overflow: bool = False, defer: int = 0,
-                 dbg: int = 0, dbg_ts: int = 0):
+                 dbg: int = 0, dbg_ts: int = 0, items: int = 0, variant: int = 0,
+                 gring: int = 0):
         import torch
         if stream is None:
             stream = torch.cuda.current_stream(device)
@@ -170,6 +171,9 @@ class Plan:
         o.reserved[1] = dbg                # diagnostics only (1: no look-back, 2: stream only, 4: timestamps)
         o.reserved[2] = ctypes.c_int32(dbg_ts & 0xffffffff).value
         o.reserved[3] = ctypes.c_int32((dbg_ts >> 32) & 0xffffffff).value
+        o.reserved[5] = items              # tuning: rows per thread of the scan tile (0 = auto)
+        o.reserved[4] = variant            # tuning: 2 = 512x4, 3 = 512x8 compute threads x rows
+        o.reserved[6] = gring              # tuning: 1 = compacted-tile ring in global memory (L2)
         self.device = device
         h = ctypes.c_void_p()
         check(lib().rw_plan_create(ctypes.byref(h), ctypes.byref(o)))
