@@ -239,6 +239,29 @@ __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, cons
     }
 }
 
+// Fused fixed-point factor (plan peephole of MUL over ADD/RSUB with a constant,
+// e.g. Q1's price * (100 - disc) and disc_price * (100 + tax), P:223 pattern (e)):
+// dst = a * (k +- b), all three of type T, wrapping mod 2^w like the two ops it replaces.
+template <int NT, int ITEMS, typename T>
+__device__ __forceinline__ void mulaff_loop(char *dst, const char *a, const char *b, T k, bool neg)
+{
+    typedef typename std::make_unsigned<T>::type U;
+    const int tid = threadIdx.x;
+    if (neg) {
+#pragma unroll
+        for (int i = 0; i < ITEMS; i++) {
+            const int r = i * NT + tid;
+            ((T *)dst)[r] = (T)((U)ld_as<T>(a, r) * ((U)k - (U)ld_as<T>(b, r)));
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < ITEMS; i++) {
+            const int r = i * NT + tid;
+            ((T *)dst)[r] = (T)((U)ld_as<T>(a, r) * ((U)k + (U)ld_as<T>(b, r)));
+        }
+    }
+}
+
 #define RW_EXPR_CASES(TT, TCODE)                                                                                  \
     case TCODE * 8 + E_COPY: expr_loop<NT, ITEMS, TT, E_COPY, false>(dst, a, ta, b, tb, (TT)k); return;       \
     case TCODE * 8 + E_CONST: expr_loop<NT, ITEMS, TT, E_CONST, false>(dst, a, ta, b, tb, (TT)k); return;     \
@@ -249,7 +272,8 @@ __device__ __forceinline__ void expr_loop(char *dst, const char *a, int ta, cons
     case TCODE * 8 + E_RSUB: expr_loop<NT, ITEMS, TT, E_RSUB, false>(dst, a, ta, b, tb, (TT)k); return;       \
     case 64 + TCODE * 8 + E_ADD: expr_loop<NT, ITEMS, TT, E_ADD, true>(dst, a, ta, b, tb, (TT)0); return;       \
     case 64 + TCODE * 8 + E_SUB: expr_loop<NT, ITEMS, TT, E_SUB, true>(dst, a, ta, b, tb, (TT)0); return;       \
-    case 64 + TCODE * 8 + E_MUL: expr_loop<NT, ITEMS, TT, E_MUL, true>(dst, a, ta, b, tb, (TT)0); return;
+    case 64 + TCODE * 8 + E_MUL: expr_loop<NT, ITEMS, TT, E_MUL, true>(dst, a, ta, b, tb, (TT)0); return;       \
+    case 64 + TCODE * 8 + E_MULAFF: mulaff_loop<NT, ITEMS, TT>(dst, a, b, (TT)k, (tb & kNegB) != 0); return;
 
 template <int NT, int ITEMS>
 __device__ __noinline__ void run_expr(uint32_t code, int ta, int tb, int64_t k, char *dst, const char *a, const char *b)
@@ -450,6 +474,41 @@ __device__ inline void agg_tile_rowwise(const ChainProg &P, const char *stage, c
     }
 }
 
+// Global-atomic terminal (agg_mode 3) for group-bys too large for per-thread
+// partials in shared memory: every row adds into the global 128-bit accumulators.
+template <int NT, int ITEMS>
+__device__ inline void agg_tile_global(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
+                                       unsigned long long *acc, int32_t *err)
+{
+    const int tid = threadIdx.x;
+    const int NA = P.nagg + 1;
+#pragma unroll 1
+    for (int k = 0; k < ITEMS; k++) {
+        if (!((mask >> k) & 1u))
+            continue;
+        const int r = k * NT + tid;
+        int g = 0;
+        bool ok = true;
+        for (int c = 0; c < P.ngc; c++) {
+            const uint64_t code = ld_ext(loc_ptr(P.g_loc[c], stage, scratch), P.g_type[c], r);
+            if (code >= (uint64_t)P.gdomain[c])
+                ok = false;
+            g = g * P.gdomain[c] + (int)code;
+        }
+        if (!ok) {
+            atomicAdd(err, 1);
+            continue;
+        }
+        unsigned long long *pg = acc + 2 * (size_t)g * NA;
+        atomic_add128(&pg[0], &pg[1], 1ull, 0ull);
+        for (int a = 0; a < P.nagg; a++) {
+            const unsigned long long v = ld_ext(loc_ptr(P.agg_loc[a], stage, scratch), P.agg_type[a], r);
+            const unsigned long long hi = (!P.agg_unsigned[a] && (long long)v < 0) ? ~0ull : 0ull;
+            atomic_add128(&pg[2 * (a + 1)], &pg[2 * (a + 1) + 1], v, hi);
+        }
+    }
+}
+
 constexpr int kAggUnroll = 8;
 
 // Tile-wise aggregate terminal: group codes of the thread's ITEMS rows computed
@@ -535,6 +594,168 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
             }
         }
     }
+}
+
+// Register terminal (agg_mode 2) for small group-bys (D <= kRegD groups, nagg <=
+// kRegA sums, e.g. Q1's 6 x 5): every compute thread keeps its int64 partials of
+// all (group, sum) pairs in registers and adds a row into the pairs of its group
+// with predicated adds (one-hot over the D groups, no shared-memory traffic and no
+// dependent read-modify-write chains).  The plan picks this mode only when the
+// interval analysis allows >= 2^16 rows per thread between flushes; a flush adds
+// the registers into the CTA's 128-bit accumulators.
+struct RegAgg {
+    uint64_t s[kRegD][kRegA];
+    uint32_t c[kRegD];
+};
+
+__device__ __forceinline__ void reg_agg_zero(RegAgg &R)
+{
+#pragma unroll
+    for (int d = 0; d < kRegD; d++) {
+        R.c[d] = 0;
+#pragma unroll
+        for (int a = 0; a < kRegA; a++)
+            R.s[d][a] = 0;
+    }
+}
+
+// adds the registers into 128-bit accumulators acc[2*(g*NA + a)] (shared, atomically)
+__device__ inline void reg_agg_flush(const ChainProg &P, RegAgg &R, unsigned long long *acc)
+{
+    const int NA = P.nagg + 1;
+#pragma unroll
+    for (int d = 0; d < kRegD; d++) {
+        if (d < P.D && R.c[d]) {
+            atomic_add128(&acc[2 * (d * NA)], &acc[2 * (d * NA) + 1], R.c[d], 0ull);
+#pragma unroll
+            for (int a = 0; a < kRegA; a++) {
+                if (a < P.nagg) {
+                    const unsigned long long v = R.s[d][a];
+                    const unsigned long long hi = (!P.agg_unsigned[a] && (long long)v < 0) ? ~0ull : 0ull;
+                    atomic_add128(&acc[2 * (d * NA + 1 + a)], &acc[2 * (d * NA + 1 + a) + 1], v, hi);
+                }
+            }
+        }
+    }
+    reg_agg_zero(R);
+}
+
+// stores the registers as thread-private partials part[(g*NA + a)*NT + tid] for agg_combine
+template <int NT>
+__device__ inline void reg_agg_store(const ChainProg &P, const RegAgg &R, unsigned long long *part)
+{
+    const int NA = P.nagg + 1, tid = threadIdx.x;
+#pragma unroll
+    for (int d = 0; d < kRegD; d++) {
+        if (d < P.D) {
+            part[(d * NA) * NT + tid] = R.c[d];
+#pragma unroll
+            for (int a = 0; a < kRegA; a++)
+                if (a < P.nagg)
+                    part[(d * NA + 1 + a) * NT + tid] = R.s[d][a];
+        }
+    }
+}
+
+// Row loop of the register terminal: NAGG sums (W64: every sum column is 64-bit, so
+// no per-row type dispatch); the one-hot over the groups becomes a jump to the
+// row's group, whose partials take predicated-free adds.
+template <int NT, int ITEMS, int NAGG, bool W64>
+__device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *at, const uint32_t *g, uint32_t ok,
+                                             RegAgg &R)
+{
+    const int tid = threadIdx.x;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const uint32_t gk = ((ok >> k) & 1u) ? g[k] : 0xffffffffu;   // failing rows match no group
+        const int r = k * NT + tid;
+        uint64_t v[kRegA];
+#pragma unroll
+        for (int a = 0; a < kRegA; a++)
+            v[a] = a < NAGG ? (W64 ? ((const uint64_t *)ab[a])[r] : ld_ext(ab[a], at[a], r)) : 0ull;
+#pragma unroll
+        for (int d = 0; d < kRegD; d++) {
+            if (gk == (uint32_t)d) {
+                R.c[d] += 1u;
+#pragma unroll
+                for (int a = 0; a < NAGG; a++)
+                    R.s[d][a] += v[a];
+            }
+        }
+    }
+}
+
+template <int NT, int ITEMS>
+__device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
+                                    RegAgg &R, unsigned long long *cta_acc, int64_t &since_flush, int32_t *err)
+{
+    const int tid = threadIdx.x;
+    uint32_t g[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++)
+        g[k] = 0;
+    uint32_t ok = mask;
+    for (int c = 0; c < P.ngc; c++) {
+        const char *b = loc_ptr(P.g_loc[c], stage, scratch);
+        const uint32_t dom = (uint32_t)P.gdomain[c];
+        switch (P.g_type[c]) {
+        case T_U8:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint8_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        case T_I32:
+        case T_U32:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint32_t *)b)[k * NT + tid];   // negative i32 -> huge
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        default:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint64_t v = ((const uint64_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + (uint32_t)v;
+            }
+            break;
+        }
+    }
+    if (ok != mask)
+        atomicAdd(err, __popc(mask & ~ok));
+    const int rows = __popc(ok);
+    if (since_flush + rows > P.flush_rows) {
+        reg_agg_flush(P, R, cta_acc);
+        since_flush = 0;
+    }
+    since_flush += rows;
+    const char *ab[kRegA];
+    int at[kRegA];
+    bool w64 = true;
+#pragma unroll
+    for (int a = 0; a < kRegA; a++) {
+        ab[a] = a < P.nagg ? loc_ptr(P.agg_loc[a], stage, scratch) : nullptr;
+        at[a] = a < P.nagg ? P.agg_type[a] : T_U64;
+        if (a < P.nagg && !(at[a] == T_I64 || at[a] == T_U64))
+            w64 = false;
+    }
+    // the sum count and the all-64-bit case are compile-time in the row loop
+    if (w64) {
+        switch (P.nagg) {
+        case 0: agg_rows_reg<NT, ITEMS, 0, true>(ab, at, g, ok, R); return;
+        case 1: agg_rows_reg<NT, ITEMS, 1, true>(ab, at, g, ok, R); return;
+        case 2: agg_rows_reg<NT, ITEMS, 2, true>(ab, at, g, ok, R); return;
+        case 3: agg_rows_reg<NT, ITEMS, 3, true>(ab, at, g, ok, R); return;
+        case 4: agg_rows_reg<NT, ITEMS, 4, true>(ab, at, g, ok, R); return;
+        default: agg_rows_reg<NT, ITEMS, kRegA, true>(ab, at, g, ok, R); return;
+        }
+    }
+    agg_rows_reg<NT, ITEMS, kRegA, false>(ab, at, g, ok, R);
 }
 
 // End-of-kernel combine of the thread-private partials: one thread per (group,

@@ -28,12 +28,16 @@ constexpr int kThreads = 256;        // threads per CTA for every chain kernel
 constexpr int kScanItems = 8;        // rows per thread per tile in the scan kernel (T = 2048)
 constexpr int kJoinItems = 9;        // outputs per thread per tile in the join expansion (T = 2304,
                                      // odd stride -> conflict-free thread-contiguous smem writes)
-constexpr int kMaxAggSlots = 4096;   // D * (nagg + 1) upper bound for the agg terminal
+constexpr int kMaxAggSlots = 4096;
+constexpr int kRegD = 6;             // register aggregate terminal: groups x sums held per thread
+constexpr int kRegA = 5;   // D * (nagg + 1) upper bound for the agg terminal
 
 enum Type : uint8_t { T_I32 = 0, T_U32 = 1, T_I64 = 2, T_U64 = 3, T_U8 = 4 };
 enum Cmp : uint8_t { C_LT = 0, C_LE = 1, C_GT = 2, C_GE = 3, C_EQ = 4, C_NE = 5 };
 enum OpKind : uint8_t { K_PRED = 0, K_EXPR = 1 };
-enum ExprOp : uint8_t { E_COPY = 0, E_CONST = 1, E_ADD = 2, E_SUB = 3, E_MUL = 4, E_DIVC = 5, E_RSUB = 6 };
+enum ExprOp : uint8_t { E_COPY = 0, E_CONST = 1, E_ADD = 2, E_SUB = 3, E_MUL = 4, E_DIVC = 5, E_RSUB = 6,
+                        E_MULAFF = 7 };   // dst = a * (k + b), or a * (k - b) when tb has kNegB set
+constexpr uint8_t kNegB = 0x80;
 
 __host__ __device__ inline int type_width(int t) { return t == T_U8 ? 1 : (t == T_I64 || t == T_U64) ? 8 : 4; }
 __host__ __device__ inline bool type_signed(int t) { return t == T_I32 || t == T_I64; }
@@ -84,6 +88,7 @@ struct ChainProg {
     uint8_t agg_type[kMaxAggs];
     uint8_t agg_unsigned[kMaxAggs];     // 1: u64 sum (unsigned partials)
     int64_t flush_rows;                 // rows a thread may add before its int64 partials can overflow
+    int32_t agg_mode;                   // 0: thread-private partials in smem; 2: register one-hot (D <= kRegD, nagg <= kRegA)
     uint32_t stage_bytes;               // bytes of one stage (all input slots, aligned)
     uint32_t scratch_bytes;             // bytes of scratch (computed slots)
 };

@@ -195,7 +195,7 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
 }
 
 template <int NT, int ITEMS, bool AGG, bool JOIN>
-__global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid_constant__ ChainProg P,
+__global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(const __grid_constant__ ChainProg P,
                                                                      const __grid_constant__ TileLaunch L,
                                                                      const __grid_constant__ JoinExpand X)
 {
@@ -215,7 +215,11 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     char *sm_after = sm_ring + ((AGG || gring) ? 0 : R);
     unsigned long long *part = (unsigned long long *)sm_after;
     const int NA = P.nagg + 1;
-    unsigned long long *cta_acc = part + (AGG ? (size_t)P.D * NA * NT : 0);
+    // agg_mode 0: thread-private int64 partials (D*NA*NT words); 2: partials in
+    // registers (stored into the stage buffers at the end); then the CTA's 128-bit
+    // accumulators
+    const size_t part_words = AGG ? (P.agg_mode == 0 ? (size_t)P.D * NA * NT : 0) : 0;
+    unsigned long long *cta_acc = part + part_words;
     char *rcache = sm_after;                // join: run-record cache for the current tile
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
@@ -237,7 +241,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
         fence_mbar_init();
     }
     if (AGG) {
-        for (int q = tid; q < P.D * NA * NT; q += blockDim.x)
+        for (size_t q = tid; q < part_words; q += blockDim.x)
             part[q] = 0;
         for (int q = tid; q < P.D * NA * 2; q += blockDim.x)
             cta_acc[q] = 0;
@@ -316,12 +320,25 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                     }
                 }
                 __syncwarp();
+                if (gring && !(L.dbg & 8)) {
+                    // the block has been copied out (every loaded value was stored): drop
+                    // its fully covered L2 lines so the ring never costs DRAM write-back
+                    const uintptr_t b0 = ((uintptr_t)blk + 127) & ~(uintptr_t)127;
+                    const uintptr_t b1 = ((uintptr_t)blk + coff) & ~(uintptr_t)127;
+                    for (uintptr_t a = b0 + (uintptr_t)lane * 128; a < b1; a += 32 * 128)
+                        discard_l2_line((const void *)a);
+                    __syncwarp();
+                }
                 if (lane == 0) {
                     if (L.dbg & 4)
                         L.dbg_ts[8 * t + 4] = globaltimer();
                     if (i > 0)   // release ring bytes in tile order
                         mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1));
-                    __threadfence_block();
+                    // the discards must land in L2 before the bytes can be rewritten
+                    if (gring && !(L.dbg & 8))
+                        __threadfence();
+                    else
+                        __threadfence_block();
                     ctl->tail = ctl->tail + ctl->blk[j].used;
                     mbar_arrive(&ctl->blk[j].oempty);
                 }
@@ -336,6 +353,9 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
         // and the compacted block handed to the writers by per-warp mbarrier arrivals
         // (count = NW); the ring reservation is replicated, deterministically, in every warp.
         int64_t since_flush = 0;
+        RegAgg racc;
+        if (AGG && P.agg_mode == 2)
+            reg_agg_zero(racc);
         int s = 0;
         uint32_t fph = 0;
         uint32_t head = 0, hpos = 0;
@@ -357,6 +377,12 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
                         ctl->blk[ju].tile = ntiles;
                         mbar_arrive_cnt(&ctl->blk[ju].aggr, NW);
                     }
+                }
+                if (AGG && P.agg_mode == 2) {
+                    // every compute warp is past its last stage (no TMA is pending once the
+                    // sentinel is reached): the stage buffers take the register partials
+                    bar_sync(kComputeBar, NT);
+                    reg_agg_store<NT>(P, racc, (unsigned long long *)stages);
                 }
                 break;
             }
@@ -406,7 +432,12 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
             if ((L.dbg & 4) && tid == 0)
                 L.dbg_ts[8 * t + 6] = globaltimer();
             if (AGG) {
-                agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
+                if (P.agg_mode == 2)
+                    agg_tile_reg<NT, ITEMS>(P, st, scratch, mask, racc, cta_acc, since_flush, L.err);
+                else if (P.agg_mode == 3)
+                    agg_tile_global<NT, ITEMS>(P, st, scratch, mask, L.agg_acc, L.err);
+                else
+                    agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
                 if ((L.dbg & 4) && tid == 0)
                     L.dbg_ts[8 * t + 2] = globaltimer();
                 release_stage();
@@ -565,7 +596,8 @@ __global__ void __launch_bounds__(NT + kAuxThreads, 2) k_scan_chain(const __grid
     }
     __syncthreads();
     if (AGG) {
-        agg_combine<NT>(P, part, cta_acc, blockDim.x);
+        if (P.agg_mode != 3)      // mode 3 added every row into the global accumulators already
+            agg_combine<NT>(P, P.agg_mode == 2 ? (unsigned long long *)stages : part, cta_acc, blockDim.x);
         __syncthreads();
         for (int qq = tid; qq < P.D * NA; qq += blockDim.x) {
             const unsigned long long lo = cta_acc[2 * qq], hi = cta_acc[2 * qq + 1];

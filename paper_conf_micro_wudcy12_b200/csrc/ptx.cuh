@@ -128,6 +128,12 @@ __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+// Drop one 128-byte L2 line without writing it back (its contents become undefined).
+__device__ __forceinline__ void discard_l2_line(const void *p)
+{
+    asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
+}
+
 __device__ __forceinline__ uint64_t globaltimer()
 {
     uint64_t t;

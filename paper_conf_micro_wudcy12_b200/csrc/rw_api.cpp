@@ -619,6 +619,47 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     if ((int)slots.size() > kMaxSlots)
         raise(RW_E_UNSUPPORTED, "fused group needs more than 24 tile columns");
 
+    // peephole: MUL(x, y) with y = k + z or k - z (z a slot, k a constant, same type,
+    // y used by nothing else) becomes one fused factor op dst = x * (k +- z)
+    {
+        std::vector<int> uses(slots.size(), 0), producer(slots.size(), -1);
+        for (size_t i = 0; i < ops.size(); i++) {
+            const HOp &o = ops[i];
+            if (o.a >= 0) uses[o.a]++;
+            if (o.b_is_slot && o.b >= 0) uses[o.b]++;
+            if (o.kind == K_EXPR && o.dst >= 0) producer[o.dst] = (int)i;
+        }
+        for (int s : term) uses[s] += 2;
+        std::vector<char> dead(ops.size(), 0);
+        for (size_t i = 0; i < ops.size(); i++) {
+            HOp &o = ops[i];
+            if (o.kind != K_EXPR || o.op != E_MUL || !o.b_is_slot || o.a < 0 || o.b < 0) continue;
+            for (int side = 0; side < 2; side++) {
+                const int y = side ? o.a : o.b, x = side ? o.b : o.a;
+                const int j = producer[y];
+                if (j < 0 || dead[j] || uses[y] != 1) continue;
+                const HOp &f = ops[j];
+                if (f.kind != K_EXPR || f.b_is_slot || f.a < 0 || (f.op != E_ADD && f.op != E_RSUB)) continue;
+                if (f.type != o.type || slots[f.a].type != o.type || slots[x].type != o.type) continue;
+                if (slots[f.a].input == false && producer[f.a] > (int)i) continue;
+                HOp m = o;
+                m.op = E_MULAFF;
+                m.a = (int16_t)x;
+                m.b = (int16_t)f.a;
+                m.b_is_slot = 1;
+                m.k = f.k;
+                m.pad = f.op == E_RSUB ? 1 : 0;          // 1: k - z
+                o = m;
+                dead[j] = 1;
+                break;
+            }
+        }
+        std::vector<HOp> kept;
+        for (size_t i = 0; i < ops.size(); i++)
+            if (!dead[i]) kept.push_back(ops[i]);
+        ops.swap(kept);
+    }
+
     // liveness
     for (size_t i = 0; i < ops.size(); i++) {
         const HOp &o = ops[i];
@@ -721,6 +762,8 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             d.code = (uint8_t)(h.type * 8 + h.op + (h.b_is_slot ? 64 : 0));
             d.ta = h.a >= 0 ? P.slot[h.a].type : (uint8_t)h.type;
             d.tb = (h.b_is_slot && h.b >= 0) ? P.slot[h.b].type : (uint8_t)h.type;
+            if (h.op == E_MULAFF && h.kind == K_EXPR && h.pad)
+                d.tb |= kNegB;
             d.a = loc(h.a);
             d.b = h.b_is_slot ? loc(h.b) : 0;
             d.dst = h.dst >= 0 ? loc(h.dst) : 0;
@@ -740,8 +783,24 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             P.agg_type[q] = P.slot[P.agg_slot[q]].type;
         }
     };
+    // aggregate terminal: warp reduce-by-key (agg_mode 1, per-warp 128-bit accumulators)
+    // when the sums fit its unrolled loop and the per-warp accumulators are small;
+    // else thread-private int64 partials (opts.reserved[7] == 1 forces the latter)
+    // aggregate terminal: 2 = register one-hot (small D x sums, long flush period);
+    // 0 = thread-private int64 partials in smem; 3 = per-row 128-bit global atomics
+    // (group-bys whose partials exceed shared memory).  opts.reserved[7] == 1 forces 0.
+    auto agg_mode_for = [&](int nt) -> int {
+        if (!L.agg) return 0;
+        const size_t slots = (size_t)P.D * (P.nagg + 1);
+        if (p->o.reserved[7] == 1) return 0;
+        if (P.D <= kRegD && P.nagg <= kRegA && P.flush_rows >= (1 << 16)) return 2;
+        return slots * nt * 8 <= 150 * 1024 ? 0 : 3;
+    };
     auto agg_bytes_for = [&](int nt) -> size_t {
-        return L.agg ? (size_t)P.D * (P.nagg + 1) * nt * 8 + al128((size_t)P.D * (P.nagg + 1) * 16) : 0;
+        if (!L.agg) return 0;
+        const size_t slots = (size_t)P.D * (P.nagg + 1);
+        const size_t part = agg_mode_for(nt) == 0 ? slots * nt * 8 : 0;
+        return part + al128(slots * 16);
     };
     if (L.agg && (size_t)P.D * (P.nagg + 1) > (size_t)kMaxAggSlots)
         raise(RW_E_UNSUPPORTED, "aggregate needs more than 4096 accumulators");
@@ -803,7 +862,8 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     const int force_items = p->o.reserved[5];              // diagnostics: force rows per thread
     if (!L.agg && p->o.reserved[4] == 2) vars.push_back({512, 4});
     if (!L.agg && p->o.reserved[4] == 3) vars.push_back({512, 8});
-    if (L.agg && p->o.reserved[4] != 1) vars.push_back({128, 16});   // halves the thread-private partials
+    if (L.agg && p->o.reserved[4] != 1 && !agg_mode_for(256))
+        vars.push_back({128, 16});   // halves the thread-private partials
     vars.push_back({256, 8});
     if (!L.agg) {
         vars.push_back({256, 6});
@@ -841,6 +901,10 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             for (int S = 1; S <= 6; S++) {
                 if (want_stages && S != want_stages) continue;
                 if (base + (size_t)S * P.stage_bytes > per_cta) continue;
+                // register terminal: the stage + scratch buffers take the partials at the end
+                if (agg_mode_for(nt) == 2 &&
+                    (size_t)S * P.stage_bytes + P.scratch_bytes < (size_t)P.D * (P.nagg + 1) * nt * 8)
+                    continue;
                 size_t Rb = 0;
                 if (!L.agg && !direct && !global_ring) {
                     Rb = want_ring ? want_ring : (per_cta - base - (size_t)S * P.stage_bytes) / 128 * 128;
@@ -852,7 +916,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 double inflight = std::min<double>((double)occ_t * S * P.stage_bytes, 192.0 * 1024);
                 double score;
                 if (L.agg || direct || global_ring) {
-                    score = inflight + (occ_t == 2 ? 1024.0 : 0) + S + (double)T * 1e4 * (global_ring ? 1 : 0);
+                    // (measured: the largest tile wins for the aggregate and the ring, since
+                    // the interpreter's per-op dispatch is amortised over the rows per thread)
+                    score = inflight + (occ_t == 2 ? 1024.0 : 0) + S + (double)T * 1e4 * ((global_ring || L.agg) ? 1 : 0);
                 } else {
                     const double q = (double)Rb / (double)W;
                     const bool ok2 = occ_t == 2 && q >= 1.9 && S >= 2;
@@ -885,6 +951,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     if (!ok)
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
     layout(L.tile);
+    P.agg_mode = agg_mode_for(L.nt);
     if (global_ring && !L.direct) {
         size_t W = 0;
         for (int c = 0; c < P.nout; c++)
@@ -1275,8 +1342,15 @@ std::string explain(rw_plan *p, int out_node)
               << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
               << L.P.nops;
             if (L.agg)
-                s << ", groups " << L.P.D << ", sums " << L.P.nagg << ", partial flush every " << L.P.flush_rows
-                  << " rows";
+            {
+                s << ", groups " << L.P.D << ", sums " << L.P.nagg;
+                if (L.P.agg_mode == 2)
+                    s << ", register one-hot terminal";
+                else if (L.P.agg_mode == 3)
+                    s << ", global-atomic terminal";
+                else
+                    s << ", partial flush every " << L.P.flush_rows << " rows";
+            }
         } catch (const RwError &e) {
             s << " | not lowerable: " << e.msg;
         }

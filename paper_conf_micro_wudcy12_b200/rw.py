@@ -155,7 +155,7 @@ class Plan:
     def __init__(self, device: int = 0, stream=None, fuse: bool = True, zero_copy_project: bool = False,
                  stages: int = 0, ctas_per_sm: int = 0, strict_overflow: bool = False, defer: int = 0,
                  dbg: int = 0, dbg_ts: int = 0, items: int = 0, variant: int = 0,
-                 gring: int = 0):
+                 gring: int = 0, agg_mode: int = 0):
         import torch
         if stream is None:
             stream = torch.cuda.current_stream(device)
@@ -174,6 +174,7 @@ class Plan:
         o.reserved[5] = items              # tuning: rows per thread of the scan tile (0 = auto)
         o.reserved[4] = variant            # tuning: 2 = 512x4, 3 = 512x8 compute threads x rows
         o.reserved[6] = gring              # tuning: 1 = compacted-tile ring in global memory (L2)
+        o.reserved[7] = agg_mode           # 1 = force the thread-private-partials aggregate terminal
         self.device = device
         h = ctypes.c_void_p()
         check(lib().rw_plan_create(ctypes.byref(h), ctypes.byref(o)))

@@ -41,6 +41,7 @@ def run_gpu(spec: Dict, inputs: Dict[str, List], capacity=None, plan=None, **opt
     ins = [(int(inputs[k][0].numel()) if inputs[k] else 0, inputs[k]) for k in spec["inputs"]]
     if capacity is None:
         capacity = max([n for n, _ in ins] + [1])
+    plan.out_id = ids[spec["out"]]
     cols, n = plan.run(ins, ids[spec["out"]], capacity)
     types = plan.node_schema(ids[spec["out"]])
     torch.cuda.synchronize()

@@ -20,6 +20,39 @@ def test_q1_aggregate(n, fuse):
     assert_same(got, run_oracle(spec, ins))
 
 
+@pytest.mark.parametrize("agg_mode", [0, 1])
+def test_q1_both_agg_terminals(agg_mode):
+    """agg_mode 0: auto (register one-hot terminal for Q1); 1: thread-private partials."""
+    spec = workloads.c4_spec()
+    ins = workloads.c4_inputs(300_001, device=DEV, cfg=0x93)
+    got, plan = run_gpu(spec, ins, capacity=6, agg_mode=agg_mode)
+    assert_same(got, run_oracle(spec, ins))
+    want = "partial flush every" if agg_mode == 1 else "register one-hot"
+    assert want in plan.explain(plan.out_id)
+
+
+@pytest.mark.parametrize("lo,hi", [(-1000, 1000), (-(2**40), 2**40), (-(2**63), 2**63 - 1), (5, 5)])
+@pytest.mark.parametrize("D", [1, 7, 64])
+def test_warp_agg_signed_bounds_and_many_groups(lo, hi, D):
+    """Signed sums whose declared bounds give 1, 2 and 3 27-bit chunks (value - lo),
+    and up to 64 groups (every batch of 32 rows visits many distinct groups)."""
+    import torch
+    n = 70_001
+    gen = torch.Generator().manual_seed(D * 7 + (hi & 0xff))
+    v = torch.randint(lo, hi + 1, (n,), dtype=torch.int64, generator=gen) if hi < 2**63 - 1 else \
+        torch.randint(-(2**63), 2**63 - 1, (n,), dtype=torch.int64, generator=gen)
+    v[:3] = torch.tensor([lo, hi, lo])
+    w = torch.randint(-(2**31), 2**31 - 1, (n,), dtype=torch.int64, generator=gen).to(torch.int32)
+    g = torch.randint(0, D, (n,), dtype=torch.int64, generator=gen).to(torch.uint8)
+    spec = {"inputs": {"R": {"types": ["u8", "i64", "i32"], "lo": [0, lo, -(2**31)], "hi": [D - 1, hi, 2**31 - 1]}},
+            "nodes": [{"id": "a", "op": "agg", "in": "R", "gcols": [0], "gdomain": [D],
+                       "aggs": [("sum", 1), ("count",), ("sum", 2), ("sum", 1)]}], "out": "a"}
+    ins = {"R": [g.to(DEV), v.to(DEV), w.to(DEV)]}
+    got, plan = run_gpu(spec, ins, capacity=D)
+    assert ("register one-hot" in plan.explain(plan.out_id)) == (D <= 6 and lo >= -(2**40))
+    assert_same(got, run_oracle(spec, ins))
+
+
 def test_q1_without_bounds_flushes_every_row():
     spec = workloads.c4_spec()
     spec["inputs"]["lineitem"] = {"types": workloads.Q1_TYPES}          # no declared bounds
