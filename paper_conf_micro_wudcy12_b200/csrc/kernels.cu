@@ -147,22 +147,30 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
             else hi = mid;
         }
         int r = lo - 1;
-        // (i, j) of the first candidate by division, the rest by a carry walk
-        uint64_t d = o - c_off[r];
+        // (i, j) of the first candidate by division, the rest by a carry walk: every
+        // run has >= 1 candidate, so a step that leaves run r lands on the first
+        // candidate (0, 0) of run r + 1
+        const uint64_t d = o - c_off[r];
         uint32_t lr = c_lenR[r];
-        uint32_t qi = (uint32_t)(d / lr), qj = (uint32_t)(d - (uint64_t)qi * lr);
+        uint32_t qi, qj;
+        if (d == 0) {
+            qi = qj = 0;
+        } else if (d <= 0xffffffffull) {
+            qi = (uint32_t)d / lr;
+            qj = (uint32_t)d - qi * lr;
+        } else {
+            qi = (uint32_t)(d / lr);
+            qj = (uint32_t)(d - (uint64_t)qi * lr);
+        }
 #pragma unroll
         for (int k = 0; k < ITEMS; k++) {
             ii[k] = jj[k] = 0;
             if (first + k < rows) {
                 const uint64_t oo = o + k;
                 if (r + 1 < nr && c_off[r + 1] <= oo) {
-                    while (r + 1 < nr && c_off[r + 1] <= oo)
-                        r++;
+                    r++;
                     lr = c_lenR[r];
-                    d = oo - c_off[r];
-                    qi = (uint32_t)(d / lr);
-                    qj = (uint32_t)(d - (uint64_t)qi * lr);
+                    qi = qj = 0;
                 }
                 ii[k] = c_s[r] + qi;
                 jj[k] = c_lo[r] + qj;
@@ -818,12 +826,6 @@ __global__ void k_merge_splits(const __grid_constant__ JoinRunsLaunch J)
     J.split[p] = merge_path((const K *)J.lkey, J.nl, (const K *)J.rkey, J.nr, d);
 }
 
-// Two streaming passes (no look-back on the critical path): WRITE = false counts
-// the matched runs and join candidates of every partition; k_scan_parts turns the
-// counts into exclusive offsets; WRITE = true recomputes the partition (identical
-// arithmetic) and writes the run records at their offsets.  Phase timing showed the
-// single-pass version spent a third of its samples parked behind per-partition
-// look-backs.
 // first index in [start, n) of a sorted smem array with a[idx] > key (a[start-1] <= key)
 template <typename K>
 __device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
@@ -848,17 +850,29 @@ __device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
 // the matched runs and join candidates of every partition; k_scan_parts turns the
 // counts into exclusive offsets; WRITE = true recomputes the partition (identical
 // arithmetic) and writes the run records at their offsets.
-// Inside a partition thread t walks merged positions [8t, 8t+8) (L before R on equal
-// keys, P:196 binary-search partitioning, one diagonal search per thread): an L
-// element's R lower bound is the walk's R index; the R and L run ends are found by
-// galloping in smem (runs are short except for hot keys, which gallop on into HBM).
+//
+// In the merged order (L before R on equal keys, P:196 binary-search partitioning)
+// every key forms one contiguous segment [its L rows][its R rows].  A segment HEAD is
+// a merged element whose key differs from its predecessor's; at a head the walk's
+// (L index, R index) are the key's first L row and its R lower bound, and the next
+// head's indices end both runs.  So a partition needs no per-run searches:
+//   1. each thread merges its 8 positions (one diagonal search) and records heads;
+//   2. a block scan places the heads in smem in merged order;
+//   3. head k's run lengths are head k+1's indices minus its own; only the
+//      partition's last head looks past the partition end (galloping in smem, then
+//      in HBM for hot keys whose segment spans later partitions);
+//   4. matched heads (lenL > 0 and lenR > 0) are compacted into run records.
 template <typename K, bool WRITE>
-__global__ void __launch_bounds__(kThreads, 5) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
+__global__ void __launch_bounds__(kThreads, 4) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
 {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    uint64_t *wtot = (uint64_t *)smem_raw;                        // 2 * kWarps + 2
+    uint64_t *wtot = (uint64_t *)smem_raw;                        // 2 * kWarps, then head counts
+    int32_t *hcount = (int32_t *)(wtot + 2 * kWarps);             // kWarps
     K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT + kRunExt
     K *sR = sL + kRunT + kRunExt;                                 // kRunT + kRunExt
+    int32_t *hL = (int32_t *)(sR + kRunT + kRunExt);              // kRunT heads (local L index)
+    int32_t *hR = hL + kRunT;                                     // kRunT heads (local R index)
+    K *hK = (K *)align_up((size_t)(hR + kRunT), 16);              // kRunT head keys
     const K *L = (const K *)J.lkey;
     const K *R = (const K *)J.rkey;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -876,62 +890,114 @@ __global__ void __launch_bounds__(kThreads, 5) k_join_runs(const __grid_constant
             sR[q] = R[j0 + q];
         __syncthreads();
 
-        // one walk over the thread's merged positions; `emit` writes the run records
-        // starting at (r, off) (second walk of the WRITE pass), else only counts
-        auto walk = [&](bool emit, int64_t r, uint64_t off, int &nrun, uint64_t &outs) {
-            nrun = 0;
-            outs = 0;
-            const int dt = tid * kRunItems;
-            if (dt >= m)
-                return;
+        // 1. merge walk over the thread's positions: bit q of hmask = position dt+q is a
+        //    segment head, bit q of tmask = it is an L element (so its L index is lo0 +
+        //    popc(tmask below q) and its R index the merged position minus that)
+        uint32_t hmask = 0, tmask = 0;
+        int lo0 = 0;
+        const int dt = tid * kRunItems;
+        if (dt < m) {
             int lo = dt > nR ? dt - nR : 0, hi = dt < nL ? dt : nL;
             while (lo < hi) {
                 const int mid = (lo + hi) >> 1;
                 if (sL[mid] <= sR[dt - mid - 1]) lo = mid + 1;
                 else hi = mid;
             }
+            lo0 = lo;
             int li = lo, rj = dt - lo;
-            const int end = min(dt + kRunItems, m);
-            for (int d = dt; d < end; d++) {
-                const bool takeL = rj >= nR || (li < nL && sL[li] <= sR[rj]);
-                if (!takeL) {
-                    rj++;
-                    continue;
-                }
-                const K key = sL[li];
-                const int64_t gi = i0 + li;
-                const bool start = gi == 0 || (li > 0 ? sL[li - 1] != key : L[gi - 1] != key);
-                if (start && rj < nRe && sR[rj] == key) {
-                    // R elements with key < this key precede it in the merge: lower bound = rj
-                    const int e = gallop_smem(sR, rj + 1, nRe, key);
-                    int64_t rhi = j0 + e;
-                    if (e == nRe)
-                        rhi = gallop_upper(R, rhi, J.nr, key);
-                    const int64_t rlo64 = j0 + rj;
-                    const int el = gallop_smem(sL, li + 1, nLe, key);
-                    int64_t iend = i0 + el;
-                    if (el == nLe)
-                        iend = gallop_upper(L, iend, J.nl, key);
-                    const uint64_t c = (uint64_t)(iend - gi) * (uint64_t)(rhi - rlo64);
-                    if (emit && r < J.cap_runs) {
-                        J.s[r] = (uint32_t)gi;
-                        J.lenL[r] = (uint32_t)(iend - gi);
-                        J.lo[r] = (uint32_t)rlo64;
-                        J.lenR[r] = (uint32_t)(rhi - rlo64);
-                        J.off[r] = off;
-                    }
-                    r++;
-                    off += c;
-                    outs += c;
-                    nrun++;
-                }
-                li++;
+            // predecessor of the first position in merged order: the larger of the
+            // preceding L and R elements (global ones at the partition start)
+            const bool pl_ok = (i0 + li) > 0, pr_ok = (j0 + rj) > 0;
+            bool has_prev = pl_ok || pr_ok;
+            K prev = K(0);
+            if (has_prev) {
+                const K pl = pl_ok ? (li > 0 ? sL[li - 1] : L[i0 - 1]) : K(0);
+                const K pr = pr_ok ? (rj > 0 ? sR[rj - 1] : R[j0 - 1]) : K(0);
+                prev = !pl_ok ? pr : (!pr_ok ? pl : (pl < pr ? pr : pl));
             }
-        };
-        int nrun;
-        uint64_t outs;
-        walk(false, 0, 0, nrun, outs);
-        // block exclusive scan of (runs, outputs) over threads (thread order = merge order)
+#pragma unroll
+            for (int q = 0; q < kRunItems; q++) {
+                if (dt + q < m) {
+                    const bool takeL = rj >= nR || (li < nL && sL[li] <= sR[rj]);
+                    const K key = takeL ? sL[li] : sR[rj];
+                    hmask |= (uint32_t)(!has_prev || key != prev) << q;
+                    tmask |= (uint32_t)takeL << q;
+                    has_prev = true;
+                    prev = key;
+                    li += takeL ? 1 : 0;
+                    rj += takeL ? 0 : 1;
+                }
+            }
+        }
+        const int nh = __popc(hmask);
+        // 2. heads in merged order into smem
+        int hinc = nh;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, hinc, o);
+            if (lane >= o) hinc += y;
+        }
+        if (lane == 31)
+            hcount[warp] = hinc;
+        __syncthreads();
+        int hbase = 0, H = 0;
+        for (int w = 0; w < kWarps; w++) {
+            if (w < warp) hbase += hcount[w];
+            H += hcount[w];
+        }
+        hbase += hinc - nh;
+        for (uint32_t hm = hmask; hm; hm &= hm - 1) {
+            const int q = __ffs(hm) - 1;
+            const int li = lo0 + __popc(tmask & ((1u << q) - 1u));
+            const int rj = dt + q - li;
+            hL[hbase] = li;
+            hR[hbase] = rj;
+            hK[hbase] = ((tmask >> q) & 1u) ? sL[li] : sR[rj];
+            hbase++;
+        }
+        __syncthreads();
+        // 3. run lengths; the last head's segment may continue past the partition
+        const int k0 = tid * kRunItems;
+        int64_t tailL = 0, tailR = 0;
+        if (k0 < H && k0 + kRunItems >= H) {
+            const K key = hK[H - 1];
+            int e = nL;
+            if (nL < nLe && sL[nL] == key)
+                e = gallop_smem(sL, nL + 1, nLe, key);
+            tailL = i0 + e;
+            if (e == nLe && i0 + e < J.nl && L[i0 + e] == key)
+                tailL = gallop_upper(L, i0 + e, J.nl, key);
+            int f = nR;
+            if (nR < nRe && sR[nR] == key)
+                f = gallop_smem(sR, nR + 1, nRe, key);
+            tailR = j0 + f;
+            if (f == nRe && j0 + f < J.nr && R[j0 + f] == key)
+                tailR = gallop_upper(R, j0 + f, J.nr, key);
+        }
+        int nrun = 0;
+        uint64_t outs = 0;
+        uint32_t matched = 0;
+        uint64_t cnt[kRunItems];
+        int64_t lenl[kRunItems], lenr[kRunItems];
+#pragma unroll
+        for (int q = 0; q < kRunItems; q++) {
+            const int k = k0 + q;
+            cnt[q] = 0;
+            lenl[q] = lenr[q] = 0;
+            if (k < H) {
+                const int64_t nl_ = k + 1 < H ? i0 + hL[k + 1] : tailL;
+                const int64_t nr_ = k + 1 < H ? j0 + hR[k + 1] : tailR;
+                lenl[q] = nl_ - (i0 + hL[k]);
+                lenr[q] = nr_ - (j0 + hR[k]);
+                if (lenl[q] > 0 && lenr[q] > 0) {
+                    matched |= 1u << q;
+                    cnt[q] = (uint64_t)lenl[q] * (uint64_t)lenr[q];
+                    nrun++;
+                    outs += cnt[q];
+                }
+            }
+        }
+        // 4. block exclusive scan of (runs, outputs) over threads (thread order = merge order)
         uint64_t ir = (uint64_t)nrun, io = outs;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -964,9 +1030,23 @@ __global__ void __launch_bounds__(kThreads, 5) k_join_runs(const __grid_constant
             }
             continue;
         }
-        int nr2;
-        uint64_t o2;
-        walk(true, (int64_t)J.pruns[p] + (int64_t)br, J.pouts[p] + bo, nr2, o2);
+        int64_t r = (int64_t)J.pruns[p] + (int64_t)br;
+        uint64_t off = J.pouts[p] + bo;
+#pragma unroll
+        for (int q = 0; q < kRunItems; q++) {
+            if ((matched >> q) & 1u) {
+                const int k = k0 + q;
+                if (r < J.cap_runs) {
+                    J.s[r] = (uint32_t)(i0 + hL[k]);
+                    J.lenL[r] = (uint32_t)lenl[q];
+                    J.lo[r] = (uint32_t)(j0 + hR[k]);
+                    J.lenR[r] = (uint32_t)lenr[q];
+                    J.off[r] = off;
+                }
+                r++;
+                off += cnt[q];
+            }
+        }
     }
 }
 
@@ -1055,7 +1135,9 @@ int join_expand_tile() { return kThreads * kJoinItems; }
 
 size_t join_runs_smem(int key_type)
 {
-    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)(kRunT + kRunExt) * type_width(key_type);
+    const size_t w = type_width(key_type);
+    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)(kRunT + kRunExt) * w + 2 * (size_t)kRunT * 4 +
+           16 + (size_t)kRunT * w;
 }
 
 template <typename F>

@@ -956,7 +956,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         size_t W = 0;
         for (int c = 0; c < P.nout; c++)
             W += (((size_t)L.tile * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
-        L.gring_bytes = (uint32_t)std::max<size_t>(128 * 1024, 4 * W);
+        L.gring_bytes = (uint32_t)std::max<size_t>(want_ring ? want_ring : 128 * 1024, 4 * W);
         L.out_bytes = L.gring_bytes;
     }
 }
