@@ -98,16 +98,27 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
     const uint32_t m = (int64_t)total < lim ? total : (lim > 0 ? (uint32_t)lim : 0u);
     T *d = dst + base;
     uint32_t j = q;
-    for (; j + 3 * nq < m; j += 4 * nq) {
-        const T a = ld_ring(src + j, gring), b = ld_ring(src + j + nq, gring), c = ld_ring(src + j + 2 * nq, gring),
-                e = ld_ring(src + j + 3 * nq, gring);
-        d[j] = a;
-        d[j + nq] = b;
-        d[j + 2 * nq] = c;
-        d[j + 3 * nq] = e;
+    // several loads in flight per lane: the ring is read from L2 (~0.5 us per round
+    // trip); phase timestamps showed a writer warp needing 6.4 us per compacted C2 tile
+    constexpr int U = sizeof(T) >= 8 ? 4 : 8;
+    for (; j + (U - 1) * nq < m; j += U * nq) {
+        T v[U];
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            v[u] = ld_ring(src + j + u * nq, gring);
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            d[j + u * nq] = v[u];
     }
-    for (; j < m; j += nq)
-        d[j] = ld_ring(src + j, gring);
+    if (j < m) {
+        T v[U];
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            if (j + u * nq < m) v[u] = ld_ring(src + j + u * nq, gring);
+#pragma unroll
+        for (int u = 0; u < U; u++)
+            if (j + u * nq < m) d[j + u * nq] = v[u];
+    }
 }
 
 // Join expansion into a tile (§8(a) a8): candidates [t*T, t*T + rows) of the
@@ -267,11 +278,11 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
             uint32_t eph = 1;                                // parity of the previous use
             for (int64_t i = 0;; ++i) {
                 if (i >= S)
-                    mbar_wait_sleep(&ctl->in[s].empty, eph);
+                    mbar_wait_sleep(&ctl->in[s].empty, eph, 64);
                 const int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
-                    L.dbg_ts[8 * t + 0] = globaltimer();
+                    L.dbg_ts[10 * t + 0] = globaltimer();
                 if (!JOIN && t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
                     char *st = stages + (size_t)s * P.stage_bytes;
                     fence_proxy_async_smem();
@@ -300,18 +311,18 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
         if (emit) {
             for (int64_t i = wi;; i += kWriterWarps) {
                 const int j = (int)(i % kRingSlots);
-                mbar_wait_sleep(&ctl->blk[j].aggr, (uint32_t)((i / kRingSlots) & 1));
+                mbar_wait_sleep(&ctl->blk[j].aggr, (uint32_t)((i / kRingSlots) & 1), 256);
                 const int64_t t = ctl->blk[j].tile;
                 if (t >= ntiles)
                     break;
                 const uint32_t total = ctl->blk[j].total;
                 if ((L.dbg & 4) && lane == 0)
-                    L.dbg_ts[8 * t + 5] = globaltimer();
+                    L.dbg_ts[10 * t + 5] = globaltimer();
                 const int64_t excl = (L.dbg & 1) ? t * T
                                                   : (int64_t)lookback_warp(L.status, t, total, L.epoch, /*aggregate_published=*/true);
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[8 * t + 3] = globaltimer();
+                        L.dbg_ts[10 * t + 3] = globaltimer();
                     if (t == ntiles - 1)
                         *L.n_dev = excl + (int64_t)total;
                 }
@@ -339,9 +350,9 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 }
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[8 * t + 4] = globaltimer();
+                        L.dbg_ts[10 * t + 4] = globaltimer();
                     if (i > 0)   // release ring bytes in tile order
-                        mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1));
+                        mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1), 64);
                     // the discards must land in L2 before the bytes can be rewritten
                     if (gring && !(L.dbg & 8))
                         __threadfence();
@@ -398,7 +409,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
             const int64_t row0 = t * T;
             const int rows = (int)min((int64_t)T, n - row0);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[8 * t + 1] = globaltimer();
+                L.dbg_ts[10 * t + 1] = globaltimer();
             auto release_stage = [&]() {
                 __syncwarp();
                 if (lane == 0)
@@ -438,7 +449,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
             }
             mask = run_ops<NT, ITEMS>(P, st, scratch, mask);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[8 * t + 6] = globaltimer();
+                L.dbg_ts[10 * t + 6] = globaltimer();
             if (AGG) {
                 if (P.agg_mode == 2)
                     agg_tile_reg<NT, ITEMS>(P, st, scratch, mask, racc, cta_acc, since_flush, L.err);
@@ -447,7 +458,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 else
                     agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
                 if ((L.dbg & 4) && tid == 0)
-                    L.dbg_ts[8 * t + 2] = globaltimer();
+                    L.dbg_ts[10 * t + 2] = globaltimer();
                 release_stage();
                 continue;
             }
@@ -488,7 +499,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
             }
             bar_sync(kComputeBar, NT);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[8 * t + 7] = globaltimer();
+                L.dbg_ts[10 * t + 7] = globaltimer();
             // every warp scans the ITEMS x NW survivor counts itself
             uint32_t pre[ITEMS];
             uint32_t total;
@@ -528,13 +539,15 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 if (t > 0 && !(L.dbg & 1))
                     st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
                 if (L.dbg & 4)
-                    L.dbg_ts[8 * t + 2] = globaltimer();
+                    L.dbg_ts[10 * t + 2] = globaltimer();
             }
             // ring bytes for the compacted tile (blocks never wrap); every warp computes
             // the same reservation from the same (head, hpos, total)
             uint32_t need = 0;
             for (int c = 0; c < P.nout; c++)
                 need += al16(total * P.out_w[c]);
+            if ((L.dbg & 4) && tid == 0)
+                L.dbg_ts[10 * t + 9] = globaltimer();
             uint32_t pos = hpos;
             uint32_t used = need;
             bool drain = false;
@@ -599,6 +612,8 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 }
                 mbar_arrive(&ctl->in[s].empty);          // this warp is done with the stage
                 mbar_arrive(&ctl->blk[j].aggr);          // and with the ring block
+                if ((L.dbg & 4) && warp == 0)
+                    L.dbg_ts[10 * t + 8] = globaltimer();
             }
         }
     }
@@ -863,7 +878,7 @@ __device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
 //      in HBM for hot keys whose segment spans later partitions);
 //   4. matched heads (lenL > 0 and lenR > 0) are compacted into run records.
 template <typename K, bool WRITE>
-__global__ void __launch_bounds__(kThreads, 4) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
+__global__ void __launch_bounds__(kThreads, 3) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
 {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     uint64_t *wtot = (uint64_t *)smem_raw;                        // 2 * kWarps, then head counts
@@ -878,17 +893,39 @@ __global__ void __launch_bounds__(kThreads, 4) k_join_runs(const __grid_constant
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t ntot = J.nl + J.nr;
 
+    // software pipeline: the keys of the CTA's next partition are loaded into
+    // registers while the current one is processed
+    constexpr int PF = (kRunT + kRunExt + kThreads - 1) / kThreads;
+    K pfL[PF], pfR[PF];
+    auto fetch = [&](int64_t pp) {
+        const int64_t a0 = J.split[pp], a1 = J.split[pp + 1];
+        const int64_t e0 = min(pp * kRunT, ntot);
+        const int64_t b0 = e0 - a0, b1 = min(e0 + kRunT, ntot) - a1;
+        const int nle = (int)(min(a1 + kRunExt, J.nl) - a0), nre = (int)(min(b1 + kRunExt, J.nr) - b0);
+#pragma unroll
+        for (int q = 0; q < PF; q++) {
+            const int idx = tid + q * kThreads;
+            pfL[q] = idx < nle ? L[a0 + idx] : K(0);
+            pfR[q] = idx < nre ? R[b0 + idx] : K(0);
+        }
+    };
+    if ((int64_t)blockIdx.x < J.nparts)
+        fetch(blockIdx.x);
     for (int64_t p = blockIdx.x; p < J.nparts; p += gridDim.x) {
         const int64_t d0 = p * kRunT, d1 = min(d0 + kRunT, ntot);
         const int64_t i0 = J.split[p], i1 = J.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
         const int nL = (int)(i1 - i0), nR = (int)(j1 - j0), m = (int)(d1 - d0);
         const int nLe = (int)(min(i1 + kRunExt, J.nl) - i0), nRe = (int)(min(j1 + kRunExt, J.nr) - j0);
         __syncthreads();
-        for (int q = tid; q < nLe; q += kThreads)
-            sL[q] = L[i0 + q];
-        for (int q = tid; q < nRe; q += kThreads)
-            sR[q] = R[j0 + q];
+#pragma unroll
+        for (int q = 0; q < PF; q++) {
+            const int idx = tid + q * kThreads;
+            if (idx < nLe) sL[idx] = pfL[q];
+            if (idx < nRe) sR[idx] = pfR[q];
+        }
         __syncthreads();
+        if (p + gridDim.x < J.nparts)
+            fetch(p + gridDim.x);
 
         // 1. merge walk over the thread's positions: bit q of hmask = position dt+q is a
         //    segment head, bit q of tmask = it is an L element (so its L index is lo0 +

@@ -76,7 +76,7 @@ __device__ __forceinline__ bool mbar_try(uint64_t *bar, uint32_t parity)
     asm volatile(
         "{\n"
         ".reg .pred p;\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
         "selp.u32 %0, 1, 0, p;\n"
         "}\n"
         : "=r"(ok)
@@ -85,14 +85,15 @@ __device__ __forceinline__ bool mbar_try(uint64_t *bar, uint32_t parity)
     return ok != 0;
 }
 
-// wait with exponential nanosleep backoff: for warps off the critical path
-// (producer, writers) so their polling does not steal issue slots
-// (try_wait with a suspend-time hint parks the warp in hardware until the phase
-// flips; measured: a nanosleep poll loop woke every ~40 cycles and issued ~10-20 % of
-// all instructions of the scan and join kernels)
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity)
+// Poll with a fixed nanosleep between non-suspending tests: for warps off the
+// critical path (producer, writers).  Measured on B200: try_wait's suspend
+// (NANOSLEEP.SYNCS) wakes on every mbarrier event of the CTA, so a warp parked in it
+// re-polls after each tile event (~25 % of all issued instructions of the join
+// expansion); __nanosleep(ns) sleeps ~ns (1000 ns -> 2010 cycles at 1.965 GHz).
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity, uint32_t ns)
 {
-    mbar_wait(bar, parity);
+    while (!mbar_try(bar, parity))
+        __nanosleep(ns);
 }
 
 // 1-D bulk copy global -> shared, completion signalled on `bar` (complete_tx).

@@ -16,7 +16,7 @@ def main(stages, ctas, ring, extra=0, cfg="c2"):
         ins = workloads.c2_inputs(rows, 0, "cuda:0")
     T = 1024 if cfg == "c4" else 2048
     nt = (rows + T - 1) // T
-    ts = torch.zeros(nt * 8, dtype=torch.int64, device="cuda:0")
+    ts = torch.zeros(nt * 10, dtype=torch.int64, device="cuda:0")
     plan, ids = build_gpu_plan(spec, stages=stages, ctas_per_sm=ctas, defer=ring, dbg=4 | extra, dbg_ts=ts.data_ptr())
     out_node = ids[spec["out"]]
     types = plan.node_schema(out_node)
@@ -29,10 +29,10 @@ def main(stages, ctas, ring, extra=0, cfg="c2"):
     for _ in range(3):
         plan.execute([(rows, ins[name])], out_node, outs, cap, n_dev=nd)
     torch.cuda.synchronize()
-    a = ts.view(nt, 8).double()
+    a = ts.view(nt, 10).double()
     t0 = a[:, 0].min()
     d = {"load(claim->data)": a[:, 1] - a[:, 0], "ops(data->ops)": a[:, 6] - a[:, 1], "ballot(ops->bar1)": a[:, 7] - a[:, 6], "scan(bar1->agg)": a[:, 2] - a[:, 7],
-         "writer queue(agg->wstart)": a[:, 5] - a[:, 2], "lookback(wstart->offset)": a[:, 3] - a[:, 5], "store(offset->stored)": a[:, 4] - a[:, 3],
+         "reserve(agg->reserved)": a[:, 9] - a[:, 2], "ring wait+scatter(->arrived)": a[:, 8] - a[:, 9], "writer queue(arrived->wstart)": a[:, 5] - a[:, 8], "lookback(wstart->offset)": a[:, 3] - a[:, 5], "store(offset->stored)": a[:, 4] - a[:, 3],
          "total(claim->stored)": a[:, 4] - a[:, 0]}
     if cfg == "c4":
         a[:, 3] = a[:, 2]; a[:, 4] = a[:, 2]; a[:, 5] = a[:, 2]; a[:, 7] = a[:, 6]
