@@ -34,6 +34,7 @@ CONFIGS = {
     "c2": dict(name="C2: SELECT->PROJECT->SELECT over 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
     "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
+    "cd": dict(name="Pattern (d) input dependence: 2 SELECTs (25% each) sharing one input of 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
     "c5": dict(name="C5: JOIN->JOIN->SELECT over three relations, 2^27 rows each per GPU (2^30 at 8 GPUs), key-range sharded", rows=1 << 27),
 }
 
@@ -45,6 +46,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="rw", choices=["rw", "reference"])
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--branches", type=int, default=2, help="cd: SELECTs sharing the input (2..4)")
     ap.add_argument("--rows", type=int, default=0, help="override rows per GPU (testing)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-unfused", action="store_true")
@@ -76,10 +78,15 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
         return workloads.c3_spec(), workloads.c3_inputs(rows, device=device)
     if cfg == "c4":
         return workloads.c4_spec(), workloads.c4_inputs(rows, start, device)
+    if cfg == "cd":
+        return workloads.cd_spec(0.25, BRANCHES), workloads.cd_inputs(rows, start, device)
     if cfg == "c5":
         world = int(os.environ.get("WORLD_SIZE", "1"))
         return workloads.c5_spec(), workloads.c5_inputs(rows, key_space=rows * world, start=start, device=device)
     raise ValueError(cfg)
+
+
+BRANCHES = 2
 
 
 def spec_rows(spec, ins):
@@ -184,7 +191,7 @@ def run_reference(args):
         return 0
     cfg = args.config
     rows = args.rows or CONFIGS[cfg]["rows"]
-    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21}[cfg]
+    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24}[cfg]
     import oracle
     oracle.build()
     vals = []
@@ -209,6 +216,8 @@ def run_reference(args):
 
 def main():
     args = parse()
+    global BRANCHES
+    BRANCHES = args.branches
     if args.impl == "reference":
         return run_reference(args)
     import torch
@@ -236,6 +245,12 @@ def main():
     def make(fuse):
         plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse, stages=args.stages,
                                    ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg, items=args.items, variant=args.variant, gring=args.gring)
+        if "outs" in spec:
+            # input-dependence fusion: one output relation per branch
+            cap = max(nrows.values())
+            out_types = [plan.node_schema(ids[o]) for o in spec["outs"]]
+            outs = [[torch.empty(cap, dtype=dtn[t], device=dev) for t in ts] for ts in out_types]
+            return plan, ids, outs, cap, out_types
         out_types = plan.node_schema(ids[spec["out"]])
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
         if cfg == "c3":
@@ -249,8 +264,17 @@ def main():
     n_dev = torch.zeros(1, dtype=torch.int64, device=dev)
     from paper_conf_micro_wudcy12_b200 import dist as rdist
 
+    n_devs = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in spec.get("outs", [])]
+
     def make_step(plan, ids, outs, cap):
         node = ids[spec["out"]]
+        if "outs" in spec:
+            nodes = [ids[o] for o in spec["outs"]]
+
+            def step():
+                plan.execute_multi(inputs, nodes, outs, [cap] * len(nodes), n_devs=n_devs)
+                return plan.last_launches()
+            return step
         if cfg == "c4" and world > 1:
             # local fused Q1, exact limb export, one NCCL all-reduce, import
             limbs = torch.empty(plan.agg_limbs(node), dtype=torch.int64, device=dev)
@@ -313,15 +337,20 @@ def main():
 
     plan, ids, outs, cap, out_types = make(True)
     total_ms, per, launches, clocks = timed(make_step(plan, ids, outs, cap), args.steps, args.warmup)
-    n_out = int(n_dev.item())
+    if "outs" in spec:
+        n_outs = [int(x.item()) for x in n_devs]
+        n_out = sum(n_outs)
+        out_bytes = sum(nk * sum(W[t] for t in ts) for nk, ts in zip(n_outs, out_types))
+    else:
+        n_out = int(n_dev.item())
+        out_bytes = n_out * sum(W[t] for t in out_types)
     ms_step = total_ms / args.steps
     value = n_in * world / (total_ms / 1e3 / args.steps)
 
     # roofline of the dominant kernel.  C1/C2: the fused k_scan_chain is the whole step;
     # C4: k_scan_chain<agg> (k_agg_finalize is a 1-CTA epilogue of a few us); C3/C5: the
     # join pair (k_join_runs + k_join_expand), algorithmic bytes = inputs + output.
-    out_w = sum(W[t] for t in out_types)
-    alg_bytes = in_bytes + n_out * out_w
+    alg_bytes = in_bytes + out_bytes
     peak, peak_src = measured_peak()
     kern_ms = statistics.mean(per)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
@@ -343,7 +372,7 @@ def main():
                        "fused": True},
             "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
 
-    if not args.no_unfused and cfg in ("c1", "c2", "c4", "c3"):
+    if not args.no_unfused and cfg in ("c1", "c2", "c4", "c3", "cd"):
         del outs
         torch.cuda.empty_cache()
         uplan, uids, uouts, ucap, _ = make(False)
@@ -386,7 +415,7 @@ def main():
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:
-        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22}[cfg]
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26}[cfg]
         v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
         line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
                                 "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}

@@ -172,6 +172,20 @@ rw_status rw_plan_node_schema(const rw_plan *plan, int32_t node, int32_t *ncols,
 rw_status rw_plan_execute(rw_plan *plan, const rw_relation_in *in, int32_t nin, int32_t out_node,
                           rw_relation_out *out);
 
+/* Input-dependence fusion (§4.4 "operators shares the same inputs ... the input
+ * data shared by different operators only need to be loaded once"; Fig. 14(d)):
+ * execute nout output nodes at once.  outs[k] receives out_nodes[k] exactly as
+ * rw_plan_execute would (same layout, capacity and n / n_dev rules, same row order).
+ * When the plan is fused, 2 <= nout <= 4, and every out_nodes[k] is reached from one
+ * common INPUT relation through SELECT / PROJECT nodes only, all branches run in ONE
+ * k_scan_chain pass: each tile is loaded once and every branch evaluates, compacts and
+ * stores its own output.  Otherwise (fuse = 0, other shapes) the nodes run one after
+ * the other, each as rw_plan_execute.  A shared SELECT/PROJECT prefix of several
+ * branches is re-evaluated per branch (thread-dependent work, no extra bytes).
+ * Errors as rw_plan_execute; RW_E_CAPACITY names the first output that overflowed. */
+rw_status rw_plan_execute_multi(rw_plan *plan, const rw_relation_in *in, int32_t nin, const int32_t *out_nodes,
+                                int32_t nout, rw_relation_out *outs);
+
 /* Same, with HOST buffers: inputs are copied host->device, the plan runs, the result
  * (up to capacity rows) is copied device->host, the stream is synchronised and out->n
  * set.  Pinned (cudaHostAlloc / registered) buffers give full PCIe bandwidth. */

@@ -289,10 +289,11 @@ __device__ __noinline__ void run_expr(uint32_t code, int ta, int tb, int64_t k, 
 // Run the fused program over one tile (§4.3.1: SELECT / PROJECT in order,
 // in the same thread, no synchronisation between thread-dependent operators).
 template <int NT, int ITEMS>
-__device__ __forceinline__ uint32_t run_ops(const ChainProg &P, const char *stage, char *scratch, uint32_t mask)
+__device__ __forceinline__ uint32_t run_ops(const ChainProg &P, int op0, int op1, const char *stage, char *scratch,
+                                            uint32_t mask)
 {
 #pragma unroll 1
-    for (int i = 0; i < P.nops; i++) {
+    for (int i = op0; i < op1; i++) {
         // fields are read once from the constant bank and passed by value (a reference
         // into kernel-parameter space would turn every field access into a generic load)
         const uint32_t kind = P.ops[i].kind, code = P.ops[i].code;

@@ -29,6 +29,7 @@ constexpr int kScanItems = 8;        // rows per thread per tile in the scan ker
 constexpr int kJoinItems = 9;        // outputs per thread per tile in the join expansion (T = 2304,
                                      // odd stride -> conflict-free thread-contiguous smem writes)
 constexpr int kMaxAggSlots = 4096;
+constexpr int kMaxBranch = 4;        // input-dependence fusion: SELECT/PROJECT chains sharing one scan
 constexpr int kRegD = 6;             // register aggregate terminal: groups x sums held per thread
 constexpr int kRegA = 5;   // D * (nagg + 1) upper bound for the agg terminal
 
@@ -89,6 +90,13 @@ struct ChainProg {
     uint8_t agg_unsigned[kMaxAggs];     // 1: u64 sum (unsigned partials)
     int64_t flush_rows;                 // rows a thread may add before its int64 partials can overflow
     int32_t agg_mode;                   // 0: thread-private partials in smem; 2: register one-hot (D <= kRegD, nagg <= kRegA)
+    // input-dependence fusion (§4.4, Fig. 14(d)): nbranch chains over the same
+    // staged tile, each with its own mask and compacted output.  Branch b runs ops
+    // [br_op_end[b-1], br_op_end[b]) and writes output columns [br_out_end[b-1], br_out_end[b]).
+    int32_t nbranch;                    // >= 1
+    uint8_t br_op_end[kMaxBranch];
+    uint8_t br_out_end[kMaxBranch];
+    int64_t br_cap[kMaxBranch];         // output capacity of branch b (b = 0: out_capacity)
     uint32_t stage_bytes;               // bytes of one stage (all input slots, aligned)
     uint32_t scratch_bytes;             // bytes of scratch (computed slots)
 };
@@ -103,7 +111,9 @@ struct TileLaunch {
     int32_t direct;            // scan kernel: no SELECT in the group, rows stored at their offsets
     int32_t use_tma;           // input slots may be bulk-copied (16B-aligned bases)
     uint32_t epoch;            // look-back epoch tag (1..65535)
-    uint64_t *status;          // look-back status words, >= ntiles
+    uint64_t *status;          // look-back status words, >= ntiles (per branch: + b * status_stride)
+    int64_t status_stride;
+    int64_t *br_n_dev[kMaxBranch];   // output row count of branch b >= 1 (branch 0: n_dev)
     uint32_t *ctrs;            // [0] tile counter, [1] done counter (reset by the last CTA)
     int64_t *n_dev;            // output row count
     unsigned long long *agg_acc;   // global 128-bit accumulators: D * (nagg+1) * 2 u64

@@ -55,6 +55,8 @@ __device__ inline void cta_exit_reset(uint32_t *ctrs)
 // ===========================================================================
 constexpr int kWriterWarps = 4;
 constexpr int kAuxThreads = 32 * (kWriterWarps + 1);      // writer warps + producer warp
+// aggregate kernels have no compacted output: no writer warps, only the producer
+__host__ __device__ constexpr int aux_threads(bool agg) { return agg ? 32 : kAuxThreads; }
 constexpr int kRingSlots = 16;          // compacted tiles awaiting their offset, per CTA
 constexpr uint32_t kComputeBar = 1;     // named barrier of the compute warps
 
@@ -68,7 +70,7 @@ struct BlkCtl {
     uint32_t total;
     uint32_t roff;                       // byte offset of the block in the ring
     uint32_t used;                       // ring bytes consumed (block + skipped tail)
-    uint32_t pad;
+    uint32_t br;                         // branch of the block (input-dependence fusion)
 };
 template <int NT, int ITEMS>
 struct ScanCtl {
@@ -214,7 +216,7 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
 }
 
 template <int NT, int ITEMS, bool AGG, bool JOIN>
-__global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(const __grid_constant__ ChainProg P,
+__global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_chain(const __grid_constant__ ChainProg P,
                                                                      const __grid_constant__ TileLaunch L,
                                                                      const __grid_constant__ JoinExpand X)
 {
@@ -244,6 +246,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
     const bool emit = !AGG && !(L.dbg & 2) && !L.direct;
+    const int NB = (AGG || JOIN) ? 1 : P.nbranch;   // input-dependence branches (host: 1 for agg / direct)
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) {
@@ -267,7 +270,8 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
     }
     __syncthreads();
 
-    if (warp == NW + kWriterWarps) {
+    constexpr int WW = AGG ? 0 : kWriterWarps;   // writer warps of this instance
+    if (warp == NW + WW) {
         // ---------------- producer warp ----------------
         if (lane == 0) {
             uint32_t tx_bytes = 0;
@@ -316,26 +320,29 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 if (t >= ntiles)
                     break;
                 const uint32_t total = ctl->blk[j].total;
+                const int b = (int)ctl->blk[j].br;
                 if ((L.dbg & 4) && lane == 0)
                     L.dbg_ts[10 * t + 5] = globaltimer();
                 const int64_t excl = (L.dbg & 1) ? t * T
-                                                  : (int64_t)lookback_warp(L.status, t, total, L.epoch, /*aggregate_published=*/true);
+                                                  : (int64_t)lookback_warp(L.status + b * L.status_stride, t, total, L.epoch,
+                                                                           /*aggregate_published=*/true);
                 if (lane == 0) {
                     if (L.dbg & 4)
                         L.dbg_ts[10 * t + 3] = globaltimer();
                     if (t == ntiles - 1)
-                        *L.n_dev = excl + (int64_t)total;
+                        *(b ? L.br_n_dev[b] : L.n_dev) = excl + (int64_t)total;
                 }
                 const char *blk = ring + ctl->blk[j].roff;
+                const int64_t cap = b ? P.br_cap[b] : P.out_capacity;
                 uint32_t coff = 0;
-                for (int c = 0; c < P.nout; c++) {
+                for (int c = b ? P.br_out_end[b - 1] : 0; c < (NB > 1 ? (int)P.br_out_end[b] : P.nout); c++) {
                     const int w = P.out_w[c];
                     const char *src = blk + coff;
                     coff += al16(total * w);
                     switch (w) {
-                    case 1: group_copy_out<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
-                    case 4: group_copy_out<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
-                    default: group_copy_out<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, P.out_capacity, lane, 32, gring); break;
+                    case 1: group_copy_out<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, cap, lane, 32, gring); break;
+                    case 4: group_copy_out<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, cap, lane, 32, gring); break;
+                    default: group_copy_out<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, cap, lane, 32, gring); break;
                     }
                 }
                 __syncwarp();
@@ -378,6 +385,7 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
         int s = 0;
         uint32_t fph = 0;
         uint32_t head = 0, hpos = 0;
+        int64_t ublk = 0;                                 // compacted blocks emitted (tiles x branches)
         for (int64_t i = 0;; ++i) {
             if (i > 0 && ++s == S) {
                 s = 0;
@@ -385,11 +393,10 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
             }
             mbar_wait(&ctl->in[s].full, fph);
             const int64_t t = ctl->in[s].tile;
-            const int j = (int)(i % kRingSlots);
             if (t >= ntiles) {
                 if (emit && tid == 0) {
                     // one sentinel per writer warp (consecutive slots)
-                    for (int64_t u = i; u < i + kWriterWarps; ++u) {
+                    for (int64_t u = ublk; u < ublk + kWriterWarps; ++u) {
                         const int ju = (int)(u % kRingSlots);
                         if (u >= kRingSlots)
                             mbar_wait(&ctl->blk[ju].oempty, (uint32_t)(((u / kRingSlots) - 1) & 1));
@@ -439,15 +446,15 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                     }
                 }
             }
-            uint32_t mask = (1u << ITEMS) - 1u;
+            uint32_t mask0 = (1u << ITEMS) - 1u;
             if (rows < T) {
-                mask = 0;
+                mask0 = 0;
 #pragma unroll
                 for (int k = 0; k < ITEMS; k++)
                     if (k * NT + tid < rows)
-                        mask |= 1u << k;
+                        mask0 |= 1u << k;
             }
-            mask = run_ops<NT, ITEMS>(P, st, scratch, mask);
+            uint32_t mask = run_ops<NT, ITEMS>(P, 0, NB > 1 ? (int)P.br_op_end[0] : P.nops, st, scratch, mask0);
             if ((L.dbg & 4) && tid == 0)
                 L.dbg_ts[10 * t + 6] = globaltimer();
             if (AGG) {
@@ -489,131 +496,143 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
                 release_stage();
                 continue;
             }
-            uint32_t *cnt = ctl->cnt[i & 1];
-            uint32_t bal[ITEMS];
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
-                if (lane == 0)
-                    cnt[k * NW + warp] = __popc(bal[k]);
-            }
-            bar_sync(kComputeBar, NT);
-            if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[10 * t + 7] = globaltimer();
-            // every warp scans the ITEMS x NW survivor counts itself
-            uint32_t pre[ITEMS];
-            uint32_t total;
-            {
-                constexpr int NV = ITEMS * NW;
-                constexpr int PER = (NV + 31) / 32;
-                uint32_t v[PER];
-                uint32_t sum = 0;
-#pragma unroll
-                for (int qq = 0; qq < PER; qq++) {
-                    const int idx = lane * PER + qq;
-                    v[qq] = idx < NV ? cnt[idx] : 0;
-                    sum += v[qq];
-                }
-                uint32_t inc = sum;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-                    if (lane >= o)
-                        inc += y;
-                }
-                total = __shfl_sync(0xffffffffu, inc, 31);
-                const uint32_t base = inc - sum;
+            // one compacted block per branch (input-dependence fusion, §4.4): the
+            // branches share the staged tile and differ in their ops, mask and outputs
+            for (int b = 0;; ) {
+                const int j = (int)(ublk % kRingSlots);
+                uint32_t *cnt = ctl->cnt[ublk & 1];
+                uint32_t bal[ITEMS];
 #pragma unroll
                 for (int k = 0; k < ITEMS; k++) {
-                    const int idx = k * NW + warp;
-                    const int owner = idx / PER, off = idx % PER;
-                    uint32_t part_sum = 0;
-#pragma unroll
-                    for (int qq = 0; qq < PER; qq++)
-                        if (qq < off) part_sum += v[qq];
-                    pre[k] = __shfl_sync(0xffffffffu, base + part_sum, owner);
+                    bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
+                    if (lane == 0)
+                        cnt[k * NW + warp] = __popc(bal[k]);
                 }
-            }
-            if (warp == 0 && lane == 31) {
-                // publish the tile aggregate before anything can block this CTA
-                if (t > 0 && !(L.dbg & 1))
-                    st_relaxed_u64(&L.status[t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
-                if (L.dbg & 4)
-                    L.dbg_ts[10 * t + 2] = globaltimer();
-            }
-            // ring bytes for the compacted tile (blocks never wrap); every warp computes
-            // the same reservation from the same (head, hpos, total)
-            uint32_t need = 0;
-            for (int c = 0; c < P.nout; c++)
-                need += al16(total * P.out_w[c]);
-            if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[10 * t + 9] = globaltimer();
-            uint32_t pos = hpos;
-            uint32_t used = need;
-            bool drain = false;
-            if (pos + need > R) {           // skip the tail [pos, R)
-                used += R - pos;
-                pos = 0;
-                if (used > R) {             // cannot fit behind live blocks: wait for an empty ring
-                    used = need;
-                    drain = true;
-                }
-            }
-            if (i >= kRingSlots)
-                mbar_wait(&ctl->blk[j].oempty, (uint32_t)(((i / kRingSlots) - 1) & 1));
-            {
-                uint32_t backoff = 32;
-                while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
-                    __nanosleep(backoff);
-                    backoff = backoff < 512 ? backoff * 2 : 512;
-                }
-            }
-            head += used;
-            hpos = pos + need == R ? 0 : pos + need;
-            char *blk = ring + pos;
-            const uint32_t lt = lanemask_lt();
-            uint32_t posk[ITEMS];
+                bar_sync(kComputeBar, NT);
+                if ((L.dbg & 4) && tid == 0)
+                    L.dbg_ts[10 * t + 7] = globaltimer();
+                // every warp scans the ITEMS x NW survivor counts itself
+                uint32_t pre[ITEMS];
+                uint32_t total;
+                {
+                    constexpr int NV = ITEMS * NW;
+                    constexpr int PER = (NV + 31) / 32;
+                    uint32_t v[PER];
+                    uint32_t sum = 0;
 #pragma unroll
-            for (int k = 0; k < ITEMS; k++)
-                posk[k] = pre[k] + __popc(bal[k] & lt);
-            uint32_t coff = 0;
-            for (int c = 0; c < P.nout; c++) {
-                const int w = P.out_w[c];
-                const char *src = loc_ptr(P.out_loc[c], st, scratch);
-                char *dst = blk + coff;
-                coff += al16(total * w);
-                switch (w) {
-                case 1:
+                    for (int qq = 0; qq < PER; qq++) {
+                        const int idx = lane * PER + qq;
+                        v[qq] = idx < NV ? cnt[idx] : 0;
+                        sum += v[qq];
+                    }
+                    uint32_t inc = sum;
 #pragma unroll
-                    for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint8_t *)dst)[posk[k]] = ((const uint8_t *)src)[k * NT + tid];
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+                        if (lane >= o)
+                            inc += y;
+                    }
+                    total = __shfl_sync(0xffffffffu, inc, 31);
+                    const uint32_t base = inc - sum;
+#pragma unroll
+                    for (int k = 0; k < ITEMS; k++) {
+                        const int idx = k * NW + warp;
+                        const int owner = idx / PER, off = idx % PER;
+                        uint32_t part_sum = 0;
+#pragma unroll
+                        for (int qq = 0; qq < PER; qq++)
+                            if (qq < off) part_sum += v[qq];
+                        pre[k] = __shfl_sync(0xffffffffu, base + part_sum, owner);
+                    }
+                }
+                if (warp == 0 && lane == 31) {
+                    // publish the tile aggregate before anything can block this CTA
+                    if (t > 0 && !(L.dbg & 1))
+                        st_relaxed_u64(&L.status[b * L.status_stride + t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
+                    if (L.dbg & 4)
+                        L.dbg_ts[10 * t + 2] = globaltimer();
+                }
+                // ring bytes for the compacted tile (blocks never wrap); every warp computes
+                // the same reservation from the same (head, hpos, total)
+                const int c0 = b ? P.br_out_end[b - 1] : 0, c1 = NB > 1 ? (int)P.br_out_end[b] : P.nout;
+                uint32_t need = 0;
+                for (int c = c0; c < c1; c++)
+                    need += al16(total * P.out_w[c]);
+                if ((L.dbg & 4) && tid == 0)
+                    L.dbg_ts[10 * t + 9] = globaltimer();
+                uint32_t pos = hpos;
+                uint32_t used = need;
+                bool drain = false;
+                if (pos + need > R) {           // skip the tail [pos, R)
+                    used += R - pos;
+                    pos = 0;
+                    if (used > R) {             // cannot fit behind live blocks: wait for an empty ring
+                        used = need;
+                        drain = true;
+                    }
+                }
+                if (ublk >= kRingSlots)
+                    mbar_wait(&ctl->blk[j].oempty, (uint32_t)(((ublk / kRingSlots) - 1) & 1));
+                {
+                    uint32_t backoff = 32;
+                    while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
+                        __nanosleep(backoff);
+                        backoff = backoff < 512 ? backoff * 2 : 512;
+                    }
+                }
+                head += used;
+                hpos = pos + need == R ? 0 : pos + need;
+                char *blk = ring + pos;
+                const uint32_t lt = lanemask_lt();
+                uint32_t posk[ITEMS];
+#pragma unroll
+                for (int k = 0; k < ITEMS; k++)
+                    posk[k] = pre[k] + __popc(bal[k] & lt);
+                uint32_t coff = 0;
+                for (int c = c0; c < c1; c++) {
+                    const int w = P.out_w[c];
+                    const char *src = loc_ptr(P.out_loc[c], st, scratch);
+                    char *dst = blk + coff;
+                    coff += al16(total * w);
+                    switch (w) {
+                    case 1:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if ((mask >> k) & 1u) ((uint8_t *)dst)[posk[k]] = ((const uint8_t *)src)[k * NT + tid];
+                        break;
+                    case 4:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if ((mask >> k) & 1u) ((uint32_t *)dst)[posk[k]] = ((const uint32_t *)src)[k * NT + tid];
+                        break;
+                    default:
+#pragma unroll
+                        for (int k = 0; k < ITEMS; k++)
+                            if ((mask >> k) & 1u) ((uint64_t *)dst)[posk[k]] = ((const uint64_t *)src)[k * NT + tid];
+                        break;
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    if (gring)
+                        __threadfence_block();
+                    if (warp == 0) {
+                        ctl->blk[j].tile = t;
+                        ctl->blk[j].total = total;
+                        ctl->blk[j].roff = pos;
+                        ctl->blk[j].used = used;
+                        ctl->blk[j].br = (uint32_t)b;
+                    }
+                    if (b == NB - 1)
+                        mbar_arrive(&ctl->in[s].empty);      // this warp is done with the stage
+                    mbar_arrive(&ctl->blk[j].aggr);          // and with the ring block
+                    if ((L.dbg & 4) && warp == 0)
+                        L.dbg_ts[10 * t + 8] = globaltimer();
+                }
+                ++ublk;
+                if (++b == NB)
                     break;
-                case 4:
-#pragma unroll
-                    for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint32_t *)dst)[posk[k]] = ((const uint32_t *)src)[k * NT + tid];
-                    break;
-                default:
-#pragma unroll
-                    for (int k = 0; k < ITEMS; k++)
-                        if ((mask >> k) & 1u) ((uint64_t *)dst)[posk[k]] = ((const uint64_t *)src)[k * NT + tid];
-                    break;
-                }
-            }
-            __syncwarp();
-            if (lane == 0) {
-                if (gring)
-                    __threadfence_block();
-                if (warp == 0) {
-                    ctl->blk[j].tile = t;
-                    ctl->blk[j].total = total;
-                    ctl->blk[j].roff = pos;
-                    ctl->blk[j].used = used;
-                }
-                mbar_arrive(&ctl->in[s].empty);          // this warp is done with the stage
-                mbar_arrive(&ctl->blk[j].aggr);          // and with the ring block
-                if ((L.dbg & 4) && warp == 0)
-                    L.dbg_ts[10 * t + 8] = globaltimer();
+                mask = run_ops<NT, ITEMS>(P, P.br_op_end[b - 1], P.br_op_end[b], st, scratch, mask0);
             }
         }
     }
@@ -629,6 +648,8 @@ __global__ void __launch_bounds__(NT + kAuxThreads, AGG ? 1 : 2) k_scan_chain(co
         }
     } else if ((ntiles == 0 || L.direct) && blockIdx.x == 0 && tid == 0) {
         *L.n_dev = L.direct ? n : 0;
+        for (int b = 1; b < NB; b++)
+            *L.br_n_dev[b] = 0;
     }
     cta_exit_reset(L.ctrs);
 }
@@ -1200,9 +1221,11 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         default: return occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
         }
     case 1:
-        if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + kAuxThreads);
-        return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + kAuxThreads)
-                          : occ(k_scan_chain<256, 8, true, false>, smem, 256 + kAuxThreads);
+        if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + 32);
+        if (nt == 384) return occ(k_scan_chain<384, 5, true, false>, smem, 384 + 32);
+        if (nt == 448) return occ(k_scan_chain<448, 4, true, false>, smem, 448 + 32);
+        return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + 32)
+                          : occ(k_scan_chain<256, 8, true, false>, smem, 256 + 32);
     case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
     default: return occ(k_join_runs<uint64_t, true>, smem);
     }
@@ -1213,7 +1236,7 @@ static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int 
 {
     JoinExpand X{};
     cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_chain<NT, ITEMS, AGG, false><<<grid, NT + kAuxThreads, smem, s>>>(P, L, X);
+    k_scan_chain<NT, ITEMS, AGG, false><<<grid, NT + aux_threads(AGG), smem, s>>>(P, L, X);
     return cudaGetLastError();
 }
 
@@ -1232,6 +1255,10 @@ cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg,
     if (agg) {
         if (nt == 128)
             return sc<128, 16, true>(P, L, smem, grid, s);
+        if (nt == 384)
+            return sc<384, 5, true>(P, L, smem, grid, s);
+        if (nt == 448)
+            return sc<448, 4, true>(P, L, smem, grid, s);
         return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
     }
     if (nt == 512)

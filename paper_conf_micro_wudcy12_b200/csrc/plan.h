@@ -44,6 +44,9 @@ struct Group {
     int source = -1;                 // G_SCAN: producer node whose relation is scanned
     int join = -1;                   // G_JOIN: the JOIN node
     std::vector<int> chain;          // SELECT / PROJECT nodes fused after the source / join
+    // input-dependence fusion (§4.4, Fig. 14(d)): several chains over the same
+    // G_SCAN source, one output each (chain unused when non-empty)
+    std::vector<std::vector<int>> branches;
     int agg = -1;                    // AGG terminal (or -1: materialising terminal)
     int out = -1;                    // node whose relation this group produces
     std::vector<int> deps;           // groups that must run first

@@ -402,6 +402,7 @@ struct HOp {
     uint8_t kind, op, type, b_is_slot;
     int16_t dst, a, b, pad;
     int64_t k;
+    int br;                     // branch (input-dependence fusion), ops are in branch order
 };
 
 struct SlotB {
@@ -439,13 +440,26 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     for (size_t c = 0; c < cur.size(); c++)
         cur[c] = -1 - (int)c;
     auto resolve = [&](int v) { return v >= 0 ? v : get_src(-1 - v); };
+    int cur_br = 0;
     auto push = [&](const HOp &o) {
         if ((int)ops.size() >= kMaxOps)
             raise(RW_E_UNSUPPORTED, "fused group exceeds the micro-op budget");
         ops.push_back(o);
+        ops.back().br = cur_br;
     };
-
-    for (int nid : g.chain) {
+    const int nbr = g.branches.empty() ? 1 : (int)g.branches.size();
+    if (nbr > kMaxBranch)
+        raise(RW_E_UNSUPPORTED, "more than 4 input-dependent branches in one group");
+    if (nbr > 1 && g.agg >= 0)
+        raise(RW_E_UNSUPPORTED, "input-dependence fusion of aggregates");
+    std::vector<int> term;
+    std::vector<int> term_end;        // per branch: end of its terminal columns in term
+    for (cur_br = 0; cur_br < nbr; cur_br++) {
+    const std::vector<int> &chain_b = g.branches.empty() ? g.chain : g.branches[cur_br];
+    cur.resize(src_types.size());
+    for (size_t c = 0; c < src_types.size(); c++)
+        cur[c] = -1 - (int)c;
+    for (int nid : chain_b) {
         const Node &nd = p->nodes[nid];
         if (nd.kind == N_SELECT) {
             for (const rw_pred &a : nd.preds) {
@@ -561,10 +575,17 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             cur = next;
         }
     }
+    if (nbr > 1) {
+        for (int v : cur)
+            term.push_back(resolve(v));
+        term_end.push_back((int)term.size());
+    }
+    }   // branches
 
     // terminal
-    std::vector<int> term;
-    if (g.agg >= 0) {
+    if (nbr > 1) {
+        // materialising terminals collected per branch above
+    } else if (g.agg >= 0) {
         const Node &a = p->nodes[g.agg];
         L.agg = true;
         L.P.is_agg = 1;
@@ -706,6 +727,14 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     P.nslots = (int)slots.size();
     P.nin = nin;
     P.nops = (int)ops.size();
+    P.nbranch = nbr;
+    for (int b = 0; b < nbr; b++) {
+        int e = 0;
+        for (size_t i = 0; i < ops.size(); i++)
+            if (ops[i].br <= b) e = (int)i + 1;
+        P.br_op_end[b] = (uint8_t)e;
+        P.br_out_end[b] = (uint8_t)(nbr > 1 ? term_end[b] : (int)term.size());
+    }
     for (size_t i = 0; i < order.size(); i++) {
         const SlotB &sb = slots[order[i]];
         P.slot[i].type = (uint8_t)sb.type;
@@ -850,7 +879,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     // per CTA, C2 2.59 -> 2.29 ms); opts.reserved[6] == 2 keeps the ring in smem
     const bool global_ring = !L.agg && p->o.reserved[6] != 2;
     L.gring_bytes = 0;
-    bool direct = !L.agg;
+    bool direct = !L.agg && nbr == 1;
     for (const HOp &h : ops)
         if (h.kind == K_PRED)
             direct = false;
@@ -870,6 +899,14 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         vars.push_back({256, 5});
     }
     vars.push_back({256, 4});
+    // register terminal: 14 compute warps per SM by default (the aggregate kernel has
+    // no writer warps, so its register file takes more compute threads; measured C4
+    // 8.56 ms at 256 x 8, 7.43 ms at 384 x 5, 7.06 ms at 448 x 4); opts.reserved[4]:
+    // 1 = the 256-thread variants, 4 = 384 x 5
+    if (L.agg && agg_mode_for(256) == 2 && p->o.reserved[4] != 1) {
+        vars.clear();
+        vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : Var{448, 4});
+    }
     if (force_items > 0) {
         std::vector<Var> v2;
         for (const Var &v : vars)
@@ -1287,6 +1324,126 @@ void execute(rw_plan *p, const rw_relation_in *in, int nin, int out_node, rw_rel
         if (out->n > out->capacity)
             raise(RW_E_CAPACITY, "output needs " + std::to_string(out->n) + " rows, capacity " +
                                      std::to_string(out->capacity));
+    }
+}
+
+// Input-dependence fusion (§4.4, Fig. 14(d)): the SELECT / PROJECT chains from
+// one common INPUT to each requested node become the branches of one scan group.
+void execute_multi(rw_plan *p, const rw_relation_in *in, int nin, const int32_t *nodes, int nout,
+                   rw_relation_out *outs)
+{
+    if (nout <= 0 || !nodes || !outs)
+        raise(RW_E_ARG, "execute_multi: no outputs");
+    for (int k = 0; k < nout; k++) {
+        node_at(p, nodes[k]);
+        if (!outs[k].cols && outs[k].capacity > 0)
+            raise(RW_E_ARG, "null output");
+    }
+    check_inputs(p, in, nin);
+    cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    std::vector<std::vector<int>> chains(nout);
+    int src = -1;
+    bool fusable = p->o.fuse && nout > 1 && nout <= kMaxBranch;
+    for (int k = 0; k < nout && fusable; k++) {
+        int cur = nodes[k];
+        while (is_unary_chain(p->nodes[cur].kind)) {
+            chains[k].insert(chains[k].begin(), cur);
+            cur = p->nodes[cur].in;
+        }
+        if (chains[k].empty() || p->nodes[cur].kind != N_INPUT || (src >= 0 && cur != src))
+            fusable = false;
+        src = cur;
+    }
+    if (!fusable) {
+        int64_t launches = 0;
+        for (int k = 0; k < nout; k++) {
+            execute(p, in, nin, nodes[k], &outs[k]);
+            launches += p->launches;
+        }
+        p->launches = launches;
+        return;
+    }
+    p->launches = 0;
+    Group g;
+    g.kind = G_SCAN;
+    g.source = src;
+    g.out = nodes[0];
+    g.branches = chains;
+    const Node &sn = p->nodes[src];
+    Lowered L;
+    lower(p, g, sn.types, L);
+    const rw_relation_in &ri = in[sn.input_index];
+    const int T = L.tile;
+    bool aligned = true;
+    for (int i = 0; i < L.P.nin; i++) {
+        L.P.in_ptr[i] = ri.cols[L.in_src[i]];
+        if (((uintptr_t)L.P.in_ptr[i]) & 15)
+            aligned = false;
+    }
+    if (p->cnt_cap < nout + 1) {
+        if (p->cnt) cudaFreeAsync(p->cnt, p->stream);
+        p->cnt_cap = nout + 8;
+        p->cnt = (int64_t *)dev_alloc(p, (size_t)p->cnt_cap * 8);
+    }
+    int c = 0;
+    for (int k = 0; k < nout; k++) {
+        const int ncol = (int)p->nodes[nodes[k]].types.size();
+        if (L.P.br_out_end[k] != c + ncol)
+            raise(RW_E_ARG, "execute_multi: branch schema mismatch");
+        for (int q = 0; q < ncol; q++)
+            L.P.out_ptr[c + q] = outs[k].cols[q];
+        c += ncol;
+        L.P.br_cap[k] = outs[k].capacity;
+    }
+    L.P.out_capacity = outs[0].capacity;
+    const int64_t max_tiles = (ri.n + T - 1) / T;
+    ensure_status(p, (int64_t)nout * (max_tiles + 1));
+    TileLaunch TL{};
+    TL.n = ri.n;
+    TL.stages = L.stages;
+    TL.dbg = p->o.reserved[1] & ~4;
+    TL.out_bytes = L.out_bytes;
+    TL.direct = 0;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(max_tiles, (int64_t)p->sms * L.ctas));
+    if (L.gring_bytes) {
+        const size_t need = (size_t)grid * L.gring_bytes;
+        if (need > p->gring_cap) {
+            if (p->gring) cudaFreeAsync(p->gring, p->stream);
+            p->gring = (char *)dev_alloc(p, need);
+            p->gring_cap = need;
+        }
+        TL.gring = p->gring;
+    }
+    TL.use_tma = aligned ? 1 : 0;
+    TL.epoch = next_epoch(p);
+    TL.status = p->status;
+    TL.status_stride = max_tiles + 1;
+    TL.ctrs = p->ctrs;
+    TL.err = p->err;
+    for (int k = 0; k < nout; k++) {
+        int64_t *nd = outs[k].n_dev ? outs[k].n_dev : p->cnt + k;
+        if (k == 0) TL.n_dev = nd;
+        else TL.br_n_dev[k] = nd;
+    }
+    cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain<multi>");
+    p->launches++;
+    bool any_sync = false;
+    for (int k = 0; k < nout; k++)
+        if (!outs[k].n_dev) {
+            cuda_check(cudaMemcpyAsync(p->jtot_host + 4 + k, p->cnt + k, 8, cudaMemcpyDeviceToHost, p->stream),
+                       "copy n");
+            any_sync = true;
+        }
+    if (any_sync)
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+    for (int k = 0; k < nout; k++) {
+        outs[k].n = -1;
+        if (outs[k].n_dev)
+            continue;
+        outs[k].n = p->jtot_host[4 + k];
+        if (outs[k].n > outs[k].capacity)
+            raise(RW_E_CAPACITY, "output " + std::to_string(k) + " needs " + std::to_string(outs[k].n) +
+                                     " rows, capacity " + std::to_string(outs[k].capacity));
     }
 }
 
@@ -1712,6 +1869,17 @@ rw_status rw_plan_execute(rw_plan *p, const rw_relation_in *in, int32_t nin, int
     if (!p)
         raise(RW_E_ARG, "null plan");
     execute(p, in, nin, out_node, out);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_execute_multi(rw_plan *p, const rw_relation_in *in, int32_t nin, const int32_t *out_nodes,
+                                int32_t nout, rw_relation_out *outs)
+{
+    RW_TRY
+    if (!p)
+        raise(RW_E_ARG, "null plan");
+    execute_multi(p, in, nin, out_nodes, nout, outs);
     return RW_OK;
     RW_CATCH
 }

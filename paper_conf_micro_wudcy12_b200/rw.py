@@ -61,7 +61,7 @@ class rw_relation_out(ctypes.Structure):
 
 EXPORTS = ["rw_plan_create", "rw_plan_destroy", "rw_plan_add_input", "rw_plan_add_select",
            "rw_plan_add_project", "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema",
-           "rw_plan_execute", "rw_plan_execute_host", "rw_plan_explain", "rw_plan_last_launches",
+           "rw_plan_execute", "rw_plan_execute_multi", "rw_plan_execute_host", "rw_plan_explain", "rw_plan_last_launches",
            "rw_status_str", "rw_last_error", "rw_split_by_splitters", "rw_merge_runs",
            "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]
 
@@ -89,6 +89,7 @@ def lib():
     L.rw_plan_node_schema.argtypes = [vp, i32, P(i32), P(i32)]
     L.rw_plan_execute.argtypes = [vp, P(rw_relation_in), i32, i32, P(rw_relation_out)]
     L.rw_plan_execute_host.argtypes = [vp, P(rw_relation_in), i32, i32, P(rw_relation_out)]
+    L.rw_plan_execute_multi.argtypes = [vp, P(rw_relation_in), i32, P(i32), i32, P(rw_relation_out)]
     L.rw_plan_explain.argtypes = [vp, i32, ctypes.c_char_p, ctypes.c_size_t]
     L.rw_plan_last_launches.argtypes = [vp]
     L.rw_plan_last_launches.restype = i64
@@ -102,7 +103,7 @@ def lib():
     L.rw_plan_agg_import.argtypes = [vp, i32, vp, P(rw_relation_out)]
     for f in ["rw_plan_create", "rw_plan_add_input", "rw_plan_add_select", "rw_plan_add_project",
               "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema", "rw_plan_execute",
-              "rw_plan_execute_host", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs",
+              "rw_plan_execute_host", "rw_plan_execute_multi", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs",
               "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]:
         getattr(L, f).restype = i32
     _lib = L
@@ -255,6 +256,34 @@ class Plan:
                               ctypes.c_void_p(_ptr(n_dev)) if n_dev is not None else None, -1)
         check(lib().rw_plan_execute(self.h, arr, len(inputs), out_node, ctypes.byref(out)))
         return None if n_dev is not None else out.n
+
+    def execute_multi(self, inputs, out_nodes, out_cols, capacities, n_devs=None):
+        """Input-dependence fusion: out_cols[k] / capacities[k] (/ n_devs[k]) receive
+        out_nodes[k].  Returns the row counts (synchronising) or None with n_devs."""
+        arr, keep = self._inputs(inputs)
+        k = len(out_nodes)
+        outs = (rw_relation_out * k)()
+        for i in range(k):
+            oc = (ctypes.c_void_p * max(1, len(out_cols[i])))(*[_ptr(x) for x in out_cols[i]])
+            keep.append(oc)
+            outs[i].cols = ctypes.cast(oc, ctypes.POINTER(ctypes.c_void_p))
+            outs[i].capacity = int(capacities[i])
+            outs[i].n_dev = _ptr(n_devs[i]) if n_devs is not None else None
+            outs[i].n = -1
+        check(lib().rw_plan_execute_multi(self.h, arr, len(inputs), _i32arr(out_nodes), k, outs))
+        return None if n_devs is not None else [outs[i].n for i in range(k)]
+
+    def run_multi(self, inputs, out_nodes, capacity: Optional[int] = None):
+        """Allocate torch outputs for every node, execute_multi, return [(tensors, n)]."""
+        import torch
+        if capacity is None:
+            capacity = max([int(n) for n, _ in inputs] + [1])
+        dt = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64,
+              "u8": torch.uint8}
+        cols = [[torch.empty(max(capacity, 1), dtype=dt[t], device=f"cuda:{self.device}")
+                 for t in self.node_schema(nd)] for nd in out_nodes]
+        ns = self.execute_multi(inputs, out_nodes, cols, [capacity] * len(out_nodes))
+        return [([c[:n] for c in cs], n) for cs, n in zip(cols, ns)]
 
     def execute_host(self, inputs, out_node: int, out_cols, capacity: int) -> int:
         """Same with HOST buffers (numpy arrays / pinned torch tensors / pointers)."""

@@ -49,13 +49,33 @@ def run_gpu(spec: Dict, inputs: Dict[str, List], capacity=None, plan=None, **opt
     return oracle.Relation(types, host), plan
 
 
-def run_oracle(spec: Dict, inputs: Dict[str, List]):
+def run_gpu_multi(spec: Dict, inputs: Dict[str, List], capacity=None, **opts):
+    """Every node of spec["outs"] through rw_plan_execute_multi.  Returns ([Relation], plan)."""
+    import torch
+    plan, ids = build_gpu_plan(spec, **opts)
+    ins = [(int(inputs[k][0].numel()) if inputs[k] else 0, inputs[k]) for k in spec["inputs"]]
+    nodes = [ids[o] for o in spec["outs"]]
+    res = plan.run_multi(ins, nodes, capacity)
+    torch.cuda.synchronize()
+    rels = []
+    for nd, (cols, n) in zip(nodes, res):
+        types = plan.node_schema(nd)
+        rels.append(oracle.Relation(types, [c.cpu().numpy().view(NPT[t]) for c, t in zip(cols, types)]))
+    return rels, plan
+
+
+def run_oracle_multi(spec: Dict, inputs: Dict[str, List]):
+    env = run_oracle(spec, inputs, keep_all=True)
+    return [env[o] for o in spec["outs"]]
+
+
+def run_oracle(spec: Dict, inputs: Dict[str, List], keep_all: bool = False):
     rels = {}
     for name, inp in spec["inputs"].items():
         cols = [(c.cpu().numpy() if hasattr(c, "cpu") else np.asarray(c)).view(NPT[t])
                 for c, t in zip(inputs[name], inp["types"])]
         rels[name] = oracle.Relation(inp["types"], cols)
-    return oracle.evaluate(spec, rels)
+    return oracle.evaluate(spec, rels, keep_all=keep_all)
 
 
 def assert_same(gpu: "oracle.Relation", ref: "oracle.Relation", ordered: bool = True):

@@ -54,6 +54,20 @@ def c2_inputs(n: int, start: int = 0, device="cpu", cfg: int = 2) -> Dict[str, L
     return {"R": [r[f"c{c}"] for c in range(4)]}
 
 
+# ---- pattern (d): input dependence (§4.4, Fig. 14(d)) ------------
+# k SELECTs filter the same 16-byte tuples; branch b keeps the rows with
+# c_b < threshold (selectivity s each, reading A13) and all four columns.
+def cd_spec(s: float = 0.25, k: int = 2) -> Dict:
+    nodes = [{"id": f"d{b}", "op": "select", "in": "R", "preds": [(b, "<", thr_i32(s))]} for b in range(k)]
+    return {"inputs": {"R": {"types": ["i32"] * 4, "nkey_sorted": 0}}, "nodes": nodes,
+            "outs": [f"d{b}" for b in range(k)], "out": "d0"}
+
+
+def cd_inputs(n: int, start: int = 0, device="cpu", cfg: int = 6) -> Dict[str, List]:
+    r = rwgen.uniform_u32_relation(cfg, 0, 4, start, n, device)
+    return {"R": [r[f"c{c}"] for c in range(4)]}
+
+
 # ---- C3: JOIN (Zipf 0.5) -> SELECT -> PROJECT ---------------------------------
 def c3_spec() -> Dict:
     return {"inputs": {"L": {"types": ["u32", "u32"], "nkey_sorted": 1},
