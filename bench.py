@@ -411,7 +411,7 @@ def main():
             et = float(t.item())
         line["e2e"] = {"value": n_in * world / et, "unit": "tuples/s", "h2d_bytes_per_step": in_bytes,
                        "d2h_bytes_per_step": n_e * sum(W[t] for t in etypes), "ms_per_step": et * 1e3,
-                       "api": "rw_plan_execute_host (pinned host buffers)"}
+                       "api": "rw_plan_execute_host (pinned host buffers; 2^25-row chunks, H2D / kernel / D2H overlapped on 3 streams)"}
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:

@@ -101,6 +101,8 @@ typedef struct {
     int32_t stages;           /* 0 = auto: TMA tiles in flight per CTA (1..8) */
     int32_t ctas_per_sm;      /* 0 = auto (occupancy) */
     int32_t strict_overflow;  /* 1: reject i64/u64 expressions whose interval may wrap */
+    int32_t host_chunk_log2;  /* rw_plan_execute_host: rows per streamed chunk = 2^this
+                                 (0 = auto, 2^25) */
     int32_t reserved[8];
 } rw_plan_opts;
 
@@ -188,7 +190,15 @@ rw_status rw_plan_execute_multi(rw_plan *plan, const rw_relation_in *in, int32_t
 
 /* Same, with HOST buffers: inputs are copied host->device, the plan runs, the result
  * (up to capacity rows) is copied device->host, the stream is synchronised and out->n
- * set.  Pinned (cudaHostAlloc / registered) buffers give full PCIe bandwidth. */
+ * set.  Pinned (cudaHostAlloc / registered) buffers give full PCIe bandwidth.
+ * Host streaming (the paper's PCIe experiment, §5.1.3): when the plan is
+ * one fused scan group over one INPUT relation (SELECT / PROJECT / arithmetic chain,
+ * optionally ending in an AGG) and the input exceeds one chunk (opts.host_chunk_log2),
+ * it runs chunk by chunk with the H2D copy of chunk k+1, the kernel of chunk k and the
+ * D2H copy of chunk k-1's compacted rows overlapped on three streams (double-buffered
+ * device chunks, allocated per call).  The result is identical to the unchunked run,
+ * row order included; an aggregate accumulates every chunk and finalises once.
+ * Other plans copy the whole inputs first. */
 rw_status rw_plan_execute_host(rw_plan *plan, const rw_relation_in *in, int32_t nin, int32_t out_node,
                                rw_relation_out *out);
 

@@ -120,7 +120,7 @@ struct TileLaunch {
     int32_t *err;              // [0] domain errors
     int32_t dbg;               // diagnostics: 1 = skip look-back (offset = tile * T, uncompacted),
                                // 2 = stream tiles only, 4 = per-tile phase timestamps into dbg_ts
-    uint64_t *dbg_ts;          // 10 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots, scattered, reserve start)
+    uint64_t *dbg_ts;          // 12 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots, scattered, reserve start; join: records cached, gathered)
 };
 
 // Join expansion inputs (run records written by k_join_runs).

@@ -130,7 +130,7 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
 // then a forward walk; ITEMS odd makes the thread-contiguous smem writes conflict-free.
 template <int NT, int ITEMS>
 __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_t t, int64_t ntiles, int rows,
-                                 char *st, char *rcache)
+                                 char *st, char *rcache, const TileLaunch &L)
 {
     constexpr int T = NT * ITEMS;
     const int tid = threadIdx.x;
@@ -143,12 +143,15 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
     const int64_t r1 = (t + 1 < ntiles) ? X.tile_run[t + 1] : X.nruns - 1;
     const int nr = (int)(r1 - r0 + 1);
     for (int q = tid; q < nr; q += NT) {
-        c_off[q] = X.off[r0 + q];
-        c_s[q] = X.s[r0 + q];
-        c_lo[q] = X.lo[r0 + q];
-        c_lenR[q] = X.lenR[r0 + q];
+        cp_async8(c_off + q, X.off + r0 + q);
+        cp_async4(c_s + q, X.s + r0 + q);
+        cp_async4(c_lo + q, X.lo + r0 + q);
+        cp_async4(c_lenR + q, X.lenR + r0 + q);
     }
+    cp_async_wait_all();
     bar_sync(kComputeBar, NT);
+    if ((L.dbg & 4) && tid == 0)
+        L.dbg_ts[12 * t + 10] = globaltimer();
     const int first = tid * ITEMS;
     if (first < rows) {
         uint32_t ii[ITEMS], jj[ITEMS];
@@ -193,6 +196,8 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
                 }
             }
         }
+        // every gather of every live column is issued as an async copy before any
+        // completes (one round trip per tile instead of one per column)
         for (int c = 0; c < X.ncols; c++) {
             char *dst = st + P.slot[X.dst_slot[c]].off;
             const int w = type_width(P.slot[X.dst_slot[c]].type);
@@ -203,15 +208,18 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
                 if (first + k < rows) {
                     const size_t row = right ? jj[k] : ii[k];
                     if (w == 4)
-                        ((uint32_t *)dst)[first + k] = ((const uint32_t *)src)[row];
+                        cp_async4((uint32_t *)dst + first + k, (const uint32_t *)src + row);
                     else if (w == 8)
-                        ((uint64_t *)dst)[first + k] = ((const uint64_t *)src)[row];
+                        cp_async8((uint64_t *)dst + first + k, (const uint64_t *)src + row);
                     else
                         ((uint8_t *)dst)[first + k] = ((const uint8_t *)src)[row];
                 }
             }
         }
+        cp_async_wait_all();
     }
+    if ((L.dbg & 4) && tid == 0)
+        L.dbg_ts[12 * t + 11] = globaltimer();
     bar_sync(kComputeBar, NT);
 }
 
@@ -286,7 +294,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 const int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
-                    L.dbg_ts[10 * t + 0] = globaltimer();
+                    L.dbg_ts[12 * t + 0] = globaltimer();
                 if (!JOIN && t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
                     char *st = stages + (size_t)s * P.stage_bytes;
                     fence_proxy_async_smem();
@@ -322,13 +330,13 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 const uint32_t total = ctl->blk[j].total;
                 const int b = (int)ctl->blk[j].br;
                 if ((L.dbg & 4) && lane == 0)
-                    L.dbg_ts[10 * t + 5] = globaltimer();
+                    L.dbg_ts[12 * t + 5] = globaltimer();
                 const int64_t excl = (L.dbg & 1) ? t * T
                                                   : (int64_t)lookback_warp(L.status + b * L.status_stride, t, total, L.epoch,
                                                                            /*aggregate_published=*/true);
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[10 * t + 3] = globaltimer();
+                        L.dbg_ts[12 * t + 3] = globaltimer();
                     if (t == ntiles - 1)
                         *(b ? L.br_n_dev[b] : L.n_dev) = excl + (int64_t)total;
                 }
@@ -357,7 +365,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 }
                 if (lane == 0) {
                     if (L.dbg & 4)
-                        L.dbg_ts[10 * t + 4] = globaltimer();
+                        L.dbg_ts[12 * t + 4] = globaltimer();
                     if (i > 0)   // release ring bytes in tile order
                         mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1), 64);
                     // the discards must land in L2 before the bytes can be rewritten
@@ -416,7 +424,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
             const int64_t row0 = t * T;
             const int rows = (int)min((int64_t)T, n - row0);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[10 * t + 1] = globaltimer();
+                L.dbg_ts[12 * t + 1] = globaltimer();
             auto release_stage = [&]() {
                 __syncwarp();
                 if (lane == 0)
@@ -427,7 +435,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 continue;
             }
             if (JOIN) {
-                join_fill<NT, ITEMS>(P, X, t, ntiles, rows, st, rcache);
+                join_fill<NT, ITEMS>(P, X, t, ntiles, rows, st, rcache, L);
             } else if (!(L.use_tma && rows == T)) {
                 // ragged last tile or unaligned column bases: each thread loads its own rows
                 for (int c = 0; c < P.nin; c++) {
@@ -456,7 +464,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
             }
             uint32_t mask = run_ops<NT, ITEMS>(P, 0, NB > 1 ? (int)P.br_op_end[0] : P.nops, st, scratch, mask0);
             if ((L.dbg & 4) && tid == 0)
-                L.dbg_ts[10 * t + 6] = globaltimer();
+                L.dbg_ts[12 * t + 6] = globaltimer();
             if (AGG) {
                 if (P.agg_mode == 2)
                     agg_tile_reg<NT, ITEMS>(P, st, scratch, mask, racc, cta_acc, since_flush, L.err);
@@ -465,7 +473,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 else
                     agg_tile<NT, ITEMS>(P, st, scratch, mask, part, cta_acc, since_flush, L.err);
                 if ((L.dbg & 4) && tid == 0)
-                    L.dbg_ts[10 * t + 2] = globaltimer();
+                    L.dbg_ts[12 * t + 2] = globaltimer();
                 release_stage();
                 continue;
             }
@@ -510,7 +518,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 }
                 bar_sync(kComputeBar, NT);
                 if ((L.dbg & 4) && tid == 0)
-                    L.dbg_ts[10 * t + 7] = globaltimer();
+                    L.dbg_ts[12 * t + 7] = globaltimer();
                 // every warp scans the ITEMS x NW survivor counts itself
                 uint32_t pre[ITEMS];
                 uint32_t total;
@@ -550,7 +558,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                     if (t > 0 && !(L.dbg & 1))
                         st_relaxed_u64(&L.status[b * L.status_stride + t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
                     if (L.dbg & 4)
-                        L.dbg_ts[10 * t + 2] = globaltimer();
+                        L.dbg_ts[12 * t + 2] = globaltimer();
                 }
                 // ring bytes for the compacted tile (blocks never wrap); every warp computes
                 // the same reservation from the same (head, hpos, total)
@@ -559,7 +567,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 for (int c = c0; c < c1; c++)
                     need += al16(total * P.out_w[c]);
                 if ((L.dbg & 4) && tid == 0)
-                    L.dbg_ts[10 * t + 9] = globaltimer();
+                    L.dbg_ts[12 * t + 9] = globaltimer();
                 uint32_t pos = hpos;
                 uint32_t used = need;
                 bool drain = false;
@@ -627,7 +635,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                         mbar_arrive(&ctl->in[s].empty);      // this warp is done with the stage
                     mbar_arrive(&ctl->blk[j].aggr);          // and with the ring block
                     if ((L.dbg & 4) && warp == 0)
-                        L.dbg_ts[10 * t + 8] = globaltimer();
+                        L.dbg_ts[12 * t + 8] = globaltimer();
                 }
                 ++ublk;
                 if (++b == NB)

@@ -123,6 +123,17 @@ struct rw_plan {
     std::map<int, unsigned long long *> agg_acc;
     uint32_t epoch = 0;
     int64_t launches = 0;
+    bool defer_finalize = false;  // host-streamed aggregate: chunks accumulate, the last one finalises
+    // host streaming (execute_host): copy streams, events and double-buffered chunk
+    // buffers, created on first use and kept for the plan's lifetime
+    struct HostStream {
+        bool init = false;
+        cudaStream_t sh = nullptr, sd = nullptr;
+        cudaEvent_t ev[4][2];
+        char *buf = nullptr;
+        size_t bytes = 0;
+        int64_t *hcnt = nullptr;
+    } hs;
     std::vector<void *> temps;    // freed (stream-ordered) at the end of every execute
 };
 
@@ -1163,8 +1174,10 @@ void run_group(ExecCtx &X, int gi)
             L.F.capacity = capacity;
             L.F.n_dev = n_dev;
             L.F.err = p->err;
-            cuda_check(agg_finalize_launch(L.F, p->stream), "k_agg_finalize");
-            p->launches++;
+            if (!p->defer_finalize) {
+                cuda_check(agg_finalize_launch(L.F, p->stream), "k_agg_finalize");
+                p->launches++;
+            }
         } else {
             for (size_t c = 0; c < outp.size(); c++)
                 L.P.out_ptr[c] = outp[c];
@@ -1256,6 +1269,7 @@ void run_group(ExecCtx &X, int gi)
         TL.err = p->err;
         TL.out_bytes = L.out_bytes;
         TL.dbg = p->o.reserved[1];
+        TL.dbg_ts = (uint64_t *)(((uint64_t)(uint32_t)p->o.reserved[3] << 32) | (uint32_t)p->o.reserved[2]);
         const int grid2 = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (int64_t)p->sms * L.ctas));
         cuda_check(join_chain_launch(L.P, TL, XJ, L.smem, grid2, p->stream), "k_scan_chain<join>");
         p->launches++;
@@ -1447,6 +1461,150 @@ void execute_multi(rw_plan *p, const rw_relation_in *in, int nin, const int32_t 
     }
 }
 
+// Host-streamed execution (the paper's PCIe experiment P:241-252):
+// a plan that is one scan group over one INPUT relation runs over row chunks.  The
+// H2D copy of chunk k+1 (copy stream), the fused kernel of chunk k (plan stream) and
+// the D2H copy of chunk k-1's compacted output (second copy stream) overlap; only
+// compacted rows cross PCIe back.  Chunk outputs are appended in chunk order, so the
+// result equals rw_plan_execute over the whole relation (row order included).  An
+// aggregate accumulates every chunk in its 128-bit accumulators and finalises once.
+// Returns false when the plan does not have that shape (the caller copies whole).
+bool execute_host_streamed(rw_plan *p, const rw_relation_in *in, int nin, int out_node, rw_relation_out *out)
+{
+    node_at(p, out_node);
+    if (p->nodes[out_node].kind == N_INPUT)
+        return false;
+    Grouping G = build_groups(p, out_node);
+    if (G.groups.size() != 1)
+        return false;
+    const Group &g = G.groups[0];
+    if (g.kind != G_SCAN || p->nodes[g.source].kind != N_INPUT)
+        return false;
+    const Node &sn = p->nodes[g.source];
+    const rw_relation_in &ri = in[sn.input_index];
+    const int lg = p->o.host_chunk_log2 > 0 ? std::min(p->o.host_chunk_log2, 31) : 25;
+    const int64_t C = (int64_t)1 << lg;
+    if (ri.n <= C)
+        return false;
+    const bool agg = g.agg >= 0;
+    const Node &on = p->nodes[out_node];
+    const int nci = (int)sn.types.size(), nco = (int)on.types.size();
+    const int64_t ocap = agg ? on.D : C;
+    const int64_t nch = (ri.n + C - 1) / C;
+    auto &H = p->hs;
+    if (!H.init) {
+        cuda_check(cudaStreamCreateWithFlags(&H.sh, cudaStreamNonBlocking), "stream");
+        cuda_check(cudaStreamCreateWithFlags(&H.sd, cudaStreamNonBlocking), "stream");
+        for (int a = 0; a < 4; a++)
+            for (int b = 0; b < 2; b++)
+                cuda_check(cudaEventCreateWithFlags(&H.ev[a][b], cudaEventDisableTiming), "event");
+        cuda_check(cudaMallocHost(&H.hcnt, 2 * sizeof(int64_t)), "cudaMallocHost");
+        H.init = true;
+    }
+    cudaStream_t sh = H.sh, sd = H.sd;
+    cudaEvent_t *ev_h2d = H.ev[0], *ev_in_free = H.ev[1], *ev_cnt = H.ev[2], *ev_out_free = H.ev[3];
+    int64_t *hcnt = H.hcnt;
+    // chunk buffers: 2 x (input columns, output columns, count), one allocation
+    size_t per = 0;
+    for (int c = 0; c < nci; c++) per += ((size_t)C * type_width(sn.types[c]) + 255) / 256 * 256;
+    for (int c = 0; c < nco; c++) per += ((size_t)ocap * type_width(on.types[c]) + 255) / 256 * 256;
+    per += 256;                                         // count; per stays a multiple of 256
+    if (2 * per > H.bytes) {
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+        if (H.buf) cudaFree(H.buf);
+        H.buf = nullptr;
+        H.bytes = 0;
+        cudaError_t e = cudaMalloc(&H.buf, 2 * per);
+        if (e == cudaErrorMemoryAllocation)
+            raise(RW_E_OOM, "host-streamed chunk buffers: out of device memory");
+        cuda_check(e, "cudaMalloc");
+        H.bytes = 2 * per;
+    }
+    auto cleanup = [&]() {
+        cudaStreamSynchronize(sh);
+        cudaStreamSynchronize(sd);
+        cudaStreamSynchronize(p->stream);
+        p->defer_finalize = false;
+    };
+    try {
+        std::vector<void *> ib[2], ob[2];
+        int64_t *nd[2];
+        for (int b = 0; b < 2; b++) {
+            char *q = H.buf + b * per;
+            for (int c = 0; c < nci; c++) {
+                ib[b].push_back(q);
+                q += ((size_t)C * type_width(sn.types[c]) + 255) / 256 * 256;
+            }
+            for (int c = 0; c < nco; c++) {
+                ob[b].push_back(q);
+                q += ((size_t)ocap * type_width(on.types[c]) + 255) / 256 * 256;
+            }
+            nd[b] = (int64_t *)q;
+        }
+        std::vector<rw_relation_in> din(in, in + nin);   // other inputs are unused by this plan
+        int64_t total = 0;
+        auto drain = [&](int64_t k) {      // compacted rows of chunk k -> host, appended
+            const int b = (int)(k & 1);
+            cuda_check(cudaEventSynchronize(ev_cnt[b]), "sync count");
+            const int64_t nk = hcnt[b];
+            const int64_t rows = std::max<int64_t>(0, std::min(nk, out->capacity - total));
+            for (int c = 0; c < nco; c++)
+                if (rows > 0)
+                    cuda_check(cudaMemcpyAsync((char *)out->cols[c] + (size_t)total * type_width(on.types[c]), ob[b][c],
+                                               (size_t)rows * type_width(on.types[c]), cudaMemcpyDeviceToHost, sd),
+                               "D2H");
+            cuda_check(cudaEventRecord(ev_out_free[b], sd), "event");
+            total += nk;
+        };
+        int64_t launches = 0;
+        for (int64_t k = 0; k < nch; k++) {
+            const int b = (int)(k & 1);
+            const int64_t r0 = k * C, rows = std::min(C, ri.n - r0);
+            if (k >= 2)
+                cuda_check(cudaStreamWaitEvent(sh, ev_in_free[b], 0), "wait");
+            for (int c = 0; c < nci; c++)
+                cuda_check(cudaMemcpyAsync(ib[b][c], (const char *)ri.cols[c] + (size_t)r0 * type_width(sn.types[c]),
+                                           (size_t)rows * type_width(sn.types[c]), cudaMemcpyHostToDevice, sh),
+                           "H2D");
+            cuda_check(cudaEventRecord(ev_h2d[b], sh), "event");
+            cuda_check(cudaStreamWaitEvent(p->stream, ev_h2d[b], 0), "wait");
+            if (k >= 2 && !agg)
+                cuda_check(cudaStreamWaitEvent(p->stream, ev_out_free[b], 0), "wait");
+            std::vector<const void *> cc(ib[b].begin(), ib[b].end());
+            din[sn.input_index].n = rows;
+            din[sn.input_index].cols = cc.data();
+            rw_relation_out dout{ob[b].data(), ocap, nd[b], -1};
+            p->defer_finalize = agg && k + 1 < nch;
+            execute(p, din.data(), nin, out_node, &dout);
+            launches += p->launches;
+            cuda_check(cudaEventRecord(ev_in_free[b], p->stream), "event");
+            cuda_check(cudaMemcpyAsync(hcnt + b, nd[b], 8, cudaMemcpyDeviceToHost, p->stream), "copy count");
+            cuda_check(cudaEventRecord(ev_cnt[b], p->stream), "event");
+            if (!agg && k >= 1)
+                drain(k - 1);
+        }
+        drain(nch - 1);
+        cuda_check(cudaStreamSynchronize(sd), "sync");
+        cuda_check(cudaStreamSynchronize(p->stream), "sync");
+        if (agg) {
+            cuda_check(cudaMemcpy(p->jtot_host + 3, p->err + 1, 4, cudaMemcpyDeviceToHost), "copy err");
+            const int32_t derr = ((int32_t *)(p->jtot_host + 3))[0];
+            if (derr)
+                raise(RW_E_DOMAIN, std::to_string(derr) + " rows had a group value outside its domain");
+        }
+        out->n = total;
+        p->launches = launches;
+    } catch (...) {
+        cleanup();
+        throw;
+    }
+    cleanup();
+    if (out->n > out->capacity)
+        raise(RW_E_CAPACITY, "output needs " + std::to_string(out->n) + " rows, capacity " +
+                                 std::to_string(out->capacity));
+    return true;
+}
+
 std::string explain(rw_plan *p, int out_node)
 {
     node_at(p, out_node);
@@ -1622,6 +1780,17 @@ void rw_plan_destroy(rw_plan *p)
     if (p->err) cudaFree(p->err);
     if (p->gring) cudaFree(p->gring);
     if (p->jtot_host) cudaFreeHost(p->jtot_host);
+    if (p->hs.init) {
+        cudaStreamSynchronize(p->hs.sh);
+        cudaStreamSynchronize(p->hs.sd);
+        if (p->hs.buf) cudaFree(p->hs.buf);
+        cudaFreeHost(p->hs.hcnt);
+        for (int a = 0; a < 4; a++)
+            for (int b = 0; b < 2; b++)
+                cudaEventDestroy(p->hs.ev[a][b]);
+        cudaStreamDestroy(p->hs.sh);
+        cudaStreamDestroy(p->hs.sd);
+    }
     delete p;
 }
 
@@ -1892,6 +2061,8 @@ rw_status rw_plan_execute_host(rw_plan *p, const rw_relation_in *in, int32_t nin
         raise(RW_E_ARG, "null argument");
     check_inputs(p, in, nin);
     cuda_check(cudaSetDevice(p->o.device), "cudaSetDevice");
+    if (execute_host_streamed(p, in, nin, out_node, out))
+        return RW_OK;
     std::vector<void *> dev;
     std::vector<std::vector<const void *>> dcols(nin);
     std::vector<rw_relation_in> din(nin);

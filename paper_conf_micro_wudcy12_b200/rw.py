@@ -47,7 +47,7 @@ class rw_plan_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("cuda_stream", ctypes.c_void_p), ("fuse", ctypes.c_int32),
                 ("zero_copy_project", ctypes.c_int32), ("stages", ctypes.c_int32),
                 ("ctas_per_sm", ctypes.c_int32), ("strict_overflow", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 8)]
+                ("host_chunk_log2", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
 
 
 class rw_relation_in(ctypes.Structure):
@@ -156,7 +156,7 @@ class Plan:
     def __init__(self, device: int = 0, stream=None, fuse: bool = True, zero_copy_project: bool = False,
                  stages: int = 0, ctas_per_sm: int = 0, strict_overflow: bool = False, defer: int = 0,
                  dbg: int = 0, dbg_ts: int = 0, items: int = 0, variant: int = 0,
-                 gring: int = 0, agg_mode: int = 0):
+                 gring: int = 0, agg_mode: int = 0, host_chunk_log2: int = 0):
         import torch
         if stream is None:
             stream = torch.cuda.current_stream(device)
@@ -168,6 +168,7 @@ class Plan:
         o.zero_copy_project = 1 if zero_copy_project else 0
         o.stages, o.ctas_per_sm = stages, ctas_per_sm
         o.strict_overflow = 1 if strict_overflow else 0
+        o.host_chunk_log2 = host_chunk_log2  # execute_host: 2^this rows per streamed chunk (0 = 2^25)
         o.reserved[0] = defer              # scan kernel store delay in tiles (0 = auto)
         o.reserved[1] = dbg                # diagnostics only (1: no look-back, 2: stream only, 4: timestamps)
         o.reserved[2] = ctypes.c_int32(dbg_ts & 0xffffffff).value
