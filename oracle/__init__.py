@@ -20,6 +20,7 @@ Plan spec (plain data, also consumed by tests/planspec.py for the CUDA side):
      "nodes": [{"id": .., "op": "select", "in": .., "preds": [(col, op, rhs)]},
                {"id": .., "op": "project", "in": .., "exprs": [...], "roots": [...]},
                {"id": .., "op": "join", "left": .., "right": .., "nkey": k},
+               {"id": .., "op": "union" | "intersect" | "difference", "left": .., "right": ..},
                {"id": .., "op": "agg", "in": .., "gcols": [..], "gdomain": [..],
                 "aggs": [("count",) | ("sum", col)]}],
      "out": id}
@@ -97,6 +98,7 @@ def lib():
         _lib.or_project.argtypes = [P(_Rel), ctypes.c_int32, P(_Expr), ctypes.c_int32,
                                     P(ctypes.c_int32), P(_Rel)]
         _lib.or_join.argtypes = [P(_Rel), P(_Rel), ctypes.c_int32, P(_Rel)]
+        _lib.or_setop.argtypes = [P(_Rel), P(_Rel), ctypes.c_int32, P(_Rel)]
         _lib.or_agg.argtypes = [P(_Rel), ctypes.c_int32, P(ctypes.c_int32), P(ctypes.c_int32),
                                 ctypes.c_int32, P(_Agg), P(_Rel)]
         _lib.or_free.argtypes = [P(_Rel)]
@@ -184,6 +186,17 @@ def project(rel: Relation, exprs, roots) -> Relation:
     return _take(out)
 
 
+SETOPS = {"union": 0, "intersect": 1, "difference": 2}
+
+
+def setop(X: Relation, Y: Relation, op: str) -> Relation:
+    """SET UNION / INTERSECTION / DIFFERENCE (Table 1, reading A24): distinct
+    whole tuples, both inputs sorted on every attribute, result ascending."""
+    out = _Rel()
+    _check(lib().or_setop(ctypes.byref(X._c()), ctypes.byref(Y._c()), SETOPS[op], ctypes.byref(out)))
+    return _take(out)
+
+
 def join(L: Relation, R: Relation, nkey: int = 1) -> Relation:
     out = _Rel()
     _check(lib().or_join(ctypes.byref(L._c()), ctypes.byref(R._c()), nkey, ctypes.byref(out)))
@@ -211,6 +224,8 @@ def evaluate(spec: Dict, inputs: Dict[str, Relation], keep_all: bool = False):
             env[nd["id"]] = select(env[nd["in"]], nd["preds"])
         elif op == "project":
             env[nd["id"]] = project(env[nd["in"]], nd["exprs"], nd["roots"])
+        elif op in SETOPS:
+            env[nd["id"]] = setop(env[nd["left"]], env[nd["right"]], op)
         elif op == "join":
             env[nd["id"]] = join(env[nd["left"]], env[nd["right"]], nd.get("nkey", 1))
         elif op == "agg":

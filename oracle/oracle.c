@@ -469,5 +469,100 @@ int or_agg(const orel *in, int32_t ng, const int32_t *gcols, const int32_t *gdom
 }
 
 /* Type helpers exported for the Python wrapper's self-checks. */
+/* ------------------------------------------------------------------------ */
+/* SET UNION / SET INTERSECTION / SET DIFFERENCE — P:69-83 Table 1: a new
+ * relation "consisting of tuples ... present in at least one of the input
+ * relations" (UNION), "present in both" (INTERSECTION), "exist in one input
+ * relation and do not exist in the other" (DIFFERENCE, x minus y).  Reading
+ * A24: membership is of the whole tuple (every attribute; the Table 1 examples
+ * agree), set semantics (reading A3: the result has no duplicate tuples),
+ * both inputs have identical schemas and are sorted on every attribute,
+ * the result is ascending in that order (reading A5).
+ * Plain definition: the distinct tuples of x ++ y in ascending order (a library
+ * sort), each kept according to its membership in x and in y (a library binary
+ * search in each sorted input).                                                */
+/* ------------------------------------------------------------------------ */
+
+enum { OS_UNION = 0, OS_INTERSECT = 1, OS_DIFFERENCE = 2 };
+
+static const orel *g_sort_a, *g_sort_b;   /* qsort context: rows < a->n index a, else b */
+
+static int row_cmp(const orel *A, int64_t i, const orel *B, int64_t j)
+{
+    return key_cmp(A, i, B, j, A->ncols);
+}
+
+static int cat_cmp(const void *pa, const void *pb)
+{
+    int64_t i = *(const int64_t *)pa, j = *(const int64_t *)pb;
+    const orel *A = i < g_sort_a->n ? g_sort_a : g_sort_b;
+    const orel *B = j < g_sort_a->n ? g_sort_a : g_sort_b;
+    int64_t ii = i < g_sort_a->n ? i : i - g_sort_a->n;
+    int64_t jj = j < g_sort_a->n ? j : j - g_sort_a->n;
+    return row_cmp(A, ii, B, jj);
+}
+
+/* is row i of T a tuple of the sorted relation S? */
+static int member(const orel *S, const orel *T, int64_t i)
+{
+    int64_t lo = 0, hi = S->n;
+    while (lo < hi) {
+        int64_t mid = lo + (hi - lo) / 2;
+        int c = row_cmp(S, mid, T, i);
+        if (c == 0) return 1;
+        if (c < 0) lo = mid + 1;
+        else hi = mid;
+    }
+    return 0;
+}
+
+int or_setop(const orel *X, const orel *Y, int32_t op, orel *out)
+{
+    if (op < OS_UNION || op > OS_DIFFERENCE || X->ncols != Y->ncols || X->ncols < 1)
+        return OR_E_ARG;
+    for (int c = 0; c < X->ncols; c++)
+        if (X->types[c] != Y->types[c])
+            return OR_E_TYPE;
+    if (!is_sorted_on_key(X, X->ncols) || !is_sorted_on_key(Y, Y->ncols))
+        return OR_E_UNSORTED;
+    const int64_t n = X->n + Y->n;
+    int64_t *idx = (int64_t *)malloc((size_t)(n > 0 ? n : 1) * sizeof(int64_t));
+    if (!idx)
+        return OR_E_OOM;
+    for (int64_t i = 0; i < n; i++)
+        idx[i] = i;
+    g_sort_a = X;
+    g_sort_b = Y;
+    qsort(idx, (size_t)n, sizeof(int64_t), cat_cmp);
+    /* distinct tuples, ascending; keep per membership */
+    int64_t *keep = (int64_t *)malloc((size_t)(n > 0 ? n : 1) * sizeof(int64_t));
+    if (!keep) {
+        free(idx);
+        return OR_E_OOM;
+    }
+    int64_t m = 0;
+    for (int64_t q = 0; q < n; q++) {
+        if (q > 0 && cat_cmp(&idx[q - 1], &idx[q]) == 0)
+            continue;                                   /* duplicate tuple */
+        const orel *T = idx[q] < X->n ? X : Y;
+        const int64_t r = idx[q] < X->n ? idx[q] : idx[q] - X->n;
+        const int inx = member(X, T, r), iny = member(Y, T, r);
+        const int k = op == OS_UNION ? (inx || iny) : op == OS_INTERSECT ? (inx && iny) : (inx && !iny);
+        if (k)
+            keep[m++] = idx[q];
+    }
+    int rc = alloc_rel(out, m, X->ncols, X->types);
+    if (rc == OR_OK)
+        for (int64_t q = 0; q < m; q++) {
+            const orel *T = keep[q] < X->n ? X : Y;
+            const int64_t r = keep[q] < X->n ? keep[q] : keep[q] - X->n;
+            for (int c = 0; c < X->ncols; c++)
+                put_value(out, c, q, get_value(T, c, r));
+        }
+    free(idx);
+    free(keep);
+    return rc;
+}
+
 int or_type_width(int t) { return type_width(t); }
 int or_type_signed(int t) { return type_signed(t); }
