@@ -35,6 +35,7 @@ CONFIGS = {
     "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
     "cd": dict(name="Pattern (d) input dependence: 2 SELECTs (25% each) sharing one input of 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
+    "cs": dict(name="Set operator (--setop, default UNION) of two sorted 2^26-tuple (u32 key, u32 val) relations", rows=1 << 26),
     "c5": dict(name="C5: JOIN->JOIN->SELECT over three relations, 2^27 rows each per GPU (2^30 at 8 GPUs), key-range sharded", rows=1 << 27),
 }
 
@@ -47,6 +48,7 @@ def parse():
     ap.add_argument("--impl", default="rw", choices=["rw", "reference"])
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--branches", type=int, default=2, help="cd: SELECTs sharing the input (2..4)")
+    ap.add_argument("--setop", default="union", choices=["union", "intersect", "difference"])
     ap.add_argument("--rows", type=int, default=0, help="override rows per GPU (testing)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-unfused", action="store_true")
@@ -80,6 +82,8 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
         return workloads.c4_spec(), workloads.c4_inputs(rows, start, device)
     if cfg == "cd":
         return workloads.cd_spec(0.25, BRANCHES), workloads.cd_inputs(rows, start, device)
+    if cfg == "cs":
+        return workloads.cs_spec(SETOP), workloads.cs_inputs(rows, device=device)
     if cfg == "c5":
         world = int(os.environ.get("WORLD_SIZE", "1"))
         return workloads.c5_spec(), workloads.c5_inputs(rows, key_space=rows * world, start=start, device=device)
@@ -87,6 +91,7 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
 
 
 BRANCHES = 2
+SETOP = "union"
 
 
 def spec_rows(spec, ins):
@@ -191,7 +196,7 @@ def run_reference(args):
         return 0
     cfg = args.config
     rows = args.rows or CONFIGS[cfg]["rows"]
-    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24}[cfg]
+    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24, "cs": 1 << 21}[cfg]
     import oracle
     oracle.build()
     vals = []
@@ -216,8 +221,9 @@ def run_reference(args):
 
 def main():
     args = parse()
-    global BRANCHES
+    global BRANCHES, SETOP
     BRANCHES = args.branches
+    SETOP = args.setop
     if args.impl == "reference":
         return run_reference(args)
     import torch
@@ -255,7 +261,7 @@ def main():
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
         if cfg == "c3":
             cap = 400_000_000 if rows == workloads.C3_ROWS else 8 * rows + 1024
-        if cfg == "c5":
+        if cfg in ("c5", "cs"):
             cap = 2 * max(nrows.values()) + 4096
         outs = [torch.empty(cap, dtype=dtn[t], device=dev) for t in out_types]
         return plan, ids, outs, cap, out_types
@@ -354,7 +360,8 @@ def main():
     peak, peak_src = measured_peak()
     kern_ms = statistics.mean(per)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
-    kname = {"c3": "k_join_runs + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand"}.get(cfg, "k_scan_chain")
+    kname = {"c3": "k_join_runs + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand",
+             "cs": "k_set_splits + k_set_op x2 + k_set_scan"}.get(cfg, "k_scan_chain")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": ncu_traffic(cfg), "kernel": kname,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
@@ -364,7 +371,7 @@ def main():
     par = {"c5": f"key-range shard x{world} (all_to_all)", "c4": f"row-shard x{world} + limb all-reduce"}
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5") else "i32"),
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs") else "i32"),
             "data": "synthetic (rwgen seeded SplitMix64 generators, generated on device)",
             "config": {"workload": CONFIGS[cfg]["name"], "rows_per_gpu": nrows, "output_rows_per_gpu": n_out,
                        "parallelism": par.get(cfg, f"row-shard x{world}"),
@@ -415,7 +422,7 @@ def main():
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:
-        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26}[cfg]
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26, "cs": 1 << 22}[cfg]
         v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
         line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
                                 "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}

@@ -60,6 +60,9 @@ typedef enum { RW_COL = 0, RW_CONST = 1, RW_ADD = 2, RW_SUB = 3, RW_MUL = 4, RW_
 
 typedef enum { RW_COUNT = 0, RW_SUM = 1 } rw_agg_op;
 
+/* Set operators (Table 1). */
+typedef enum { RW_UNION = 0, RW_INTERSECT = 1, RW_DIFFERENCE = 2 } rw_setop;
+
 /* One SELECT atom: (col OP rhs).  rhs = column rhs_col (same type as col, else
  * RW_E_TYPE) when rhs_is_col, else rhs_const reduced mod 2^w into col's type. */
 typedef struct {
@@ -154,6 +157,16 @@ rw_status rw_plan_add_project(rw_plan *plan, int32_t in, const rw_expr *e, int32
  * identical key types (RW_E_TYPE).  Output schema = (key, left non-key..., right
  * non-key...), rows ordered by (key, left row, right row) (A5). */
 rw_status rw_plan_add_join(rw_plan *plan, int32_t left, int32_t right, int32_t nkey, int32_t *node);
+
+/* SET UNION / SET INTERSECTION / SET DIFFERENCE (Table 1; reading A24):
+ * membership of whole tuples, set semantics (the result has no duplicate tuple even
+ * if an input has), RW_DIFFERENCE = left minus right.  Both inputs need identical
+ * schemas (RW_E_TYPE) of at most 4 columns (RW_E_UNSUPPORTED) and must be sorted on
+ * every column, lexicographically in the declared signedness (nkey_sorted == ncols,
+ * else RW_E_UNSORTED).  Output: same schema, ascending, sorted on every column.
+ * Runs as a merge-path kernel over the materialised inputs; a
+ * downstream SELECT / PROJECT scans its output. */
+rw_status rw_plan_add_setop(rw_plan *plan, int32_t left, int32_t right, int32_t op, int32_t *node);
 
 /* Group-by aggregate (§2.2, §5.2 Q1; A10-A12): group columns are dense
  * codes 0 <= v < gdomain[c] (prod of domains <= 4096, else RW_E_UNSUPPORTED).  Output:

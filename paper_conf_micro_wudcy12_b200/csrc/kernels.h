@@ -49,6 +49,23 @@ struct JoinExpand {
     int16_t dst_slot[kMaxSlots];
 };
 
+// set operators (setops.cu): inputs sorted on every column, identical schemas
+constexpr int kMaxSetCols = 4;
+struct SetLaunch {
+    int32_t ncols;
+    int32_t op;                      // 0 UNION, 1 INTERSECT, 2 DIFFERENCE (x - y)
+    uint8_t types[kMaxSetCols];
+    const void *x[kMaxSetCols], *y[kMaxSetCols];
+    void *out[kMaxSetCols];
+    int64_t nx, ny, nparts, cap;
+    int64_t *split;                  // nparts + 1 merge-path splits
+    uint64_t *pcount;                // per-partition emitted rows, then exclusive offsets
+    int64_t *total;                  // device row count of the result
+};
+size_t set_op_smem(int ncols);
+int set_partition_rows();
+cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st);   // 4 launches
+
 size_t scan_ctl_bytes();
 size_t join_run_cache_bytes();
 int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs

@@ -15,7 +15,7 @@ struct Interval {
     i128 lo, hi;
 };
 
-enum NodeKind { N_INPUT = 0, N_SELECT = 1, N_PROJECT = 2, N_JOIN = 3, N_AGG = 4 };
+enum NodeKind { N_INPUT = 0, N_SELECT = 1, N_PROJECT = 2, N_JOIN = 3, N_AGG = 4, N_SETOP = 5 };
 
 struct Node {
     NodeKind kind;
@@ -28,6 +28,7 @@ struct Node {
     std::vector<rw_expr> exprs;      // N_PROJECT
     std::vector<int> roots;
     int nkey = 0;                    // N_JOIN
+    int setop = 0;                   // N_SETOP: RW_UNION / RW_INTERSECT / RW_DIFFERENCE
     std::vector<int> gcols, gdomain; // N_AGG
     std::vector<rw_agg> aggs;
     int D = 1;
@@ -38,11 +39,11 @@ enum DepClass { DEP_THREAD = 0, DEP_CTA = 1, DEP_KERNEL = 2 };
 const char *dep_name(int d);
 
 // A fused group: one kernel template instance (plus its helper launches).
-enum GroupKind { G_SCAN = 0, G_JOIN = 1 };
+enum GroupKind { G_SCAN = 0, G_JOIN = 1, G_SET = 2 };
 struct Group {
     GroupKind kind;
     int source = -1;                 // G_SCAN: producer node whose relation is scanned
-    int join = -1;                   // G_JOIN: the JOIN node
+    int join = -1;                   // G_JOIN: the JOIN node; G_SET: the set-operator node
     std::vector<int> chain;          // SELECT / PROJECT nodes fused after the source / join
     // input-dependence fusion (§4.4, Fig. 14(d)): several chains over the same
     // G_SCAN source, one output each (chain unused when non-empty)

@@ -320,6 +320,16 @@ int make_group(const rw_plan *p, int id, Grouping &G)
             return G.produced_by[id] = (int)G.groups.size() - 1;
         }
     }
+    if (n.kind == N_SETOP) {
+        // set operators read both (materialised, fully sorted) inputs by merge path
+        g.kind = G_SET;
+        g.join = id;
+        int a = dep_group(p, n.left, G), b = dep_group(p, n.right, G);
+        if (a >= 0) g.deps.push_back(a);
+        if (b >= 0) g.deps.push_back(b);
+        G.groups.push_back(g);
+        return G.produced_by[id] = (int)G.groups.size() - 1;
+    }
     if (n.kind == N_JOIN) {
         g.kind = G_JOIN;
         g.join = id;
@@ -402,6 +412,8 @@ int classify_edge(const rw_plan *p, int prod, int cons)
         return a.nkey_sorted >= b.nkey ? DEP_CTA : DEP_KERNEL;   // Fig. 8(b); unsorted -> SORT boundary
     if (b.kind == N_AGG)
         return DEP_CTA;                          // block reduction + one global atomic stage
+    if (b.kind == N_SETOP)
+        return a.nkey_sorted >= (int)a.types.size() ? DEP_CTA : DEP_KERNEL;   // merge path over whole tuples
     return DEP_KERNEL;
 }
 
@@ -1186,6 +1198,30 @@ void run_group(ExecCtx &X, int gi)
             cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
             p->launches++;
         }
+    } else if (g.kind == G_SET) {
+        const Node &sn = p->nodes[g.join];
+        Rel xr = rel_of(X, sn.left), yr = rel_of(X, sn.right);
+        const int64_t nx = host_count(X, xr), ny = host_count(X, yr);
+        const int64_t cap = sn.setop == RW_UNION ? nx + ny : sn.setop == RW_INTERSECT ? std::min(nx, ny) : nx;
+        make_output(X, gi, outn.types, cap, o, outp, capacity, n_dev);
+        SetLaunch S{};
+        S.ncols = (int)sn.types.size();
+        S.op = sn.setop == RW_UNION ? 0 : sn.setop == RW_INTERSECT ? 1 : 2;
+        for (int c = 0; c < S.ncols; c++) {
+            S.types[c] = (uint8_t)sn.types[c];
+            S.x[c] = xr.cols[c];
+            S.y[c] = yr.cols[c];
+            S.out[c] = outp[c];
+        }
+        S.nx = nx;
+        S.ny = ny;
+        S.nparts = (nx + ny + set_partition_rows() - 1) / set_partition_rows();
+        S.cap = capacity;
+        S.split = (int64_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 8);
+        S.pcount = (uint64_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 8);
+        S.total = n_dev;
+        cuda_check(set_op_launch(S, p->sms, p->stream), "k_set_op");
+        p->launches += S.nparts > 0 ? 4 : 2;
     } else {
         const Node &jn = p->nodes[g.join];
         Rel lr = rel_of(X, jn.left), rr = rel_of(X, jn.right);
@@ -1609,7 +1645,7 @@ std::string explain(rw_plan *p, int out_node)
 {
     node_at(p, out_node);
     std::ostringstream s;
-    static const char *kn[] = {"INPUT", "SELECT", "PROJECT", "JOIN", "AGG"};
+    static const char *kn[] = {"INPUT", "SELECT", "PROJECT", "JOIN", "AGG", "SETOP"};
     Grouping G = build_groups(p, out_node);
     s << "plan: " << p->nodes.size() << " nodes, output node " << out_node << ", fuse=" << p->o.fuse << "\n";
     s << "edges:\n";
@@ -1640,14 +1676,23 @@ std::string explain(rw_plan *p, int out_node)
     s << "groups:\n";
     for (size_t q = 0; q < G.groups.size(); q++) {
         const Group &g = G.groups[q];
-        s << "  group " << q << ": " << (g.kind == G_SCAN ? "k_scan_chain" : "k_merge_splits+k_join_runs+k_tile_runs+k_scan_chain<join>");
+        s << "  group " << q << ": "
+          << (g.kind == G_SCAN ? "k_scan_chain"
+                               : g.kind == G_SET ? "k_set_splits+k_set_op+k_set_scan+k_set_op<write>"
+                                                 : "k_merge_splits+k_join_runs+k_tile_runs+k_scan_chain<join>");
         if (g.agg >= 0) s << "<agg>+k_agg_finalize";
         s << " nodes [";
         if (g.kind == G_SCAN) s << "src " << g.source;
+        else if (g.kind == G_SET) s << "setop " << g.join;
         else s << "join " << g.join;
         for (int c : g.chain) s << ", " << kn[p->nodes[c].kind] << " " << c;
         if (g.agg >= 0) s << ", AGG " << g.agg;
         s << "] -> node " << g.out;
+        if (g.kind == G_SET) {
+            s << " | merge-path partitions of " << set_partition_rows() << " merged rows, smem "
+              << set_op_smem((int)p->nodes[g.join].types.size()) << " B\n";
+            continue;
+        }
         try {
             Lowered L;
             std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
@@ -1959,6 +2004,41 @@ rw_status rw_plan_add_join(rw_plan *p, int32_t left, int32_t right, int32_t nkey
     if ((int)n.types.size() > kMaxOut)
         raise(RW_E_UNSUPPORTED, "join output wider than 32 columns");
     n.nkey_sorted = nkey;
+    add_node(p, std::move(n), node);
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_plan_add_setop(rw_plan *p, int32_t left, int32_t right, int32_t op, int32_t *node)
+{
+    RW_TRY
+    if (!p)
+        raise(RW_E_ARG, "null plan");
+    const Node &L = node_at(p, left);
+    const Node &R = node_at(p, right);
+    if (op != RW_UNION && op != RW_INTERSECT && op != RW_DIFFERENCE)
+        raise(RW_E_ARG, "bad set operator");
+    if (L.types != R.types)
+        raise(RW_E_TYPE, "set operator inputs need identical schemas");
+    if ((int)L.types.size() > kMaxSetCols)
+        raise(RW_E_UNSUPPORTED, "set operators take at most 4 columns");
+    if (L.nkey_sorted < (int)L.types.size() || R.nkey_sorted < (int)R.types.size())
+        raise(RW_E_UNSORTED, "set operator inputs must be sorted on every column");
+    Node n;
+    n.kind = N_SETOP;
+    n.left = left;
+    n.right = right;
+    n.setop = op;
+    n.types = L.types;
+    for (size_t c = 0; c < L.types.size(); c++) {
+        Interval b = L.bounds[c];
+        if (op == RW_UNION) {
+            b.lo = std::min(b.lo, R.bounds[c].lo);
+            b.hi = std::max(b.hi, R.bounds[c].hi);
+        }
+        n.bounds.push_back(b);
+    }
+    n.nkey_sorted = (int)n.types.size();
     add_node(p, std::move(n), node);
     return RW_OK;
     RW_CATCH

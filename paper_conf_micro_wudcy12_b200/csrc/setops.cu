@@ -1,0 +1,277 @@
+// setops.cu — SET UNION / SET INTERSECTION / SET DIFFERENCE (Table 1,
+// reading A24: whole-tuple membership, set semantics, inputs sorted on every
+// attribute, ascending output) on the merge-path machinery of the JOIN
+// (§4.3.3 sizes the INTERSECT output by min(|x|, |y|)).
+//
+// The merged order of x and y (x first on equal tuples, P:196 binary-search
+// partitioning) puts every distinct tuple value into one contiguous segment
+// [its x rows][its y rows].  With pred / succ the merged neighbours of an element e:
+//   UNION      emits e  iff  pred != e                      (first row of each segment)
+//   INTERSECT  emits e  iff  e in y, pred in x, pred == e    (the x->y step of a segment)
+//   DIFFERENCE emits e  iff  e in x, succ != e               (last x row of a segment
+//                                                            that has no y row)
+// so each segment emits at most once and the output is ascending without a sort.
+//   k_set_splits   merge-path split of every partition boundary (2048 merged rows);
+//   k_set_op<0>    per partition: stage both inputs' rows in smem as order-preserving
+//                  u64 keys, merge walk (8 positions per thread), emission flags,
+//                  count per partition;
+//   k_set_scan     exclusive scan of the partition counts (one CTA);
+//   k_set_op<1>    recomputes the flags and writes the emitted tuples at their offsets.
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace rw {
+
+constexpr int kSetItems = 8;
+constexpr int kSetT = kThreads * kSetItems;     // merged rows per partition
+
+// order-preserving 64-bit image of a value (signed types: sign bit flipped)
+__device__ __forceinline__ uint64_t okey(const void *col, int type, int64_t i)
+{
+    switch (type) {
+    case T_I32: return (uint64_t)(((const uint32_t *)col)[i] ^ 0x80000000u);
+    case T_U32: return ((const uint32_t *)col)[i];
+    case T_I64: return ((const uint64_t *)col)[i] ^ 0x8000000000000000ull;
+    case T_U64: return ((const uint64_t *)col)[i];
+    default: return ((const uint8_t *)col)[i];
+    }
+}
+
+__device__ __forceinline__ void store_okey(void *col, int type, int64_t i, uint64_t k)
+{
+    switch (type) {
+    case T_I32: ((uint32_t *)col)[i] = (uint32_t)k ^ 0x80000000u; break;
+    case T_U32: ((uint32_t *)col)[i] = (uint32_t)k; break;
+    case T_I64: ((uint64_t *)col)[i] = k ^ 0x8000000000000000ull; break;
+    case T_U64: ((uint64_t *)col)[i] = k; break;
+    default: ((uint8_t *)col)[i] = (uint8_t)k; break;
+    }
+}
+
+// lexicographic compare of global rows x[i] and y[j]: <0, 0, >0
+__device__ inline int gcmp(const SetLaunch &S, const void *const *a, int64_t i, const void *const *b, int64_t j)
+{
+    for (int c = 0; c < S.ncols; c++) {
+        const uint64_t u = okey(a[c], S.types[c], i), v = okey(b[c], S.types[c], j);
+        if (u != v)
+            return u < v ? -1 : 1;
+    }
+    return 0;
+}
+
+// smem rows: column c of staged row r at s[c * kSetS + r]
+constexpr int kSetS = kSetT + 2;                // + pred and succ slots
+__device__ __forceinline__ int scmp(const uint64_t *s, int nc, int r, int q)
+{
+    for (int c = 0; c < nc; c++) {
+        const uint64_t u = s[c * kSetS + r], v = s[c * kSetS + q];
+        if (u != v)
+            return u < v ? -1 : 1;
+    }
+    return 0;
+}
+
+__global__ void k_set_splits(const __grid_constant__ SetLaunch S)
+{
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p > S.nparts)
+        return;
+    const int64_t d = min(p * kSetT, S.nx + S.ny);
+    int64_t lo = d > S.ny ? d - S.ny : 0, hi = d < S.nx ? d : S.nx;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (gcmp(S, S.x, mid, S.y, d - mid - 1) <= 0)   // x first on equal tuples
+            lo = mid + 1;
+        else
+            hi = mid;
+    }
+    S.split[p] = lo;
+}
+
+template <bool WRITE>
+__global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ SetLaunch S)
+{
+    extern __shared__ __align__(16) uint64_t sm[];
+    uint64_t *s = sm;                                     // ncols * kSetS staged keys
+    int32_t *msrc = (int32_t *)(s + (size_t)S.ncols * kSetS);   // merged position -> staged row
+    __shared__ int32_t wcnt[kThreads / 32 + 1];
+    __shared__ int32_t nbr[4];                            // has_pred, pred_is_x, has_succ, succ_is_x
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int nc = S.ncols;
+    for (int64_t p = blockIdx.x; p < S.nparts; p += gridDim.x) {
+        const int64_t d0 = p * kSetT, d1 = min(d0 + kSetT, S.nx + S.ny);
+        const int64_t i0 = S.split[p], i1 = S.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
+        const int nX = (int)(i1 - i0), nY = (int)(j1 - j0), m = (int)(d1 - d0);
+        __syncthreads();
+        // stage x rows at [0, nX), y rows at [nX, nX + nY), pred at kSetT, succ at kSetT + 1
+        for (int c = 0; c < nc; c++) {
+            for (int r = tid; r < nX; r += kThreads)
+                s[c * kSetS + r] = okey(S.x[c], S.types[c], i0 + r);
+            for (int r = tid; r < nY; r += kThreads)
+                s[c * kSetS + nX + r] = okey(S.y[c], S.types[c], j0 + r);
+        }
+        if (tid == 0) {
+            // merged neighbours outside the partition: pred = the later of x[i0-1], y[j0-1]
+            // (y after x on ties), succ = the earlier of x[i1], y[j1] (x first on ties)
+            const bool px = i0 > 0, py = j0 > 0;
+            bool pis_x = px && (!py || gcmp(S, S.x, i0 - 1, S.y, j0 - 1) > 0);
+            nbr[0] = px || py;
+            nbr[1] = pis_x;
+            if (px || py)
+                for (int c = 0; c < nc; c++)
+                    s[c * kSetS + kSetT] = pis_x ? okey(S.x[c], S.types[c], i0 - 1) : okey(S.y[c], S.types[c], j0 - 1);
+            const bool sx = i1 < S.nx, sy = j1 < S.ny;
+            const bool sis_x = sx && (!sy || gcmp(S, S.x, i1, S.y, j1) <= 0);
+            nbr[2] = sx || sy;
+            nbr[3] = sis_x;
+            if (sx || sy)
+                for (int c = 0; c < nc; c++)
+                    s[c * kSetS + kSetT + 1] = sis_x ? okey(S.x[c], S.types[c], i1) : okey(S.y[c], S.types[c], j1);
+        }
+        __syncthreads();
+        // merge walk: thread positions [dt, dt + 8) of the partition's merged order
+        const int dt = tid * kSetItems;
+        if (dt < m) {
+            int lo = dt > nY ? dt - nY : 0, hi = dt < nX ? dt : nX;
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (scmp(s, nc, mid, nX + dt - mid - 1) <= 0) lo = mid + 1;
+                else hi = mid;
+            }
+            int xi = lo, yj = dt - lo;
+#pragma unroll
+            for (int q = 0; q < kSetItems; q++) {
+                if (dt + q < m) {
+                    const bool takex = yj >= nY || (xi < nX && scmp(s, nc, xi, nX + yj) <= 0);
+                    msrc[dt + q] = takex ? xi : nX + yj;
+                    xi += takex ? 1 : 0;
+                    yj += takex ? 0 : 1;
+                }
+            }
+        }
+        __syncthreads();
+        // emission flags (see the header)
+        uint32_t emit = 0;
+        if (dt < m) {
+#pragma unroll
+            for (int q = 0; q < kSetItems; q++) {
+                const int pos = dt + q;
+                if (pos >= m)
+                    break;
+                const int e = msrc[pos];
+                const bool ex = e < nX;
+                bool f;
+                if (S.op == 0) {                     // UNION
+                    const bool hp = pos > 0 || nbr[0];
+                    const int pr = pos > 0 ? msrc[pos - 1] : kSetT;
+                    f = !(hp && scmp(s, nc, pr, e) == 0);
+                } else if (S.op == 1) {              // INTERSECT
+                    const bool hp = pos > 0 || nbr[0];
+                    const int pr = pos > 0 ? msrc[pos - 1] : kSetT;
+                    const bool prx = pos > 0 ? (pr < nX) : (nbr[1] != 0);
+                    f = !ex && hp && prx && scmp(s, nc, pr, e) == 0;
+                } else {                             // DIFFERENCE x - y
+                    const bool hs = pos + 1 < m || nbr[2];
+                    const int sc = pos + 1 < m ? msrc[pos + 1] : kSetT + 1;
+                    f = ex && !(hs && scmp(s, nc, sc, e) == 0);
+                }
+                emit |= (uint32_t)f << q;
+            }
+        }
+        // block exclusive scan of the per-thread emission counts (thread order = merged order)
+        const int cnt = __popc(emit);
+        int inc = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += y;
+        }
+        if (lane == 31)
+            wcnt[warp] = inc;
+        __syncthreads();
+        int base = 0, tot = 0;
+        for (int w = 0; w < kThreads / 32; w++) {
+            if (w < warp) base += wcnt[w];
+            tot += wcnt[w];
+        }
+        base += inc - cnt;
+        if (!WRITE) {
+            if (tid == 0)
+                S.pcount[p] = (uint64_t)tot;
+            continue;
+        }
+        int64_t o = (int64_t)S.pcount[p] + base;
+        for (uint32_t em = emit; em; em &= em - 1) {
+            const int q = __ffs(em) - 1;
+            const int e = msrc[dt + q];
+            if (o < S.cap)
+                for (int c = 0; c < nc; c++)
+                    store_okey(S.out[c], S.types[c], o, s[c * kSetS + e]);
+            o++;
+        }
+    }
+}
+
+// exclusive scan of the per-partition counts (one CTA) and the total
+__global__ void __launch_bounds__(1024) k_set_scan(const __grid_constant__ SetLaunch S)
+{
+    __shared__ uint64_t ws[32];
+    __shared__ uint64_t carry;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0)
+        carry = 0;
+    __syncthreads();
+    for (int64_t b0 = 0; b0 < S.nparts; b0 += 1024) {
+        const int64_t p = b0 + tid;
+        const uint64_t v = p < S.nparts ? S.pcount[p] : 0;
+        uint64_t x = v;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint64_t y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= d) x += y;
+        }
+        if (lane == 31)
+            ws[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+            uint64_t w = ws[lane];
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint64_t y = __shfl_up_sync(0xffffffffu, w, d);
+                if (lane >= d) w += y;
+            }
+            ws[lane] = w;
+        }
+        __syncthreads();
+        if (p < S.nparts)
+            S.pcount[p] = carry + (warp ? ws[warp - 1] : 0) + x - v;
+        __syncthreads();
+        if (tid == 0)
+            carry += ws[31];
+        __syncthreads();
+    }
+    if (tid == 0)
+        *S.total = (int64_t)carry;
+}
+
+size_t set_op_smem(int ncols) { return (size_t)ncols * kSetS * 8 + (size_t)kSetT * 4; }
+int set_partition_rows() { return kSetT; }
+
+cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st)
+{
+    const size_t smem = set_op_smem(S.ncols);
+    k_set_splits<<<(unsigned)((S.nparts + 1 + 255) / 256), 256, 0, st>>>(S);
+    cudaFuncSetAttribute(k_set_op<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_set_op<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_set_op<true>, kThreads, smem);
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(S.nparts, (int64_t)sms * std::max(occ, 1)));
+    if (S.nparts > 0)
+        k_set_op<false><<<grid, kThreads, smem, st>>>(S);
+    k_set_scan<<<1, 1024, 0, st>>>(S);
+    if (S.nparts > 0)
+        k_set_op<true><<<grid, kThreads, smem, st>>>(S);
+    return cudaGetLastError();
+}
+
+}  // namespace rw

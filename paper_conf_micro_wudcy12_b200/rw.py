@@ -16,6 +16,7 @@ TYPES = {"i32": 0, "u32": 1, "i64": 2, "u64": 3, "u8": 4}
 TYPE_NAMES = {v: k for k, v in TYPES.items()}
 WIDTH = {"i32": 4, "u32": 4, "i64": 8, "u64": 8, "u8": 1}
 CMP = {"<": 0, "<=": 1, ">": 2, ">=": 3, "==": 4, "!=": 5}
+SETOPS = {"union": 0, "intersect": 1, "difference": 2}
 EXPR = {"col": 0, "const": 1, "add": 2, "sub": 3, "mul": 4, "divc": 5}
 STATUS = {0: "RW_OK", -1: "RW_E_ARG", -2: "RW_E_TYPE", -3: "RW_E_UNSORTED", -4: "RW_E_OVERFLOW",
           -5: "RW_E_UNSUPPORTED", -6: "RW_E_CAPACITY", -7: "RW_E_OOM", -8: "RW_E_CUDA",
@@ -60,7 +61,7 @@ class rw_relation_out(ctypes.Structure):
 
 
 EXPORTS = ["rw_plan_create", "rw_plan_destroy", "rw_plan_add_input", "rw_plan_add_select",
-           "rw_plan_add_project", "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema",
+           "rw_plan_add_project", "rw_plan_add_join", "rw_plan_add_setop", "rw_plan_add_agg", "rw_plan_node_schema",
            "rw_plan_execute", "rw_plan_execute_multi", "rw_plan_execute_host", "rw_plan_explain", "rw_plan_last_launches",
            "rw_status_str", "rw_last_error", "rw_split_by_splitters", "rw_merge_runs",
            "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]
@@ -85,6 +86,7 @@ def lib():
     L.rw_plan_add_select.argtypes = [vp, i32, P(rw_pred), i32, P(i32)]
     L.rw_plan_add_project.argtypes = [vp, i32, P(rw_expr), i32, P(i32), i32, P(i32)]
     L.rw_plan_add_join.argtypes = [vp, i32, i32, i32, P(i32)]
+    L.rw_plan_add_setop.argtypes = [vp, i32, i32, i32, P(i32)]
     L.rw_plan_add_agg.argtypes = [vp, i32, P(i32), P(i32), i32, P(rw_agg), i32, P(i32)]
     L.rw_plan_node_schema.argtypes = [vp, i32, P(i32), P(i32)]
     L.rw_plan_execute.argtypes = [vp, P(rw_relation_in), i32, i32, P(rw_relation_out)]
@@ -102,7 +104,7 @@ def lib():
     L.rw_plan_agg_export.argtypes = [vp, i32, P(vp), vp, i64, vp]
     L.rw_plan_agg_import.argtypes = [vp, i32, vp, P(rw_relation_out)]
     for f in ["rw_plan_create", "rw_plan_add_input", "rw_plan_add_select", "rw_plan_add_project",
-              "rw_plan_add_join", "rw_plan_add_agg", "rw_plan_node_schema", "rw_plan_execute",
+              "rw_plan_add_join", "rw_plan_add_setop", "rw_plan_add_agg", "rw_plan_node_schema", "rw_plan_execute",
               "rw_plan_execute_host", "rw_plan_execute_multi", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs",
               "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]:
         getattr(L, f).restype = i32
@@ -219,6 +221,12 @@ class Plan:
         node = ctypes.c_int32()
         check(lib().rw_plan_add_join(self.h, left, right, nkey, ctypes.byref(node)))
         return node.value
+
+    def add_setop(self, left: int, right: int, op: str) -> int:
+        """op: "union" | "intersect" | "difference" (left minus right)."""
+        n = ctypes.c_int32()
+        check(lib().rw_plan_add_setop(self.h, left, right, SETOPS[op], ctypes.byref(n)))
+        return n.value
 
     def add_agg(self, in_node: int, gcols, gdomain, aggs) -> int:
         a = (rw_agg * max(1, len(aggs)))()

@@ -166,6 +166,15 @@ def uniform_join_relation(cfg: int, rel: int, start: int, n: int, key_space: int
     return {"key": to_u32_storage(k), "val": to_u32_storage(v)}
 
 
+def setop_relation(cfg: int, rel: int, n: int, key_space: int, nval: int, device="cpu") -> Dict[str, torch.Tensor]:
+    """Set-operator input: key uniform in [0, key_space), val uniform
+    in [0, nval) (small, so whole tuples repeat across relations), sorted by (key, val)."""
+    k = uniform_int(seed_col(cfg, rel, 0), 0, n, 0, key_space - 1, device)
+    v = uniform_int(seed_col(cfg, rel, 1), 0, n, 0, nval - 1, device)
+    k, v = sort_by_key_val(k, v)
+    return {"key": to_u32_storage(k), "val": to_u32_storage(v)}
+
+
 # TPC-H-like lineitem (SURVEY.md §8(d) C4; TPC-H spec §4.2.3 distributions [ext]).
 # Dates are int32 days since 1970-01-01.
 D_1992_01_01 = 8035

@@ -26,6 +26,8 @@ def build_gpu_plan(spec: Dict, **opts):
             ids[nd["id"]] = plan.add_project(ids[nd["in"]], nd["exprs"], nd["roots"])
         elif op == "join":
             ids[nd["id"]] = plan.add_join(ids[nd["left"]], ids[nd["right"]], nd.get("nkey", 1))
+        elif op in ("union", "intersect", "difference"):
+            ids[nd["id"]] = plan.add_setop(ids[nd["left"]], ids[nd["right"]], op)
         elif op == "agg":
             ids[nd["id"]] = plan.add_agg(ids[nd["in"]], nd["gcols"], nd["gdomain"], nd["aggs"])
     return plan, ids

@@ -68,6 +68,22 @@ def cd_inputs(n: int, start: int = 0, device="cpu", cfg: int = 6) -> Dict[str, L
     return {"R": [r[f"c{c}"] for c in range(4)]}
 
 
+# ---- set operators (Table 1) --------------------------
+# x, y: n tuples (u32 key uniform in [0, n), u32 val in [0, 4)), each sorted on both
+# columns; about 22 % of y's distinct tuples also occur in x.
+def cs_spec(op: str = "union") -> Dict:
+    return {"inputs": {"X": {"types": ["u32", "u32"], "nkey_sorted": 2},
+                       "Y": {"types": ["u32", "u32"], "nkey_sorted": 2}},
+            "nodes": [{"id": "s", "op": op, "left": "X", "right": "Y"}], "out": "s"}
+
+
+def cs_inputs(n: int, device="cpu", cfg: int = 7, nval: int = 4, key_space: int = None) -> Dict[str, List]:
+    ks = key_space or max(n, 1)
+    X = rwgen.setop_relation(cfg, 0, n, ks, nval, device)
+    Y = rwgen.setop_relation(cfg, 1, n, ks, nval, device)
+    return {"X": [X["key"], X["val"]], "Y": [Y["key"], Y["val"]]}
+
+
 # ---- C3: JOIN (Zipf 0.5) -> SELECT -> PROJECT ---------------------------------
 def c3_spec() -> Dict:
     return {"inputs": {"L": {"types": ["u32", "u32"], "nkey_sorted": 1},
