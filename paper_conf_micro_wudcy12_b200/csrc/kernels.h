@@ -59,6 +59,7 @@ struct SetLaunch {
     void *out[kMaxSetCols];
     int64_t nx, ny, nparts, cap;
     int64_t *split;                  // nparts + 1 merge-path splits
+    int32_t *nbr;                    // per split: has_pred | pred_is_x << 1 | has_succ << 2 | succ_is_x << 3
     uint64_t *pcount;                // per-partition emitted rows, then exclusive offsets
     int64_t *total;                  // device row count of the result
 };

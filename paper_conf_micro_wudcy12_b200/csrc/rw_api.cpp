@@ -1219,6 +1219,7 @@ void run_group(ExecCtx &X, int gi)
         S.cap = capacity;
         S.split = (int64_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 8);
         S.pcount = (uint64_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 8);
+        S.nbr = (int32_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 4);
         S.total = n_dev;
         cuda_check(set_op_launch(S, p->sms, p->stream), "k_set_op");
         p->launches += S.nparts > 0 ? 4 : 2;

@@ -48,6 +48,31 @@ __device__ __forceinline__ void store_okey(void *col, int type, int64_t i, uint6
     }
 }
 
+// Tuples whose columns total <= 8 bytes are staged as ONE packed key: the columns'
+// order-preserving images concatenated, first column most significant, so a tuple
+// compare is a single u64 compare (e.g. (u32 key, u32 val) -> key << 32 | val).
+__device__ __forceinline__ uint64_t pack_row(const SetLaunch &S, const void *const *a, int64_t i)
+{
+    uint64_t k = 0;
+    for (int c = 0; c < S.ncols; c++) {
+        const int w = type_width(S.types[c]);
+        const uint64_t v = okey(a[c], S.types[c], i);
+        const uint64_t img = w == 4 ? (uint64_t)(uint32_t)v : w == 1 ? (v & 0xffu) : v;
+        k = w == 8 ? img : ((k << (8 * w)) | img);
+    }
+    return k;
+}
+
+__device__ __forceinline__ void store_packed(const SetLaunch &S, int64_t o, uint64_t k)
+{
+    for (int c = S.ncols - 1; c >= 0; c--) {
+        const int w = type_width(S.types[c]);
+        const uint64_t v = w == 8 ? k : (k & ((1ull << (8 * w)) - 1));
+        store_okey(S.out[c], S.types[c], o, S.types[c] == T_I32 ? (v & 0xffffffffull) : v);
+        k = w == 8 ? 0 : (k >> (8 * w));
+    }
+}
+
 // lexicographic compare of global rows x[i] and y[j]: <0, 0, >0
 __device__ inline int gcmp(const SetLaunch &S, const void *const *a, int64_t i, const void *const *b, int64_t j)
 {
@@ -61,9 +86,11 @@ __device__ inline int gcmp(const SetLaunch &S, const void *const *a, int64_t i, 
 
 // smem rows: column c of staged row r at s[c * kSetS + r]
 constexpr int kSetS = kSetT + 2;                // + pred and succ slots
-__device__ __forceinline__ int scmp(const uint64_t *s, int nc, int r, int q)
+template <int NC>
+__device__ __forceinline__ int scmp(const uint64_t *s, int r, int q)
 {
-    for (int c = 0; c < nc; c++) {
+#pragma unroll
+    for (int c = 0; c < NC; c++) {
         const uint64_t u = s[c * kSetS + r], v = s[c * kSetS + q];
         if (u != v)
             return u < v ? -1 : 1;
@@ -86,47 +113,64 @@ __global__ void k_set_splits(const __grid_constant__ SetLaunch S)
             hi = mid;
     }
     S.split[p] = lo;
+    // merged neighbours of the boundary: pred = element d-1 (the later of x[lo-1],
+    // y[d-lo-1]; y after x on ties), succ = element d (the earlier of x[lo], y[d-lo])
+    const int64_t j = d - lo;
+    const bool px = lo > 0, py = j > 0, sx = lo < S.nx, sy = j < S.ny;
+    const bool pis_x = px && (!py || gcmp(S, S.x, lo - 1, S.y, j - 1) > 0);
+    const bool sis_x = sx && (!sy || gcmp(S, S.x, lo, S.y, j) <= 0);
+    S.nbr[p] = (int32_t)((px || py) | (pis_x << 1) | ((sx || sy) << 2) | (sis_x << 3));
 }
 
-template <bool WRITE>
+template <int NC, bool WRITE, bool PACKED>
 __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ SetLaunch S)
 {
     extern __shared__ __align__(16) uint64_t sm[];
     uint64_t *s = sm;                                     // ncols * kSetS staged keys
-    int32_t *msrc = (int32_t *)(s + (size_t)S.ncols * kSetS);   // merged position -> staged row
+    int32_t *msrc = (int32_t *)(s + (size_t)NC * kSetS);       // merged position -> staged row
     __shared__ int32_t wcnt[kThreads / 32 + 1];
     __shared__ int32_t nbr[4];                            // has_pred, pred_is_x, has_succ, succ_is_x
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int nc = S.ncols;
+    constexpr int nc = NC;
     for (int64_t p = blockIdx.x; p < S.nparts; p += gridDim.x) {
         const int64_t d0 = p * kSetT, d1 = min(d0 + kSetT, S.nx + S.ny);
         const int64_t i0 = S.split[p], i1 = S.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
         const int nX = (int)(i1 - i0), nY = (int)(j1 - j0), m = (int)(d1 - d0);
         __syncthreads();
         // stage x rows at [0, nX), y rows at [nX, nX + nY), pred at kSetT, succ at kSetT + 1
-        for (int c = 0; c < nc; c++) {
+        if (PACKED) {
             for (int r = tid; r < nX; r += kThreads)
-                s[c * kSetS + r] = okey(S.x[c], S.types[c], i0 + r);
+                s[r] = pack_row(S, S.x, i0 + r);
             for (int r = tid; r < nY; r += kThreads)
-                s[c * kSetS + nX + r] = okey(S.y[c], S.types[c], j0 + r);
+                s[nX + r] = pack_row(S, S.y, j0 + r);
+        } else {
+            for (int c = 0; c < nc; c++) {
+                for (int r = tid; r < nX; r += kThreads)
+                    s[c * kSetS + r] = okey(S.x[c], S.types[c], i0 + r);
+                for (int r = tid; r < nY; r += kThreads)
+                    s[c * kSetS + nX + r] = okey(S.y[c], S.types[c], j0 + r);
+            }
         }
+        // merged neighbours outside the partition (decided by k_set_splits): one
+        // thread per (neighbour, column) stages them
+        const int32_t fp = S.nbr[p], fs = S.nbr[p + 1];
         if (tid == 0) {
-            // merged neighbours outside the partition: pred = the later of x[i0-1], y[j0-1]
-            // (y after x on ties), succ = the earlier of x[i1], y[j1] (x first on ties)
-            const bool px = i0 > 0, py = j0 > 0;
-            bool pis_x = px && (!py || gcmp(S, S.x, i0 - 1, S.y, j0 - 1) > 0);
-            nbr[0] = px || py;
-            nbr[1] = pis_x;
-            if (px || py)
-                for (int c = 0; c < nc; c++)
-                    s[c * kSetS + kSetT] = pis_x ? okey(S.x[c], S.types[c], i0 - 1) : okey(S.y[c], S.types[c], j0 - 1);
-            const bool sx = i1 < S.nx, sy = j1 < S.ny;
-            const bool sis_x = sx && (!sy || gcmp(S, S.x, i1, S.y, j1) <= 0);
-            nbr[2] = sx || sy;
-            nbr[3] = sis_x;
-            if (sx || sy)
-                for (int c = 0; c < nc; c++)
-                    s[c * kSetS + kSetT + 1] = sis_x ? okey(S.x[c], S.types[c], i1) : okey(S.y[c], S.types[c], j1);
+            nbr[0] = fp & 1;
+            nbr[1] = (fp >> 1) & 1;
+            nbr[2] = (fs >> 2) & 1;
+            nbr[3] = (fs >> 3) & 1;
+        }
+        if (PACKED) {
+            if (tid == 0 && (fp & 1))
+                s[kSetT] = (fp & 2) ? pack_row(S, S.x, i0 - 1) : pack_row(S, S.y, j0 - 1);
+            else if (tid == 32 && (fs & 4))
+                s[kSetT + 1] = (fs & 8) ? pack_row(S, S.x, i1) : pack_row(S, S.y, j1);
+        } else if (tid < nc && (fp & 1)) {
+            const int c = tid;
+            s[c * kSetS + kSetT] = (fp & 2) ? okey(S.x[c], S.types[c], i0 - 1) : okey(S.y[c], S.types[c], j0 - 1);
+        } else if (tid >= 32 && tid < 32 + nc && (fs & 4)) {
+            const int c = tid - 32;
+            s[c * kSetS + kSetT + 1] = (fs & 8) ? okey(S.x[c], S.types[c], i1) : okey(S.y[c], S.types[c], j1);
         }
         __syncthreads();
         // merge walk: thread positions [dt, dt + 8) of the partition's merged order
@@ -135,14 +179,14 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
             int lo = dt > nY ? dt - nY : 0, hi = dt < nX ? dt : nX;
             while (lo < hi) {
                 const int mid = (lo + hi) >> 1;
-                if (scmp(s, nc, mid, nX + dt - mid - 1) <= 0) lo = mid + 1;
+                if (scmp<NC>(s, mid, nX + dt - mid - 1) <= 0) lo = mid + 1;
                 else hi = mid;
             }
             int xi = lo, yj = dt - lo;
 #pragma unroll
             for (int q = 0; q < kSetItems; q++) {
                 if (dt + q < m) {
-                    const bool takex = yj >= nY || (xi < nX && scmp(s, nc, xi, nX + yj) <= 0);
+                    const bool takex = yj >= nY || (xi < nX && scmp<NC>(s, xi, nX + yj) <= 0);
                     msrc[dt + q] = takex ? xi : nX + yj;
                     xi += takex ? 1 : 0;
                     yj += takex ? 0 : 1;
@@ -164,16 +208,16 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
                 if (S.op == 0) {                     // UNION
                     const bool hp = pos > 0 || nbr[0];
                     const int pr = pos > 0 ? msrc[pos - 1] : kSetT;
-                    f = !(hp && scmp(s, nc, pr, e) == 0);
+                    f = !(hp && scmp<NC>(s, pr, e) == 0);
                 } else if (S.op == 1) {              // INTERSECT
                     const bool hp = pos > 0 || nbr[0];
                     const int pr = pos > 0 ? msrc[pos - 1] : kSetT;
                     const bool prx = pos > 0 ? (pr < nX) : (nbr[1] != 0);
-                    f = !ex && hp && prx && scmp(s, nc, pr, e) == 0;
+                    f = !ex && hp && prx && scmp<NC>(s, pr, e) == 0;
                 } else {                             // DIFFERENCE x - y
                     const bool hs = pos + 1 < m || nbr[2];
                     const int sc = pos + 1 < m ? msrc[pos + 1] : kSetT + 1;
-                    f = ex && !(hs && scmp(s, nc, sc, e) == 0);
+                    f = ex && !(hs && scmp<NC>(s, sc, e) == 0);
                 }
                 emit |= (uint32_t)f << q;
             }
@@ -204,9 +248,13 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
         for (uint32_t em = emit; em; em &= em - 1) {
             const int q = __ffs(em) - 1;
             const int e = msrc[dt + q];
-            if (o < S.cap)
-                for (int c = 0; c < nc; c++)
-                    store_okey(S.out[c], S.types[c], o, s[c * kSetS + e]);
+            if (o < S.cap) {
+                if (PACKED)
+                    store_packed(S, o, s[e]);
+                else
+                    for (int c = 0; c < nc; c++)
+                        store_okey(S.out[c], S.types[c], o, s[c * kSetS + e]);
+            }
             o++;
         }
     }
@@ -257,20 +305,37 @@ __global__ void __launch_bounds__(1024) k_set_scan(const __grid_constant__ SetLa
 size_t set_op_smem(int ncols) { return (size_t)ncols * kSetS * 8 + (size_t)kSetT * 4; }
 int set_partition_rows() { return kSetT; }
 
-cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st)
+template <int NC, bool PACKED>
+static void set_passes(const SetLaunch &S, int sms, cudaStream_t st)
 {
-    const size_t smem = set_op_smem(S.ncols);
-    k_set_splits<<<(unsigned)((S.nparts + 1 + 255) / 256), 256, 0, st>>>(S);
-    cudaFuncSetAttribute(k_set_op<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(k_set_op<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = set_op_smem(NC);
+    cudaFuncSetAttribute(k_set_op<NC, false, PACKED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k_set_op<NC, true, PACKED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_set_op<true>, kThreads, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_set_op<NC, true, PACKED>, kThreads, smem);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(S.nparts, (int64_t)sms * std::max(occ, 1)));
     if (S.nparts > 0)
-        k_set_op<false><<<grid, kThreads, smem, st>>>(S);
+        k_set_op<NC, false, PACKED><<<grid, kThreads, smem, st>>>(S);
     k_set_scan<<<1, 1024, 0, st>>>(S);
     if (S.nparts > 0)
-        k_set_op<true><<<grid, kThreads, smem, st>>>(S);
+        k_set_op<NC, true, PACKED><<<grid, kThreads, smem, st>>>(S);
+}
+
+cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st)
+{
+    k_set_splits<<<(unsigned)((S.nparts + 1 + 255) / 256), 256, 0, st>>>(S);
+    int bytes = 0;
+    for (int c = 0; c < S.ncols; c++)
+        bytes += type_width(S.types[c]);
+    if (bytes <= 8) {
+        set_passes<1, true>(S, sms, st);      // one packed u64 per tuple
+        return cudaGetLastError();
+    }
+    switch (S.ncols) {
+    case 2: set_passes<2, false>(S, sms, st); break;
+    case 3: set_passes<3, false>(S, sms, st); break;
+    default: set_passes<4, false>(S, sms, st); break;
+    }
     return cudaGetLastError();
 }
 
