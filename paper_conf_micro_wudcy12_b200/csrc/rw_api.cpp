@@ -922,13 +922,13 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         vars.push_back({256, 5});
     }
     vars.push_back({256, 4});
-    // register terminal: 14 compute warps per SM by default (the aggregate kernel has
+    // register terminal: 15 compute warps per SM by default (the aggregate kernel has
     // no writer warps, so its register file takes more compute threads; measured C4
-    // 8.56 ms at 256 x 8, 7.43 ms at 384 x 5, 7.06 ms at 448 x 4); opts.reserved[4]:
-    // 1 = the 256-thread variants, 4 = 384 x 5
+    // 8.56 ms at 256 x 8, 7.43 ms at 384 x 5, 7.06 ms at 448 x 4, 6.52 ms at 480 x 4);
+    // opts.reserved[4]: 1 = the 256-thread variants, 4 = 384 x 5, 5 = 448 x 4
     if (L.agg && agg_mode_for(256) == 2 && p->o.reserved[4] != 1) {
         vars.clear();
-        vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : Var{448, 4});
+        vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : p->o.reserved[4] == 5 ? Var{448, 4} : Var{480, 4});
     }
     if (force_items > 0) {
         std::vector<Var> v2;
