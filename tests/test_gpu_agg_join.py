@@ -165,3 +165,17 @@ def test_join_then_aggregate():
     ins = workloads.c3_inputs(20_000, device=DEV, cfg=0x95)
     got, _ = run_gpu(spec, ins, capacity=1)
     assert_same(got, run_oracle(spec, ins))
+
+
+def test_pattern_c_selects_upstream_of_join():
+    """Fig. 14(c) shape: SELECTs on both JOIN inputs, then the join and a
+    downstream SELECT + PROJECT.  The upstream SELECTs keep key order (their outputs
+    stay join-able); they run as their own materialised groups (N2 not fused)."""
+    spec = workloads.c3_spec()
+    spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(1, "<", workloads.thr_u32(0.6))]},
+                     {"id": "fr", "op": "select", "in": "R", "preds": [(1, ">=", workloads.thr_u32(0.3))]},
+                     {"id": "j", "op": "join", "left": "fl", "right": "fr", "nkey": 1}] + spec["nodes"][1:]
+    ins = workloads.c3_inputs(30_000, device=DEV, cfg=0x96)
+    got, plan = run_gpu(spec, ins, capacity=400_000)
+    assert_same(got, run_oracle(spec, ins))
+    assert "materialised" in plan.explain(plan.out_id)
