@@ -7,4 +7,4 @@ timeout 1500 python -m pytest tests -m gpu -q --timeout 300 ${PYTEST_ARGS} > gpu
 for c in ${CONFIGS:-c2 c1 c3 c4 c5}; do
   timeout 600 python bench.py --config $c ${BENCH_ARGS} > gpurun_out/bench_$c.log 2>&1; echo "bench $c rc=$?" >> gpurun_out/bench_$c.log
 done
-tail -3 gpurun_out/smoke.log gpurun_out/pytest_gpu.log gpurun_out/bench_*.log
+for f in gpurun_out/smoke.log gpurun_out/pytest_gpu.log gpurun_out/bench_*.log; do tail -n 3 $f; done
