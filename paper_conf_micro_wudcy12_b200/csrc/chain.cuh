@@ -32,7 +32,7 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v)
 }
 
 __device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_t agg, uint32_t epoch,
-                                         bool aggregate_published = false)
+                                         bool aggregate_published = false, uint32_t max_backoff = 1024)
 {
     const int lane = threadIdx.x & 31;
     const uint64_t tag = (uint64_t)epoch << 48;
@@ -63,8 +63,9 @@ __device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_
         while (pending) {
             // back off: hundreds of look-back warps polling the same few status
             // lines would otherwise starve the stores that publish them
-            __nanosleep(backoff);
-            backoff = backoff < 1024 ? backoff * 2 : 1024;
+            if (max_backoff)
+                __nanosleep(backoff);
+            backoff = backoff < max_backoff ? backoff * 2 : max_backoff;
 #pragma unroll
             for (int q = 0; q < Q; q++) {
                 if ((pending >> q) & 1u) {

@@ -99,10 +99,43 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
     const int64_t lim = cap - base;
     const uint32_t m = (int64_t)total < lim ? total : (lim > 0 ? (uint32_t)lim : 0u);
     T *d = dst + base;
-    uint32_t j = q;
-    // several loads in flight per lane: the ring is read from L2 (~0.5 us per round
-    // trip); phase timestamps showed a writer warp needing 6.4 us per compacted C2 tile
-    constexpr int U = sizeof(T) >= 8 ? 4 : 8;
+    uint32_t j0 = 0;
+    if (sizeof(T) >= 4) {
+        // 16-byte loads from the (16-byte aligned) ring block, U in flight per lane:
+        // the ring is read from L2 (~0.5-1 us per round trip) and phase stamps showed
+        // the scalar copy (8 loads in flight) taking 5.4 us per 6 KB C2 block, which
+        // backed up the compute warps' ring reservations.  Destination offsets are
+        // arbitrary, so the stores stay element-wide.
+        constexpr int V = 16 / sizeof(T);
+        constexpr int U = 4;
+        const uint4 *s4 = (const uint4 *)src;
+        const uint32_t nv = m / V;
+        uint32_t j = q;
+        for (; j + (U - 1) * nq < nv; j += U * nq) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; u++)
+                v[u] = ld_ring(s4 + j + u * nq, gring);
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const T *e = (const T *)&v[u];
+#pragma unroll
+                for (int x = 0; x < V; x++)
+                    d[(size_t)(j + u * nq) * V + x] = e[x];
+            }
+        }
+        for (; j < nv; j += nq) {
+            const uint4 v = ld_ring(s4 + j, gring);
+            const T *e = (const T *)&v;
+#pragma unroll
+            for (int x = 0; x < V; x++)
+                d[(size_t)j * V + x] = e[x];
+        }
+        j0 = nv * V;
+    }
+    // byte columns, and the last partial vector
+    constexpr int U = 8;
+    uint32_t j = j0 + q;
     for (; j + (U - 1) * nq < m; j += U * nq) {
         T v[U];
 #pragma unroll
@@ -112,15 +145,8 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
         for (int u = 0; u < U; u++)
             d[j + u * nq] = v[u];
     }
-    if (j < m) {
-        T v[U];
-#pragma unroll
-        for (int u = 0; u < U; u++)
-            if (j + u * nq < m) v[u] = ld_ring(src + j + u * nq, gring);
-#pragma unroll
-        for (int u = 0; u < U; u++)
-            if (j + u * nq < m) d[j + u * nq] = v[u];
-    }
+    for (; j < m; j += nq)
+        d[j] = ld_ring(src + j, gring);
 }
 
 // Join expansion into a tile (§8(a) a8): candidates [t*T, t*T + rows) of the
@@ -290,7 +316,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
             uint32_t eph = 1;                                // parity of the previous use
             for (int64_t i = 0;; ++i) {
                 if (i >= S)
-                    mbar_wait_sleep(&ctl->in[s].empty, eph, 64);
+                    mbar_wait_aux(&ctl->in[s].empty, eph, 64, L.dbg);
                 const int64_t t = (int64_t)atomicAdd(&L.ctrs[0], 1u);
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
@@ -323,7 +349,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
         if (emit) {
             for (int64_t i = wi;; i += kWriterWarps) {
                 const int j = (int)(i % kRingSlots);
-                mbar_wait_sleep(&ctl->blk[j].aggr, (uint32_t)((i / kRingSlots) & 1), 256);
+                mbar_wait_aux(&ctl->blk[j].aggr, (uint32_t)((i / kRingSlots) & 1), 256, L.dbg);
                 const int64_t t = ctl->blk[j].tile;
                 if (t >= ntiles)
                     break;
@@ -333,7 +359,8 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                     L.dbg_ts[12 * t + 5] = globaltimer();
                 const int64_t excl = (L.dbg & 1) ? t * T
                                                   : (int64_t)lookback_warp(L.status + b * L.status_stride, t, total, L.epoch,
-                                                                           /*aggregate_published=*/true);
+                                                                           /*aggregate_published=*/true,
+                                                                           (L.dbg & 128) ? 0u : (L.dbg & 64) ? 256u : (L.dbg & 256) ? 4096u : 1024u);
                 if (lane == 0) {
                     if (L.dbg & 4)
                         L.dbg_ts[12 * t + 3] = globaltimer();
@@ -367,7 +394,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                     if (L.dbg & 4)
                         L.dbg_ts[12 * t + 4] = globaltimer();
                     if (i > 0)   // release ring bytes in tile order
-                        mbar_wait_sleep(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1), 64);
+                        mbar_wait_aux(&ctl->blk[(i - 1) % kRingSlots].oempty, (uint32_t)(((i - 1) / kRingSlots) & 1), 64, L.dbg);
                     // the discards must land in L2 before the bytes can be rewritten
                     if (gring && !(L.dbg & 8))
                         __threadfence();
@@ -622,7 +649,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 }
                 __syncwarp();
                 if (lane == 0) {
-                    if (gring)
+                    if (gring && !(L.dbg & 512))
                         __threadfence_block();
                     if (warp == 0) {
                         ctl->blk[j].tile = t;

@@ -96,6 +96,24 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity, 
         __nanosleep(ns);
 }
 
+// Off-critical-path wait with a selectable policy (diagnostics dbg bits 16 / 32):
+// 0 = fixed nanosleep polls, 16 = suspending try_wait, 32 = nanosleep with
+// exponential backoff (ns .. 32 ns x 2^k, capped at 4 us).
+__device__ __forceinline__ void mbar_wait_aux(uint64_t *bar, uint32_t parity, uint32_t ns, int mode)
+{
+    if (mode & 16) {
+        mbar_wait(bar, parity);
+    } else if (mode & 32) {
+        uint32_t t = ns;
+        while (!mbar_try(bar, parity)) {
+            __nanosleep(t);
+            t = t < 4096 ? t * 2 : 4096;
+        }
+    } else {
+        mbar_wait_sleep(bar, parity, ns);
+    }
+}
+
 // 1-D bulk copy global -> shared, completion signalled on `bar` (complete_tx).
 // dst, src 16-B aligned; bytes a multiple of 16.
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar,

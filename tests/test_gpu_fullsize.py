@@ -108,3 +108,63 @@ def test_c3_full_size_cardinality_and_key_ranges():
         assert_same(got, ref)
         b = int(torch.searchsorted(okey, torch.tensor([hi], device=DEV)).item())
         assert b - a == ref.n
+
+
+def test_pattern_d_full_size_chunks():
+    """Input-dependence fusion (bench config cd) at 2^29 x 4 i32, 2 branches, in the
+    bench launch configuration: per branch the total count vs a torch count of its
+    predicate, and the first / an interior / the last 2^22-row input chunk's
+    survivors compared with the oracle element by element."""
+    import torch
+    n = workloads.C2_ROWS
+    spec = workloads.cd_spec(0.25, 2)
+    ins = workloads.cd_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    nodes = [ids[o] for o in spec["outs"]]
+    cap = n // 2
+    outs = [[torch.empty(cap, dtype=torch.int32, device=DEV) for _ in range(4)] for _ in nodes]
+    ms = plan.execute_multi([(n, ins["R"])], nodes, outs, [cap, cap])
+    R = ins["R"]
+    for b in range(2):
+        keep = R[b] < workloads.thr_i32(0.25)
+        assert ms[b] == int(keep.sum().item())
+        one = {"inputs": spec["inputs"], "nodes": [spec["nodes"][b]], "out": spec["outs"][b]}
+        for a in [0, 91 * CH + 3, n - CH]:
+            e = min(a + CH, n)
+            ref = run_oracle(one, {"R": [c[a:e] for c in R]})
+            off = int(keep[:a].sum().item())
+            got = oracle.Relation(ref.types, [o[off:off + ref.n].cpu().numpy().view(np.int32) for o in outs[b]])
+            assert_same(got, ref)
+
+
+def test_setop_full_size_key_ranges():
+    """Set operators (bench config cs) at 2 x 2^26 tuples: the result restricted to a
+    key range equals the oracle on the inputs restricted to that range (tuples are
+    whole, so ranges of the sorted key split every operator exactly); ranges at the
+    start, the middle and the end.  Row counts vs torch.unique on packed tuples."""
+    import torch
+    n = 1 << 26
+    ins = workloads.cs_inputs(n, device=DEV)
+    X, Y = ins["X"], ins["Y"]
+    px = (X[0].to(torch.int64) & 0xffffffff) * 4 + X[1].to(torch.int64)
+    py = (Y[0].to(torch.int64) & 0xffffffff) * 4 + Y[1].to(torch.int64)
+    ux, uy = torch.unique(px), torch.unique(py)
+    both = torch.isin(ux, uy)
+    expect = {"union": int(torch.unique(torch.cat([ux, uy])).numel()), "intersect": int(both.sum().item()),
+              "difference": int((~both).sum().item())}
+    for op in ("union", "intersect", "difference"):
+        spec = workloads.cs_spec(op)
+        plan, ids = build_gpu_plan(spec)
+        outs = [torch.empty(2 * n, dtype=torch.int32, device=DEV) for _ in range(2)]
+        m = plan.execute([(n, X), (n, Y)], ids["s"], outs, 2 * n)
+        assert m == expect[op]
+        key = outs[0][:m].to(torch.int64) & 0xffffffff
+        for lo, hi in [(0, 1 << 16), (n // 2, n // 2 + (1 << 16)), (n - (1 << 16), n)]:
+            xs = (X[0].to(torch.int64) & 0xffffffff)
+            ys = (Y[0].to(torch.int64) & 0xffffffff)
+            xa, xb = int(torch.searchsorted(xs, lo)), int(torch.searchsorted(xs, hi))
+            ya, yb = int(torch.searchsorted(ys, lo)), int(torch.searchsorted(ys, hi))
+            ref = run_oracle(spec, {"X": [c[xa:xb] for c in X], "Y": [c[ya:yb] for c in Y]})
+            oa, ob = int(torch.searchsorted(key, lo)), int(torch.searchsorted(key, hi))
+            got = oracle.Relation(ref.types, [o[oa:ob].cpu().numpy().view(np.uint32) for o in outs])
+            assert_same(got, ref)
