@@ -1,7 +1,7 @@
 #!/bin/bash
-timeout 900 python -m pytest tests/test_gpu_scan.py tests/test_gpu_multi.py tests/test_gpu_agg_join.py -m gpu -q -x > gpurun_out/pt.log 2>&1; tail -n 2 gpurun_out/pt.log
-for c in c2 cd c3 c1; do
-  timeout 300 python bench.py --config $c --no-cpu --no-e2e --steps 10 > gpurun_out/b.log 2>&1
-  python -c "import json; j=json.loads(open('gpurun_out/b.log').read().strip().splitlines()[-1]); print('$c', round(j['ms_per_step'],3), round(j['roofline']['frac'],3), j.get('unfused',{}).get('speedup_fused_vs_unfused'))" || tail -n 2 gpurun_out/b.log
+for a in "" "--variant 7 --items 6" "" "--variant 7 --items 6"; do
+  for c in c2 cd; do
+  timeout 300 python bench.py --config $c $a --no-cpu --no-e2e --no-unfused --steps 10 > gpurun_out/b.log 2>&1
+  python -c "import json; j=json.loads(open('gpurun_out/b.log').read().strip().splitlines()[-1]); print('$c [$a]', round(j['ms_per_step'],3), round(j['roofline']['frac'],3))" || tail -n 2 gpurun_out/b.log
+  done
 done
-timeout 300 python scripts/phases.py 0 0 0 0 c2 2>&1 | tail -n 1
