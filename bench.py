@@ -35,7 +35,7 @@ CONFIGS = {
     "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
     "cd": dict(name="Pattern (d) input dependence: 2 SELECTs (25% each) sharing one input of 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
-    "cs": dict(name="Set operator (--setop, default UNION) of two sorted 2^26-tuple (u32 key, u32 val) relations", rows=1 << 26),
+    "cs": dict(name="Set operator (--setop, default UNION) of two sorted (u32 key, u32 val) relations, 2^26 tuples each per GPU, key-range sharded", rows=1 << 26),
     "c5": dict(name="C5: JOIN->JOIN->SELECT over three relations, 2^27 rows each per GPU (2^30 at 8 GPUs), key-range sharded", rows=1 << 27),
 }
 
@@ -83,7 +83,8 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
     if cfg == "cd":
         return workloads.cd_spec(0.25, BRANCHES), workloads.cd_inputs(rows, start, device)
     if cfg == "cs":
-        return workloads.cs_spec(SETOP), workloads.cs_inputs(rows, device=device)
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        return workloads.cs_spec(SETOP), workloads.cs_inputs(rows, device=device, key_space=rows * world, start=start)
     if cfg == "c5":
         world = int(os.environ.get("WORLD_SIZE", "1"))
         return workloads.c5_spec(), workloads.c5_inputs(rows, key_space=rows * world, start=start, device=device)
@@ -294,7 +295,7 @@ def main():
                 plan.agg_import(node, limbs, outs, cap, n_dev=n_dev)
                 return plan.last_launches() + 2
             return step
-        if cfg == "c5" and world > 1:
+        if cfg in ("c5", "cs") and world > 1:
             schema = {k: v["types"] for k, v in spec["inputs"].items()}
             backend = rdist.GpuBackend(local)
 
@@ -368,7 +369,8 @@ def main():
                 "note": "achieved = (input bytes + compacted output bytes) / CUDA-event time per step; "
                         "peak = measured copy bandwidth (MEASURED_PEAKS.json hbm_gbs)"}
 
-    par = {"c5": f"key-range shard x{world} (all_to_all)", "c4": f"row-shard x{world} + limb all-reduce"}
+    par = {"c5": f"key-range shard x{world} (all_to_all)", "cs": f"key-range shard x{world} (all_to_all)",
+           "c4": f"row-shard x{world} + limb all-reduce"}
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs") else "i32"),

@@ -166,11 +166,13 @@ def uniform_join_relation(cfg: int, rel: int, start: int, n: int, key_space: int
     return {"key": to_u32_storage(k), "val": to_u32_storage(v)}
 
 
-def setop_relation(cfg: int, rel: int, n: int, key_space: int, nval: int, device="cpu") -> Dict[str, torch.Tensor]:
-    """Set-operator input: key uniform in [0, key_space), val uniform
-    in [0, nval) (small, so whole tuples repeat across relations), sorted by (key, val)."""
-    k = uniform_int(seed_col(cfg, rel, 0), 0, n, 0, key_space - 1, device)
-    v = uniform_int(seed_col(cfg, rel, 1), 0, n, 0, nval - 1, device)
+def setop_relation(cfg: int, rel: int, n: int, key_space: int, nval: int, device="cpu",
+                   start: int = 0) -> Dict[str, torch.Tensor]:
+    """Set-operator input: rows [start, start + n) of a relation with
+    key uniform in [0, key_space), val uniform in [0, nval) (small, so whole tuples
+    repeat across relations), sorted by (key, val)."""
+    k = uniform_int(seed_col(cfg, rel, 0), start, n, 0, key_space - 1, device)
+    v = uniform_int(seed_col(cfg, rel, 1), start, n, 0, nval - 1, device)
     k, v = sort_by_key_val(k, v)
     return {"key": to_u32_storage(k), "val": to_u32_storage(v)}
 

@@ -59,6 +59,13 @@ def _worker(rank, world, port, q):
         res = {"join_rows": [c.tolist() for c in out.cols],
                "ranges": {k: [mine[k][0].min().item() if mine[k][0].numel() else None,
                               mine[k][0].max().item() if mine[k][0].numel() else None] for k in "RST"}}
+        # --- key-range sharded set operators (same exchange as the join) ---
+        ns = 5000
+        ss, ms = rd.row_range(ns, rank, world)
+        lset = workloads.cs_inputs(ms, key_space=ns, start=ss, cfg=0xB3)
+        mset = rd.exchange_all(be, lset, {"X": ["u32", "u32"], "Y": ["u32", "u32"]}, world, samples=64)
+        res["set_rows"] = {op: [c.tolist() for c in run_oracle(workloads.cs_spec(op), mset).cols]
+                           for op in ("union", "intersect", "difference")}
         # --- row-sharded aggregate combined with an int64 SUM all-reduce of limbs ---
         n4 = 20000
         s4, m4 = rd.row_range(n4, rank, world)
@@ -80,7 +87,7 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-def test_world2_gloo_key_range_join_and_aggregate_combine():
+def test_world2_gloo_key_range_join_setops_and_aggregate_combine():
     sys.path.insert(0, ROOT)
     import oracle
     import workloads
@@ -104,6 +111,11 @@ def test_world2_gloo_key_range_join_and_aggregate_combine():
     for c in range(len(ref.types)):
         cat = got[0]["join_rows"][c] + got[1]["join_rows"][c]
         assert cat == ref.cols[c].tolist()
+    # rank-order concatenation of the sharded set operators == single-process result
+    for op in ("union", "intersect", "difference"):
+        ref = run_oracle(workloads.cs_spec(op), workloads.cs_inputs(5000, cfg=0xB3))
+        for c in range(2):
+            assert got[0]["set_rows"][op][c] + got[1]["set_rows"][op][c] == ref.cols[c].tolist(), op
     # all-reduced limbs decode to the single-process aggregate
     assert got[0]["limbs"] == got[1]["limbs"]
     full = run_oracle(workloads.c4_spec(), workloads.c4_inputs(20000, cfg=0xB2))

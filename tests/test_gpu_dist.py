@@ -69,6 +69,37 @@ def test_key_range_sharded_three_way_join_equals_single_gpu(P):
     assert_same(merged, ref)
 
 
+@pytest.mark.parametrize("op", ["union", "intersect", "difference"])
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_key_range_sharded_setop_equals_single_gpu(op, P):
+    """Set operators shard like the JOIN: equal tuples share their key,
+    so after the key-range exchange every rank's result is the global result's slice
+    of its key range; the rank-order concatenation equals the single-GPU result."""
+    import torch
+    from paper_conf_micro_wudcy12_b200 import dist as rd
+    n = 30_000
+    spec = workloads.cs_spec(op)
+    full = workloads.cs_inputs(n, device=DEV, cfg=0xA5)
+    shards = {k: [] for k in "XY"}
+    for r in range(P):
+        s, m = rd.row_range(n, r, P)
+        part = workloads.cs_inputs(m, key_space=n, start=s, device=DEV, cfg=0xA5)
+        for k in "XY":
+            shards[k].append(part[k])
+    backend = rd.GpuBackend(0)
+    allk, _ = torch.sort(torch.cat([rd.key_values(c[0], "u32") for k in "XY" for c in shards[k]]))
+    spl = [int(allk[(allk.numel() * (r + 1)) // P].item()) for r in range(P - 1)]
+    ex = {k: simulated_exchange(backend, shards[k], ["u32", "u32"], spl) for k in "XY"}
+    outs = []
+    for r in range(P):
+        ins = {k: ex[k][r] for k in "XY"}
+        got, _ = run_gpu(spec, ins, capacity=2 * n)
+        outs.append(got)
+    ref = run_oracle(spec, full)
+    merged = oracle.Relation(ref.types, [np.concatenate([o.cols[c] for o in outs]) for c in range(2)])
+    assert_same(merged, ref)
+
+
 def test_split_bounds_and_merge_small():
     import torch
     from paper_conf_micro_wudcy12_b200 import dist as rd

@@ -77,10 +77,12 @@ def cs_spec(op: str = "union") -> Dict:
             "nodes": [{"id": "s", "op": op, "left": "X", "right": "Y"}], "out": "s"}
 
 
-def cs_inputs(n: int, device="cpu", cfg: int = 7, nval: int = 4, key_space: int = None) -> Dict[str, List]:
+def cs_inputs(n: int, device="cpu", cfg: int = 7, nval: int = 4, key_space: int = None,
+              start: int = 0) -> Dict[str, List]:
+    """Rows [start, start + n) of x and y (each returned sorted on both columns)."""
     ks = key_space or max(n, 1)
-    X = rwgen.setop_relation(cfg, 0, n, ks, nval, device)
-    Y = rwgen.setop_relation(cfg, 1, n, ks, nval, device)
+    X = rwgen.setop_relation(cfg, 0, n, ks, nval, device, start)
+    Y = rwgen.setop_relation(cfg, 1, n, ks, nval, device, start)
     return {"X": [X["key"], X["val"]], "Y": [Y["key"], Y["val"]]}
 
 
