@@ -624,7 +624,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 for (int k = 0; k < ITEMS; k++)
                     posk[k] = pre[k] + __popc(bal[k] & lt);
                 uint32_t coff = 0;
-                for (int c = c0; c < c1; c++) {
+                for (int c = c0; c < c1 && !(L.dbg & 1024); c++) {   // dbg 1024: skip the ring stores (ablation)
                     const int w = P.out_w[c];
                     const char *src = loc_ptr(P.out_loc[c], st, scratch);
                     char *dst = blk + coff;
