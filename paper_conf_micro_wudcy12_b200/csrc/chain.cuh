@@ -607,6 +607,7 @@ __device__ inline void agg_tile(const ChainProg &P, const char *stage, const cha
 // the registers into the CTA's 128-bit accumulators.
 struct RegAgg {
     uint64_t s[kRegD][kRegA];
+    uint32_t n[kRegD][kRegA];      // narrow sums (a < P.agg_narrow): 32-bit partials
     uint32_t c[kRegD];
 };
 
@@ -616,8 +617,10 @@ __device__ __forceinline__ void reg_agg_zero(RegAgg &R)
     for (int d = 0; d < kRegD; d++) {
         R.c[d] = 0;
 #pragma unroll
-        for (int a = 0; a < kRegA; a++)
+        for (int a = 0; a < kRegA; a++) {
             R.s[d][a] = 0;
+            R.n[d][a] = 0;
+        }
     }
 }
 
@@ -632,8 +635,9 @@ __device__ inline void reg_agg_flush(const ChainProg &P, RegAgg &R, unsigned lon
 #pragma unroll
             for (int a = 0; a < kRegA; a++) {
                 if (a < P.nagg) {
-                    const unsigned long long v = R.s[d][a];
-                    const unsigned long long hi = (!P.agg_unsigned[a] && (long long)v < 0) ? ~0ull : 0ull;
+                    const bool nar = a < P.agg_narrow;
+                    const unsigned long long v = nar ? (unsigned long long)R.n[d][a] : R.s[d][a];
+                    const unsigned long long hi = (!nar && !P.agg_unsigned[a] && (long long)v < 0) ? ~0ull : 0ull;
                     atomic_add128(&acc[2 * (d * NA + 1 + a)], &acc[2 * (d * NA + 1 + a) + 1], v, hi);
                 }
             }
@@ -654,7 +658,7 @@ __device__ inline void reg_agg_store(const ChainProg &P, const RegAgg &R, unsign
 #pragma unroll
             for (int a = 0; a < kRegA; a++)
                 if (a < P.nagg)
-                    part[(d * NA + 1 + a) * NT + tid] = R.s[d][a];
+                    part[(d * NA + 1 + a) * NT + tid] = a < P.agg_narrow ? (unsigned long long)R.n[d][a] : R.s[d][a];
         }
     }
 }
@@ -662,7 +666,7 @@ __device__ inline void reg_agg_store(const ChainProg &P, const RegAgg &R, unsign
 // Row loop of the register terminal: NAGG sums (W64: every sum column is 64-bit, so
 // no per-row type dispatch); the one-hot over the groups becomes a jump to the
 // row's group, whose partials take predicated-free adds.
-template <int NT, int ITEMS, int NAGG, bool W64>
+template <int NT, int ITEMS, int NAGG, bool W64, int NN = 0>
 __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *at, const uint32_t *g, uint32_t ok,
                                              RegAgg &R)
 {
@@ -680,8 +684,12 @@ __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *a
             if (gk == (uint32_t)d) {
                 R.c[d] += 1u;
 #pragma unroll
-                for (int a = 0; a < NAGG; a++)
-                    R.s[d][a] += v[a];
+                for (int a = 0; a < NAGG; a++) {
+                    if (a < NN)
+                        R.n[d][a] += (uint32_t)v[a];
+                    else
+                        R.s[d][a] += v[a];
+                }
             }
         }
     }
@@ -747,6 +755,23 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
             w64 = false;
     }
     // the sum count and the all-64-bit case are compile-time in the row loop
+    if (NT == kNarrowNT) {
+        // the 544-thread instance is specialised (host-selected) for 5 all-64-bit sums of
+        // which the first 2 are narrow: only this row loop is compiled into it, which is
+        // what lets 17 compute warps fit the register file
+        agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R);
+        return;
+    }
+    if (w64 && P.agg_narrow) {
+        switch (P.nagg * 4 + P.agg_narrow) {
+        case 3 * 4 + 1: agg_rows_reg<NT, ITEMS, 3, true, 1>(ab, at, g, ok, R); return;
+        case 3 * 4 + 2: agg_rows_reg<NT, ITEMS, 3, true, 2>(ab, at, g, ok, R); return;
+        case 4 * 4 + 1: agg_rows_reg<NT, ITEMS, 4, true, 1>(ab, at, g, ok, R); return;
+        case 4 * 4 + 2: agg_rows_reg<NT, ITEMS, 4, true, 2>(ab, at, g, ok, R); return;
+        case 5 * 4 + 1: agg_rows_reg<NT, ITEMS, 5, true, 1>(ab, at, g, ok, R); return;
+        default: agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R); return;
+        }
+    }
     if (w64) {
         switch (P.nagg) {
         case 0: agg_rows_reg<NT, ITEMS, 0, true>(ab, at, g, ok, R); return;

@@ -31,7 +31,8 @@ constexpr int kJoinItems = 9;        // outputs per thread per tile in the join 
 constexpr int kMaxAggSlots = 4096;
 constexpr int kMaxBranch = 4;        // input-dependence fusion: SELECT/PROJECT chains sharing one scan
 constexpr int kRegD = 6;             // register aggregate terminal: groups x sums held per thread
-constexpr int kRegA = 5;   // D * (nagg + 1) upper bound for the agg terminal
+constexpr int kRegA = 5;
+constexpr int kNarrowNT = 544;       // aggregate variant specialised for 5 sums with 2 narrow (TPC-H Q1 shape)   // D * (nagg + 1) upper bound for the agg terminal
 
 enum Type : uint8_t { T_I32 = 0, T_U32 = 1, T_I64 = 2, T_U64 = 3, T_U8 = 4 };
 enum Cmp : uint8_t { C_LT = 0, C_LE = 1, C_GT = 2, C_GE = 3, C_EQ = 4, C_NE = 5 };
@@ -90,6 +91,8 @@ struct ChainProg {
     uint8_t agg_unsigned[kMaxAggs];     // 1: u64 sum (unsigned partials)
     int64_t flush_rows;                 // rows a thread may add before its int64 partials can overflow
     int32_t agg_mode;                   // 0: thread-private partials in smem; 2: register one-hot (D <= kRegD, nagg <= kRegA)
+    int32_t agg_narrow;                 // mode 2: the first agg_narrow sums are non-negative with |v| < 2^16 and
+                                        // accumulate in 32-bit registers (flush_rows keeps them below 2^32)
     // input-dependence fusion (§4.4, Fig. 14(d)): nbranch chains over the same
     // staged tile, each with its own mask and compacted output.  Branch b runs ops
     // [br_op_end[b-1], br_op_end[b]) and writes output columns [br_out_end[b-1], br_out_end[b]).

@@ -1260,6 +1260,7 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         if (nt == 384) return occ(k_scan_chain<384, 5, true, false>, smem, 384 + 32);
         if (nt == 448) return occ(k_scan_chain<448, 4, true, false>, smem, 448 + 32);
         if (nt == 480) return occ(k_scan_chain<480, 4, true, false>, smem, 480 + 32);
+        if (nt == kNarrowNT) return occ(k_scan_chain<kNarrowNT, 4, true, false>, smem, kNarrowNT + 32);
         return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + 32)
                           : occ(k_scan_chain<256, 8, true, false>, smem, 256 + 32);
     case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
@@ -1297,6 +1298,8 @@ cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg,
             return sc<448, 4, true>(P, L, smem, grid, s);
         if (nt == 480)
             return sc<480, 4, true>(P, L, smem, grid, s);
+        if (nt == kNarrowNT)
+            return sc<kNarrowNT, 4, true>(P, L, smem, grid, s);
         return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
     }
     if (nt == 512)

@@ -606,6 +606,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     }   // branches
 
     // terminal
+    int narrow_n = 0;
+    bool narrow_all64 = true;
+    unsigned __int128 narrow_flush = 0;
     if (nbr > 1) {
         // materialising terminals collected per branch above
     } else if (g.agg >= 0) {
@@ -625,8 +628,24 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         // flush period: rows whose |values| sum cannot leave int64 (uint64 for u64 sums)
         unsigned __int128 flush = ((unsigned __int128)1) << 40;
         L.F.nreq = (int)a.aggs.size();
-        for (size_t q = 0; q < a.aggs.size(); q++) {
-            if (a.aggs[q].op == RW_SUM) {
+        // sums whose values are non-negative and below 2^16 ("narrow") are numbered
+        // first: the register terminal accumulates them in 32-bit registers
+        std::vector<size_t> order_q;
+        for (int pass = 0; pass < 2; pass++)
+            for (size_t q = 0; q < a.aggs.size(); q++) {
+                if (a.aggs[q].op != RW_SUM) continue;
+                const Interval b = an.bounds[a.aggs[q].col];
+                const bool nar = b.lo >= 0 && b.hi < 65536;
+                if (nar == (pass == 0)) order_q.push_back(q);
+            }
+        narrow_n = 0;
+        narrow_flush = ((unsigned __int128)1) << 40;
+        for (size_t q = 0; q < a.aggs.size(); q++)
+            if (a.aggs[q].op != RW_SUM) {
+                L.F.req_is_sum[q] = 0;
+                L.F.req_acc[q] = 0;
+            }
+        for (size_t q : order_q) {
                 int s = resolve(cur[a.aggs[q].col]);
                 L.P.agg_slot[ns] = (int16_t)s;
                 const bool uns = slots[s].type == T_U64;
@@ -639,13 +658,14 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 if (mx == 0) mx = 1;
                 unsigned __int128 lim = uns ? (unsigned __int128)UINT64_MAX : (unsigned __int128)INT64_MAX;
                 flush = std::min(flush, std::max<unsigned __int128>(1, lim / mx));
+                narrow_all64 = narrow_all64 && (slots[s].type == T_I64 || slots[s].type == T_U64);
+                if (b.lo >= 0 && b.hi < 65536) {
+                    narrow_n++;
+                    narrow_flush = std::min(narrow_flush, (unsigned __int128)UINT32_MAX / mx);
+                }
                 L.F.req_is_sum[q] = 1;
                 L.F.req_acc[q] = (int16_t)(1 + ns);
                 ns++;
-            } else {
-                L.F.req_is_sum[q] = 0;
-                L.F.req_acc[q] = 0;
-            }
         }
         L.P.nagg = ns;
         L.P.flush_rows = (int64_t)flush;
@@ -928,7 +948,13 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     // opts.reserved[4]: 1 = the 256-thread variants, 4 = 384 x 5, 5 = 448 x 4
     if (L.agg && agg_mode_for(256) == 2 && p->o.reserved[4] != 1) {
         vars.clear();
-        vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : p->o.reserved[4] == 5 ? Var{448, 4} : Var{480, 4});
+        // 5 all-64-bit sums with 2 narrow ones: the specialised 544-thread instance
+        // (32-bit partials for the narrow sums, 17 compute warps); opts.reserved[4] == 6
+        // keeps the generic 480 x 4
+        const bool q1shape = P.nagg == 5 && narrow_n == 2 && narrow_all64 &&
+                             narrow_flush >= (1 << 16) && p->o.reserved[4] == 0;
+        vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : p->o.reserved[4] == 5 ? Var{448, 4}
+                       : q1shape ? Var{kNarrowNT, 4} : Var{480, 4});
     }
     if (force_items > 0) {
         std::vector<Var> v2;
@@ -1012,6 +1038,17 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
     layout(L.tile);
     P.agg_mode = agg_mode_for(L.nt);
+    // 32-bit partials for the narrow sums (register terminal, kernel variants for
+    // (sums, narrow) in {3,4,5} x {1,2}; flush before any could pass 2^32)
+    P.agg_narrow = 0;
+    bool all64 = true;
+    for (int q = 0; q < P.nagg; q++)
+        all64 = all64 && (P.agg_type[q] == T_I64 || P.agg_type[q] == T_U64);
+    if (P.agg_mode == 2 && all64 && narrow_n >= 1 && narrow_n <= 2 && P.nagg >= 3 && P.nagg <= 5 &&
+        p->o.reserved[4] != 1 && narrow_flush >= (1 << 16)) {
+        P.agg_narrow = narrow_n;
+        P.flush_rows = std::min<int64_t>(P.flush_rows, (int64_t)narrow_flush);
+    }
     if (global_ring && !L.direct) {
         size_t W = 0;
         for (int c = 0; c < P.nout; c++)

@@ -31,16 +31,18 @@ def test_q1_both_agg_terminals(agg_mode):
     assert want in plan.explain(plan.out_id)
 
 
-@pytest.mark.parametrize("variant", [4, 5, 1, 0])
+@pytest.mark.parametrize("variant", [4, 5, 1, 6, 0])
 @pytest.mark.parametrize("n", [1, 1919, 1921, 300_001])
 def test_q1_wide_cta_variants(variant, n):
-    """384 x 5 / 448 x 4 / 256 x 8 / 480 x 4 (default) compute threads (aggregate kernels
-    carry no writer warps): tiles of 1920 / 1792 / 2048 / 1920 rows, ragged tails."""
+    """384 x 5 / 448 x 4 / 256 x 8 / 480 x 4 / 544 x 4 (default for Q1's 5 sums with 2
+    narrow ones, 32-bit partials) compute threads (aggregate kernels carry no writer
+    warps): tiles of 1920 / 1792 / 2048 / 1920 / 2176 rows, ragged tails."""
     spec = workloads.c4_spec()
     ins = workloads.c4_inputs(n, device=DEV, cfg=0x94)
     got, plan = run_gpu(spec, ins, capacity=6, variant=variant)
     assert_same(got, run_oracle(spec, ins))
-    assert {4: "tile 1920", 5: "tile 1792", 1: "tile 2048", 0: "tile 1920 rows (4/thread)"}[variant] in plan.explain(plan.out_id)
+    assert {4: "tile 1920", 5: "tile 1792", 1: "tile 2048", 6: "tile 1920 rows (4/thread)",
+            0: "tile 2176 rows (4/thread)"}[variant] in plan.explain(plan.out_id)
 
 
 @pytest.mark.parametrize("lo,hi", [(-1000, 1000), (-(2**40), 2**40), (-(2**63), 2**63 - 1), (5, 5)])
