@@ -663,6 +663,48 @@ __device__ inline void reg_agg_store(const ChainProg &P, const RegAgg &R, unsign
     }
 }
 
+// End of the register terminal: every (group, sum) partial is reduced across the
+// warp exactly in 128 bits (shuffles), then lane 0 adds the warp's total into the
+// CTA's 128-bit accumulators (one shared atomic pair per warp, not per thread).
+__device__ __forceinline__ void warp_sum128(unsigned long long &lo, unsigned long long &hi)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long l2 = __shfl_xor_sync(0xffffffffu, lo, o);
+        const unsigned long long h2 = __shfl_xor_sync(0xffffffffu, hi, o);
+        const unsigned long long nl = lo + l2;
+        hi = hi + h2 + (nl < lo ? 1ull : 0ull);
+        lo = nl;
+    }
+}
+
+__device__ inline void reg_agg_reduce_warp(const ChainProg &P, RegAgg &R, unsigned long long *acc)
+{
+    const int NA = P.nagg + 1;
+    const bool lane0 = (threadIdx.x & 31) == 0;
+#pragma unroll
+    for (int d = 0; d < kRegD; d++) {
+        if (d < P.D) {
+            unsigned long long lo = R.c[d], hi = 0;
+            warp_sum128(lo, hi);
+            if (lane0 && (lo | hi))
+                atomic_add128(&acc[2 * (d * NA)], &acc[2 * (d * NA) + 1], lo, hi);
+#pragma unroll
+            for (int a = 0; a < kRegA; a++) {
+                if (a < P.nagg) {
+                    const bool nar = a < P.agg_narrow;
+                    unsigned long long v = nar ? (unsigned long long)R.n[d][a] : R.s[d][a];
+                    unsigned long long h = (!nar && !P.agg_unsigned[a] && (long long)v < 0) ? ~0ull : 0ull;
+                    warp_sum128(v, h);
+                    if (lane0 && (v | h))
+                        atomic_add128(&acc[2 * (d * NA + 1 + a)], &acc[2 * (d * NA + 1 + a) + 1], v, h);
+                }
+            }
+        }
+    }
+    reg_agg_zero(R);
+}
+
 // Row loop of the register terminal: NAGG sums (W64: every sum column is 64-bit, so
 // no per-row type dispatch); the one-hot over the groups becomes a jump to the
 // row's group, whose partials take predicated-free adds.

@@ -31,8 +31,9 @@ constexpr int kJoinItems = 9;        // outputs per thread per tile in the join 
 constexpr int kMaxAggSlots = 4096;
 constexpr int kMaxBranch = 4;        // input-dependence fusion: SELECT/PROJECT chains sharing one scan
 constexpr int kRegD = 6;             // register aggregate terminal: groups x sums held per thread
-constexpr int kRegA = 5;
-constexpr int kNarrowNT = 544;       // aggregate variant specialised for 5 sums with 2 narrow (TPC-H Q1 shape)   // D * (nagg + 1) upper bound for the agg terminal
+constexpr int kRegA = 5;             // sums held per thread per group
+constexpr int kNarrowNT = 576;       // aggregate variant specialised for 5 sums with 2 narrow (TPC-H Q1 shape)
+constexpr int kNarrowItems = 4;      // rows per thread of that variant (tile 2304)
 
 enum Type : uint8_t { T_I32 = 0, T_U32 = 1, T_I64 = 2, T_U64 = 3, T_U8 = 4 };
 enum Cmp : uint8_t { C_LT = 0, C_LE = 1, C_GT = 2, C_GE = 3, C_EQ = 4, C_NE = 5 };

@@ -439,12 +439,8 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                         mbar_arrive_cnt(&ctl->blk[ju].aggr, NW);
                     }
                 }
-                if (AGG && P.agg_mode == 2) {
-                    // every compute warp is past its last stage (no TMA is pending once the
-                    // sentinel is reached): the stage buffers take the register partials
-                    bar_sync(kComputeBar, NT);
-                    reg_agg_store<NT>(P, racc, (unsigned long long *)stages);
-                }
+                if (AGG && P.agg_mode == 2)
+                    reg_agg_reduce_warp(P, racc, cta_acc);   // warp-reduced, 128-bit exact
                 break;
             }
             char *st = stages + (size_t)s * P.stage_bytes;
@@ -673,8 +669,8 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
     }
     __syncthreads();
     if (AGG) {
-        if (P.agg_mode != 3)      // mode 3 added every row into the global accumulators already
-            agg_combine<NT>(P, P.agg_mode == 2 ? (unsigned long long *)stages : part, cta_acc, blockDim.x);
+        if (P.agg_mode == 0)      // modes 2 / 3 added their rows into cta_acc / the global accumulators already
+            agg_combine<NT>(P, part, cta_acc, blockDim.x);
         __syncthreads();
         for (int qq = tid; qq < P.D * NA; qq += blockDim.x) {
             const unsigned long long lo = cta_acc[2 * qq], hi = cta_acc[2 * qq + 1];
@@ -1260,7 +1256,7 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         if (nt == 384) return occ(k_scan_chain<384, 5, true, false>, smem, 384 + 32);
         if (nt == 448) return occ(k_scan_chain<448, 4, true, false>, smem, 448 + 32);
         if (nt == 480) return occ(k_scan_chain<480, 4, true, false>, smem, 480 + 32);
-        if (nt == kNarrowNT) return occ(k_scan_chain<kNarrowNT, 4, true, false>, smem, kNarrowNT + 32);
+        if (nt == kNarrowNT) return occ(k_scan_chain<kNarrowNT, kNarrowItems, true, false>, smem, kNarrowNT + 32);
         return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + 32)
                           : occ(k_scan_chain<256, 8, true, false>, smem, 256 + 32);
     case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
@@ -1299,7 +1295,7 @@ cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg,
         if (nt == 480)
             return sc<480, 4, true>(P, L, smem, grid, s);
         if (nt == kNarrowNT)
-            return sc<kNarrowNT, 4, true>(P, L, smem, grid, s);
+            return sc<kNarrowNT, kNarrowItems, true>(P, L, smem, grid, s);
         return items == 4 ? sc<256, 4, true>(P, L, smem, grid, s) : sc<256, 8, true>(P, L, smem, grid, s);
     }
     if (nt == 512)

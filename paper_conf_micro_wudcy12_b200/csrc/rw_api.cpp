@@ -942,7 +942,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         vars.push_back({256, 5});
     }
     vars.push_back({256, 4});
-    // register terminal: 15 compute warps per SM by default (the aggregate kernel has
+    // register terminal: 15 (generic) or 18 (narrow sums) compute warps per SM (the aggregate kernel has
     // no writer warps, so its register file takes more compute threads; measured C4
     // 8.56 ms at 256 x 8, 7.43 ms at 384 x 5, 7.06 ms at 448 x 4, 6.52 ms at 480 x 4);
     // opts.reserved[4]: 1 = the 256-thread variants, 4 = 384 x 5, 5 = 448 x 4
@@ -954,7 +954,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         const bool q1shape = P.nagg == 5 && narrow_n == 2 && narrow_all64 &&
                              narrow_flush >= (1 << 16) && p->o.reserved[4] == 0;
         vars.push_back(p->o.reserved[4] == 4 ? Var{384, 5} : p->o.reserved[4] == 5 ? Var{448, 4}
-                       : q1shape ? Var{kNarrowNT, 4} : Var{480, 4});
+                       : q1shape ? Var{kNarrowNT, kNarrowItems} : Var{480, 4});
     }
     if (force_items > 0) {
         std::vector<Var> v2;
@@ -987,10 +987,6 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             for (int S = 1; S <= 6; S++) {
                 if (want_stages && S != want_stages) continue;
                 if (base + (size_t)S * P.stage_bytes > per_cta) continue;
-                // register terminal: the stage + scratch buffers take the partials at the end
-                if (agg_mode_for(nt) == 2 &&
-                    (size_t)S * P.stage_bytes + P.scratch_bytes < (size_t)P.D * (P.nagg + 1) * nt * 8)
-                    continue;
                 size_t Rb = 0;
                 if (!L.agg && !direct && !global_ring) {
                     Rb = want_ring ? want_ring : (per_cta - base - (size_t)S * P.stage_bytes) / 128 * 128;

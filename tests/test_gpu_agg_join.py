@@ -42,7 +42,7 @@ def test_q1_wide_cta_variants(variant, n):
     got, plan = run_gpu(spec, ins, capacity=6, variant=variant)
     assert_same(got, run_oracle(spec, ins))
     assert {4: "tile 1920", 5: "tile 1792", 1: "tile 2048", 6: "tile 1920 rows (4/thread)",
-            0: "tile 2176 rows (4/thread)"}[variant] in plan.explain(plan.out_id)
+            0: "tile 2304 rows (4/thread)"}[variant] in plan.explain(plan.out_id)
 
 
 @pytest.mark.parametrize("lo,hi", [(-1000, 1000), (-(2**40), 2**40), (-(2**63), 2**63 - 1), (5, 5)])
