@@ -65,10 +65,11 @@ def main(rep, name, cfg, alg_bytes=None, note=""):
         lines += ["", "warp stall samples (share of all samples):", "", "| reason | share |", "|---|---|"]
         for c, v in sorted(tot.items(), key=lambda x: -x[1])[:10]:
             lines.append(f"| {c[6:]} | {100 * v / s:.1f}% |")
-    os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
-    with open(os.path.join(ROOT, "profiles", f"{name}.md"), "w") as f:
+    outdir = os.environ.get("RW_PROFILE_DIR", os.path.join(ROOT, "profiles"))
+    os.makedirs(outdir, exist_ok=True)
+    with open(os.path.join(outdir, f"{name}.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
-    tj = os.path.join(ROOT, "profiles", "traffic.json")
+    tj = os.path.join(outdir, "traffic.json")
     t = json.load(open(tj)) if os.path.exists(tj) else {}
     t[cfg] = traffic
     json.dump(t, open(tj, "w"), indent=1)
