@@ -164,8 +164,8 @@ rw_status rw_plan_add_join(rw_plan *plan, int32_t left, int32_t right, int32_t n
  * schemas (RW_E_TYPE) of at most 4 columns (RW_E_UNSUPPORTED) and must be sorted on
  * every column, lexicographically in the declared signedness (nkey_sorted == ncols,
  * else RW_E_UNSORTED).  Output: same schema, ascending, sorted on every column.
- * Runs as a merge-path kernel over the materialised inputs; a
- * downstream SELECT / PROJECT scans its output. */
+ * Runs as a merge-path kernel with a decoupled look-back over the materialised inputs
+ * (SURVEY §8(f) N3); a downstream SELECT / PROJECT scans its output. */
 rw_status rw_plan_add_setop(rw_plan *plan, int32_t left, int32_t right, int32_t op, int32_t *node);
 
 /* Group-by aggregate (§2.2, §5.2 Q1; A10-A12): group columns are dense

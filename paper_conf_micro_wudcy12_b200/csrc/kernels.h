@@ -62,10 +62,12 @@ struct SetLaunch {
     int32_t *nbr;                    // per split: has_pred | pred_is_x << 1 | has_succ << 2 | succ_is_x << 3
     uint64_t *pcount;                // per-partition emitted rows, then exclusive offsets
     int64_t *total;                  // device row count of the result
+    uint64_t *status;                // non-null: single pass with decoupled look-back (nparts words)
+    uint32_t epoch;
 };
 size_t set_op_smem(int ncols);
 int set_partition_rows();
-cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st);   // 4 launches
+cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st);   // 2 launches (look-back) or 4
 
 size_t scan_ctl_bytes();
 size_t join_run_cache_bytes();

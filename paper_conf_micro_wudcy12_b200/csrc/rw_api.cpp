@@ -1254,8 +1254,15 @@ void run_group(ExecCtx &X, int gi)
         S.pcount = (uint64_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 8);
         S.nbr = (int32_t *)temp_alloc(p, (size_t)(S.nparts + 1) * 4);
         S.total = n_dev;
+        // one pass with a decoupled look-back over the partitions (opts.reserved[1] & 1:
+        // the count / scan / write passes)
+        if (!(p->o.reserved[1] & 1)) {
+            ensure_status(p, S.nparts + 1);
+            S.status = p->status;
+            S.epoch = next_epoch(p);
+        }
         cuda_check(set_op_launch(S, p->sms, p->stream), "k_set_op");
-        p->launches += S.nparts > 0 ? 4 : 2;
+        p->launches += S.status ? (S.nparts > 0 ? 2 : 1) : (S.nparts > 0 ? 4 : 2);
     } else {
         const Node &jn = p->nodes[g.join];
         Rel lr = rel_of(X, jn.left), rr = rel_of(X, jn.right);

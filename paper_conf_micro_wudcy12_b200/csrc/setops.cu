@@ -11,14 +11,15 @@
 //   DIFFERENCE emits e  iff  e in x, succ != e               (last x row of a segment
 //                                                            that has no y row)
 // so each segment emits at most once and the output is ascending without a sort.
-//   k_set_splits   merge-path split of every partition boundary (2048 merged rows);
-//   k_set_op<0>    per partition: stage both inputs' rows in smem as order-preserving
-//                  u64 keys, merge walk (8 positions per thread), emission flags,
-//                  count per partition;
-//   k_set_scan     exclusive scan of the partition counts (one CTA);
-//   k_set_op<1>    recomputes the flags and writes the emitted tuples at their offsets.
+//   k_set_splits   merge-path split of every partition boundary (2048 merged rows)
+//                  and the boundary's merged neighbours;
+//   k_set_op       per partition: stage both inputs' rows in smem as order-preserving
+//                  u64 keys (one packed key when a tuple is <= 8 bytes), merge walk
+//                  (8 positions per thread), emission flags, block scan, decoupled
+//                  look-back over the partitions for the output offset, store.
+// (diagnostics: a count pass + k_set_scan + a write pass instead of the look-back)
+#include "chain.cuh"
 #include "kernels.h"
-#include "ptx.cuh"
 
 namespace rw {
 
@@ -130,6 +131,7 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
     int32_t *msrc = (int32_t *)(s + (size_t)NC * kSetS);       // merged position -> staged row
     __shared__ int32_t wcnt[kThreads / 32 + 1];
     __shared__ int32_t nbr[4];                            // has_pred, pred_is_x, has_succ, succ_is_x
+    __shared__ int64_t pbase;                             // single pass: the partition's output offset
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     constexpr int nc = NC;
     for (int64_t p = blockIdx.x; p < S.nparts; p += gridDim.x) {
@@ -244,7 +246,24 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
                 S.pcount[p] = (uint64_t)tot;
             continue;
         }
-        int64_t o = (int64_t)S.pcount[p] + base;
+        int64_t o;
+        if (S.status) {
+            // single pass: decoupled look-back over the partitions (every CTA of the
+            // grid is resident and walks its partitions in increasing order, so the
+            // predecessors a partition waits for always make progress)
+            if (warp == 0) {
+                const uint64_t excl = lookback_warp(S.status, p, (uint64_t)tot, S.epoch);
+                if (lane == 0) {
+                    pbase = (int64_t)excl;
+                    if (p == S.nparts - 1)
+                        *S.total = (int64_t)excl + tot;
+                }
+            }
+            __syncthreads();
+            o = pbase + base;
+        } else {
+            o = (int64_t)S.pcount[p] + base;
+        }
         for (uint32_t em = emit; em; em &= em - 1) {
             const int q = __ffs(em) - 1;
             const int e = msrc[dt + q];
@@ -314,6 +333,13 @@ static void set_passes(const SetLaunch &S, int sms, cudaStream_t st)
     int occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_set_op<NC, true, PACKED>, kThreads, smem);
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(S.nparts, (int64_t)sms * std::max(occ, 1)));
+    if (S.status) {                       // single pass with decoupled look-back
+        if (S.nparts > 0)
+            k_set_op<NC, true, PACKED><<<grid, kThreads, smem, st>>>(S);
+        else
+            cudaMemsetAsync(S.total, 0, sizeof(int64_t), st);
+        return;
+    }
     if (S.nparts > 0)
         k_set_op<NC, false, PACKED><<<grid, kThreads, smem, st>>>(S);
     k_set_scan<<<1, 1024, 0, st>>>(S);
