@@ -34,6 +34,7 @@ CONFIGS = {
     "c2": dict(name="C2: SELECT->PROJECT->SELECT over 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
     "c3": dict(name="C3: JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "c4": dict(name="C4: TPC-H Q1-shaped select/arith/group-by over 6e8 lineitem rows per GPU", rows=workloads.C4_ROWS),
+    "cc": dict(name="Pattern (c): key SELECTs on both inputs -> JOIN (2 x 2^26, Zipf 0.5) -> SELECT -> PROJECT", rows=workloads.C3_ROWS),
     "cd": dict(name="Pattern (d) input dependence: 2 SELECTs (25% each) sharing one input of 2^29 x 4 int32 per GPU", rows=workloads.C2_ROWS),
     "cs": dict(name="Set operator (--setop, default UNION) of two sorted (u32 key, u32 val) relations, 2^26 tuples each per GPU, key-range sharded", rows=1 << 26),
     "c5": dict(name="C5: JOIN->JOIN->SELECT over three relations, 2^27 rows each per GPU (2^30 at 8 GPUs), key-range sharded", rows=1 << 27),
@@ -78,6 +79,8 @@ def spec_and_inputs(cfg: str, rows: int, start: int, device):
         return workloads.c2_spec(), workloads.c2_inputs(rows, start, device)
     if cfg == "c3":
         return workloads.c3_spec(), workloads.c3_inputs(rows, device=device)
+    if cfg == "cc":
+        return workloads.cc_spec(), workloads.c3_inputs(rows, device=device)
     if cfg == "c4":
         return workloads.c4_spec(), workloads.c4_inputs(rows, start, device)
     if cfg == "cd":
@@ -197,7 +200,7 @@ def run_reference(args):
         return 0
     cfg = args.config
     rows = args.rows or CONFIGS[cfg]["rows"]
-    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24, "cs": 1 << 21}[cfg]
+    sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24, "cs": 1 << 21, "cc": 1 << 21}[cfg]
     import oracle
     oracle.build()
     vals = []
@@ -260,7 +263,7 @@ def main():
             return plan, ids, outs, cap, out_types
         out_types = plan.node_schema(ids[spec["out"]])
         cap = {"c4": 6}.get(cfg, max(nrows.values()))
-        if cfg == "c3":
+        if cfg in ("c3", "cc"):
             cap = 400_000_000 if rows == workloads.C3_ROWS else 8 * rows + 1024
         if cfg in ("c5", "cs"):
             cap = 2 * max(nrows.values()) + 4096
@@ -361,7 +364,7 @@ def main():
     peak, peak_src = measured_peak()
     kern_ms = statistics.mean(per)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
-    kname = {"c3": "k_join_runs + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand",
+    kname = {"c3": "k_join_runs + k_join_expand", "cc": "k_join_runs (key SELECTs fused) + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand",
              "cs": "k_set_splits + k_set_op x2 + k_set_scan"}.get(cfg, "k_scan_chain")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": ncu_traffic(cfg), "kernel": kname,
@@ -373,7 +376,7 @@ def main():
            "c4": f"row-shard x{world} + limb all-reduce"}
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs") else "i32"),
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs", "cc") else "i32"),
             "data": "synthetic (rwgen seeded SplitMix64 generators, generated on device)",
             "config": {"workload": CONFIGS[cfg]["name"], "rows_per_gpu": nrows, "output_rows_per_gpu": n_out,
                        "parallelism": par.get(cfg, f"row-shard x{world}"),
@@ -381,7 +384,7 @@ def main():
                        "fused": True},
             "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
 
-    if not args.no_unfused and cfg in ("c1", "c2", "c4", "c3", "cd"):
+    if not args.no_unfused and cfg in ("c1", "c2", "c4", "c3", "cd", "cc"):
         del outs
         torch.cuda.empty_cache()
         uplan, uids, uouts, ucap, _ = make(False)
@@ -424,7 +427,7 @@ def main():
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:
-        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26, "cs": 1 << 22}[cfg]
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26, "cs": 1 << 22, "cc": 1 << 22}[cfg]
         v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
         line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
                                 "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}

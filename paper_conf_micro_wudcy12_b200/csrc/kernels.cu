@@ -913,6 +913,25 @@ __device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
     return lo;
 }
 
+// fused upstream SELECT on the join key (N2): every atom must hold for the run's key
+template <typename K>
+__device__ __forceinline__ bool key_pass(const JoinRunsLaunch &J, K key)
+{
+    bool ok = true;
+    for (int i = 0; i < J.nkpred; i++) {
+        const K c = (K)J.kpk[i];
+        switch (J.kop[i]) {
+        case C_LT: ok = ok && key < c; break;
+        case C_LE: ok = ok && key <= c; break;
+        case C_GT: ok = ok && key > c; break;
+        case C_GE: ok = ok && key >= c; break;
+        case C_EQ: ok = ok && key == c; break;
+        default: ok = ok && key != c; break;
+        }
+    }
+    return ok;
+}
+
 // Two streaming passes (no look-back on the critical path): WRITE = false counts
 // the matched runs and join candidates of every partition; k_scan_parts turns the
 // counts into exclusive offsets; WRITE = true recomputes the partition (identical
@@ -1078,7 +1097,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_join_runs(const __grid_constant
                 const int64_t nr_ = k + 1 < H ? j0 + hR[k + 1] : tailR;
                 lenl[q] = nl_ - (i0 + hL[k]);
                 lenr[q] = nr_ - (j0 + hR[k]);
-                if (lenl[q] > 0 && lenr[q] > 0) {
+                if (lenl[q] > 0 && lenr[q] > 0 && key_pass<K>(J, hK[k])) {
                     matched |= 1u << q;
                     cnt[q] = (uint64_t)lenl[q] * (uint64_t)lenr[q];
                     nrun++;

@@ -7,6 +7,7 @@
 namespace rw {
 
 constexpr int kMaxStages = 8;
+constexpr int kMaxKeyPreds = 8;      // key-predicate atoms fused into one JOIN
 
 struct AggFinal {
     const unsigned long long *acc;   // D * NA * 2 (lo, hi); zeroed by the finalize kernel after reading
@@ -36,6 +37,12 @@ struct JoinRunsLaunch {
     int64_t *totals;                 // [0] runs, [1] join candidates
     int64_t *split;                  // nparts + 1 merge-path splits (k_merge_splits)
     uint64_t *pruns, *pouts;         // per-partition counts, then exclusive offsets
+    // SELECTs on the join key fused into the run matching (SURVEY §8(f) N2
+    // Fig. 13): a run is matched only if its key passes every atom (key op kpk[i]),
+    // compared in the key type; a key predicate keeps or drops whole runs
+    int32_t nkpred;
+    uint8_t kop[kMaxKeyPreds];
+    int64_t kpk[kMaxKeyPreds];
 };
 
 struct JoinExpand {

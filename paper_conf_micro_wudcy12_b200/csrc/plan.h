@@ -51,6 +51,10 @@ struct Group {
     int agg = -1;                    // AGG terminal (or -1: materialising terminal)
     int out = -1;                    // node whose relation this group produces
     std::vector<int> deps;           // groups that must run first
+    // G_JOIN: SELECT nodes on the join key fused into the run matching (N2); the
+    // join then reads their source relations (jl, jr) directly
+    std::vector<int> pre;            // absorbed SELECT nodes
+    int jl = -1, jr = -1;            // relations feeding the join (after absorption)
 };
 
 Interval type_range(int t);

@@ -297,6 +297,27 @@ int dep_group(const rw_plan *p, int id, Grouping &G)
     return make_group(p, id, G);
 }
 
+// SELECTs on the key column only, directly upstream of a JOIN input (single consumer):
+// they keep or drop whole key runs, so the join's run matching applies them and the
+// join reads their source relation (CTA dependence fused, Fig. 13; N2).
+int absorb_key_selects(const rw_plan *p, int nd, const Grouping &G, Group &g, int &npred)
+{
+    if (!p->o.fuse)
+        return nd;
+    while (p->nodes[nd].kind == N_SELECT && G.consumers[nd] == 1) {
+        const Node &sn = p->nodes[nd];
+        bool keyonly = !sn.preds.empty();
+        for (const rw_pred &a : sn.preds)
+            keyonly = keyonly && a.col == 0 && !a.rhs_is_col;
+        if (!keyonly || npred + (int)sn.preds.size() > kMaxKeyPreds)
+            break;
+        npred += (int)sn.preds.size();
+        g.pre.push_back(nd);
+        nd = sn.in;
+    }
+    return nd;
+}
+
 int make_group(const rw_plan *p, int id, Grouping &G)
 {
     auto it = G.produced_by.find(id);
@@ -333,7 +354,10 @@ int make_group(const rw_plan *p, int id, Grouping &G)
     if (n.kind == N_JOIN) {
         g.kind = G_JOIN;
         g.join = id;
-        int a = dep_group(p, n.left, G), b = dep_group(p, n.right, G);
+        int np = 0;
+        g.jl = absorb_key_selects(p, n.left, G, g, np);
+        g.jr = absorb_key_selects(p, n.right, G, g, np);
+        int a = dep_group(p, g.jl, G), b = dep_group(p, g.jr, G);
         if (a >= 0) g.deps.push_back(a);
         if (b >= 0) g.deps.push_back(b);
         G.groups.push_back(g);
@@ -368,7 +392,10 @@ int make_group(const rw_plan *p, int id, Grouping &G)
         g.kind = G_JOIN;
         g.join = src;
         const Node &j = p->nodes[src];
-        int a = dep_group(p, j.left, G), b = dep_group(p, j.right, G);
+        int np = 0;
+        g.jl = absorb_key_selects(p, j.left, G, g, np);
+        g.jr = absorb_key_selects(p, j.right, G, g, np);
+        int a = dep_group(p, g.jl, G), b = dep_group(p, g.jr, G);
         if (a >= 0) g.deps.push_back(a);
         if (b >= 0) g.deps.push_back(b);
     } else {
@@ -1265,7 +1292,7 @@ void run_group(ExecCtx &X, int gi)
         p->launches += S.status ? (S.nparts > 0 ? 2 : 1) : (S.nparts > 0 ? 4 : 2);
     } else {
         const Node &jn = p->nodes[g.join];
-        Rel lr = rel_of(X, jn.left), rr = rel_of(X, jn.right);
+        Rel lr = rel_of(X, g.jl >= 0 ? g.jl : jn.left), rr = rel_of(X, g.jr >= 0 ? g.jr : jn.right);
         const int64_t nl = host_count(X, lr), nr = host_count(X, rr);
         const int kt = lr.types[0];
         // phase 1: run records
@@ -1294,6 +1321,13 @@ void run_group(ExecCtx &X, int gi)
         J.split = (int64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
         J.pruns = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
         J.pouts = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
+        J.nkpred = 0;
+        for (int sid : g.pre)
+            for (const rw_pred &a : p->nodes[sid].preds) {
+                J.kop[J.nkpred] = (uint8_t)a.op;
+                J.kpk[J.nkpred] = (int64_t)wrap_to(kt, a.rhs_const);
+                J.nkpred++;
+            }
         const size_t smem1 = join_runs_smem(kt);
         const int occ1 = std::max(1, chain_occupancy(3, kThreads, 8, smem1));
         const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
@@ -1700,13 +1734,15 @@ std::string explain(rw_plan *p, int out_node)
             for (size_t q = 0; q < G.groups.size(); q++) {
                 const Group &g = G.groups[q];
                 if (g.out == (int)i || g.join == (int)i || g.agg == (int)i ||
-                    std::find(g.chain.begin(), g.chain.end(), (int)i) != g.chain.end())
+                    std::find(g.chain.begin(), g.chain.end(), (int)i) != g.chain.end() ||
+                    std::find(g.pre.begin(), g.pre.end(), (int)i) != g.pre.end())
                     gc = (int)q;
             }
             bool fused = false;
             if (gc >= 0) {
                 const Group &g = G.groups[gc];
-                fused = pr == g.join || std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end();
+                fused = pr == g.join || std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end() ||
+                        std::find(g.pre.begin(), g.pre.end(), pr) != g.pre.end();
             }
             (void)gp;
             s << "  " << pr << "(" << kn[p->nodes[pr].kind] << ") -> " << i << "(" << kn[n.kind]
@@ -1726,6 +1762,7 @@ std::string explain(rw_plan *p, int out_node)
         if (g.kind == G_SCAN) s << "src " << g.source;
         else if (g.kind == G_SET) s << "setop " << g.join;
         else s << "join " << g.join;
+        for (int c : g.pre) s << ", key SELECT " << c << " (fused into the run matching)";
         for (int c : g.chain) s << ", " << kn[p->nodes[c].kind] << " " << c;
         if (g.agg >= 0) s << ", AGG " << g.agg;
         s << "] -> node " << g.out;

@@ -181,3 +181,54 @@ def test_pattern_c_selects_upstream_of_join():
     got, plan = run_gpu(spec, ins, capacity=400_000)
     assert_same(got, run_oracle(spec, ins))
     assert "materialised" in plan.explain(plan.out_id)
+
+
+@pytest.mark.parametrize("n", [0, 1000, 30_000, 200_000])
+@pytest.mark.parametrize("fuse", [True, False])
+def test_n2_key_selects_fused_into_join(n, fuse):
+    """SELECTs on the join key upstream of both JOIN inputs (pattern (c), Fig. 13,
+    SURVEY §8(f) N2): fused into the run matching (whole key runs kept or dropped), the
+    join reads the unfiltered relations; no SELECT kernel runs.  Bit-exact vs oracle."""
+    spec = workloads.c3_spec()
+    k1, k2, k3 = workloads.thr_u32(0.7), workloads.thr_u32(0.2), workloads.thr_u32(0.5)
+    spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(0, "<", k1)]},
+                     {"id": "fl2", "op": "select", "in": "fl", "preds": [(0, "!=", k3)]},
+                     {"id": "fr", "op": "select", "in": "R", "preds": [(0, ">=", k2), (0, "<=", k1 + 12345)]},
+                     {"id": "j", "op": "join", "left": "fl2", "right": "fr", "nkey": 1}] + spec["nodes"][1:]
+    ins = workloads.c3_inputs(n, device=DEV, cfg=0x97)
+    got, plan = run_gpu(spec, ins, capacity=8 * max(n, 1) + 1024, fuse=fuse)
+    assert_same(got, run_oracle(spec, ins))
+    ex = plan.explain(plan.out_id)
+    if fuse:
+        assert ex.count("key SELECT") == 3 and "group 1" not in ex, ex
+
+
+def test_n2_mixed_key_and_value_selects():
+    """A key SELECT on L is fused; a value SELECT on R stays a materialised group."""
+    spec = workloads.c3_spec()
+    spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(0, ">", workloads.thr_u32(0.1))]},
+                     {"id": "fr", "op": "select", "in": "R", "preds": [(1, "<", workloads.thr_u32(0.5))]},
+                     {"id": "j", "op": "join", "left": "fl", "right": "fr", "nkey": 1}] + spec["nodes"][1:]
+    ins = workloads.c3_inputs(50_000, device=DEV, cfg=0x98)
+    got, plan = run_gpu(spec, ins, capacity=500_000)
+    assert_same(got, run_oracle(spec, ins))
+    ex = plan.explain(plan.out_id)
+    assert ex.count("key SELECT") == 1 and "group 1" in ex
+
+
+def test_n2_signed_keys():
+    import torch
+    rng = np.random.default_rng(3)
+    def rel(n):
+        k = np.sort(rng.integers(-500, 500, n)).astype(np.int32)
+        v = rng.integers(0, 1000, n).astype(np.int32)
+        o = np.lexsort((v, k))
+        return [torch.from_numpy(k[o].copy()).to(DEV), torch.from_numpy(v[o].copy()).to(DEV)]
+    spec = {"inputs": {"L": {"types": ["i32", "i32"], "nkey_sorted": 1}, "R": {"types": ["i32", "i32"], "nkey_sorted": 1}},
+            "nodes": [{"id": "fl", "op": "select", "in": "L", "preds": [(0, ">=", -100), (0, "<", 250)]},
+                      {"id": "j", "op": "join", "left": "fl", "right": "R", "nkey": 1}],
+            "out": "j"}
+    ins = {"L": rel(20_000), "R": rel(15_000)}
+    got, plan = run_gpu(spec, ins, capacity=2_000_000)
+    assert_same(got, run_oracle(spec, ins))
+    assert "key SELECT" in plan.explain(plan.out_id)

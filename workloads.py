@@ -97,6 +97,17 @@ def c3_spec() -> Dict:
             "out": "p"}
 
 
+def cc_spec() -> Dict:
+    """Pattern (c) (Fig. 14(c), Fig. 13): SELECTs on the join key of both C3
+    inputs, then the C3 join -> SELECT -> PROJECT.  Key ranges keep about half of L's
+    and three quarters of R's keys (thresholds on the scattered key values)."""
+    spec = c3_spec()
+    spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(0, "<", thr_u32(0.5))]},
+                     {"id": "fr", "op": "select", "in": "R", "preds": [(0, ">=", thr_u32(0.25))]},
+                     {"id": "j", "op": "join", "left": "fl", "right": "fr", "nkey": 1}] + spec["nodes"][1:]
+    return spec
+
+
 def c3_inputs(n: int, K: int = None, device="cpu", cfg: int = 3, cdf=None) -> Dict[str, List]:
     K = K or max(n, 1)
     if cdf is None and n > 0:
