@@ -249,7 +249,7 @@ __device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_
     bar_sync(kComputeBar, NT);
 }
 
-template <int NT, int ITEMS, bool AGG, bool JOIN>
+template <int NT, int ITEMS, bool AGG, bool JOIN, bool MULTI = false>
 __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_chain(const __grid_constant__ ChainProg P,
                                                                      const __grid_constant__ TileLaunch L,
                                                                      const __grid_constant__ JoinExpand X)
@@ -280,7 +280,9 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
     const bool emit = !AGG && !(L.dbg & 2) && !L.direct;
-    const int NB = (AGG || JOIN) ? 1 : P.nbranch;   // input-dependence branches (host: 1 for agg / direct)
+    // input-dependence branches: only the MULTI instance carries the branch loop, so
+    // the single-chain instances compile with NB == 1
+    const int NB = (AGG || JOIN || !MULTI) ? 1 : P.nbranch;
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) {
@@ -1270,6 +1272,9 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
         case 6: return occ(k_scan_chain<256, 6, false, false>, smem, 256 + kAuxThreads);
         default: return occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
         }
+    case 4:   // input-dependence branches
+        return items == 4 ? occ(k_scan_chain<256, 4, false, false, true>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, false, false, true>, smem, 256 + kAuxThreads);
     case 1:
         if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + 32);
         if (nt == 384) return occ(k_scan_chain<384, 5, true, false>, smem, 384 + 32);
@@ -1283,12 +1288,13 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
     }
 }
 
-template <int NT, int ITEMS, bool AGG>
+template <int NT, int ITEMS, bool AGG, bool MULTI = false>
 static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
     JoinExpand X{};
-    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_chain<NT, ITEMS, AGG, false><<<grid, NT + aux_threads(AGG), smem, s>>>(P, L, X);
+    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, false, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+    k_scan_chain<NT, ITEMS, AGG, false, MULTI><<<grid, NT + aux_threads(AGG), smem, s>>>(P, L, X);
     return cudaGetLastError();
 }
 
@@ -1304,6 +1310,8 @@ cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const Joi
 cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem,
                               int grid, cudaStream_t s)
 {
+    if (!agg && P.nbranch > 1)
+        return items == 4 ? sc<256, 4, false, true>(P, L, smem, grid, s) : sc<256, 8, false, true>(P, L, smem, grid, s);
     if (agg) {
         if (nt == 128)
             return sc<128, 16, true>(P, L, smem, grid, s);

@@ -78,7 +78,7 @@ cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st);   // 2 
 
 size_t scan_ctl_bytes();
 size_t join_run_cache_bytes();
-int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs
+int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs, 4 scan branches
 cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem, int grid,
                               cudaStream_t s);
 cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s);

@@ -969,6 +969,12 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         vars.push_back({256, 5});
     }
     vars.push_back({256, 4});
+    if (nbr > 1) {   // the branch-loop instance exists for 256 x 8 and 256 x 4
+        std::vector<Var> v2;
+        for (const Var &v : vars)
+            if (v.nt == 256 && (v.items == 8 || v.items == 4)) v2.push_back(v);
+        vars = v2;
+    }
     // register terminal: 15 (generic) or 18 (narrow sums) compute warps per SM (the aggregate kernel has
     // no writer warps, so its register file takes more compute threads; measured C4
     // 8.56 ms at 256 x 8, 7.43 ms at 384 x 5, 7.06 ms at 448 x 4, 6.52 ms at 480 x 4);
@@ -1021,7 +1027,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 }
                 const size_t smem = base + (size_t)S * P.stage_bytes + Rb;
                 if (smem > per_cta) continue;
-                if (chain_occupancy(L.agg ? 1 : 0, nt, items, smem) < occ_t) continue;
+                if (chain_occupancy(L.agg ? 1 : (nbr > 1 ? 4 : 0), nt, items, smem) < occ_t) continue;
                 double inflight = std::min<double>((double)occ_t * S * P.stage_bytes, 192.0 * 1024);
                 double score;
                 if (L.agg || direct || global_ring) {
