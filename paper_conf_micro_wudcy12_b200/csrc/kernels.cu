@@ -298,7 +298,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
         ctl->hpos = 0;
         fence_mbar_init();
     }
-    if (AGG) {
+    if constexpr (AGG) {
         for (size_t q = tid; q < part_words; q += blockDim.x)
             part[q] = 0;
         for (int q = tid; q < P.D * NA * 2; q += blockDim.x)
