@@ -105,6 +105,22 @@ __device__ inline uint64_t lookback_warp(uint64_t *status, int64_t tile, uint64_
     return excl;
 }
 
+// Persistent kernels claim work items in order with ctrs[0] (so a decoupled look-back
+// always has forward progress, whatever number of CTAs is resident); the last CTA to
+// leave resets both counters for the next launch.
+__device__ inline void cta_exit_reset(uint32_t *ctrs)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&ctrs[1], 1u) == gridDim.x - 1) {
+            ctrs[0] = 0;
+            ctrs[1] = 0;
+            __threadfence();
+        }
+    }
+}
+
 // ---------------------------------------------------------------------------
 // Slot access.  Locations are resolved on the host (kLocScratch | byte offset),
 // so the interpreter never walks a slot table on the device.
@@ -317,90 +333,6 @@ __device__ __forceinline__ uint32_t run_ops(const ChainProg &P, int op0, int op1
             run_expr<NT, ITEMS>(code, P.ops[i].ta, P.ops[i].tb, k, (char *)loc_ptr(P.ops[i].dst, stage, scratch), a, b);
     }
     return mask;
-}
-
-// ---------------------------------------------------------------------------
-// Materialising terminal: ballot compaction + block scan + look-back + store.
-// ---------------------------------------------------------------------------
-template <int ITEMS>
-struct EmitSmem {
-    uint32_t cnt[ITEMS * kWarps];   // survivors per (item k, warp), then exclusive prefixes
-    int64_t tile_off;
-};
-
-template <int ITEMS, typename T>
-__device__ __forceinline__ void store_col(T *dst, const T *src, uint32_t mask, const uint32_t *bal,
-                                          const uint32_t *pre, int64_t base, int64_t cap)
-{
-    const int tid = threadIdx.x, warp = tid >> 5;
-    const uint32_t lt = lanemask_lt();
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        if ((mask >> k) & 1u) {
-            int64_t pos = base + pre[k * kWarps + warp] + __popc(bal[k] & lt);
-            if (pos < cap)
-                dst[pos] = src[k * kThreads + tid];
-        }
-    }
-}
-
-template <int ITEMS>
-__device__ inline void emit_tile(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
-                                 int64_t tile, int64_t ntiles, const TileLaunch &L, EmitSmem<ITEMS> *es)
-{
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    uint32_t bal[ITEMS];
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        bal[k] = __ballot_sync(0xffffffffu, (mask >> k) & 1u);
-        if (lane == 0)
-            es->cnt[k * kWarps + warp] = __popc(bal[k]);
-    }
-    __syncthreads();
-    if (warp == 0) {
-        constexpr int NV = ITEMS * kWarps;
-        constexpr int PER = (NV + 31) / 32;
-        uint32_t v[PER];
-        uint32_t s = 0;
-#pragma unroll
-        for (int q = 0; q < PER; q++) {
-            int idx = lane * PER + q;
-            v[q] = idx < NV ? es->cnt[idx] : 0;
-            s += v[q];
-        }
-        uint32_t inc = s;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o)
-                inc += y;
-        }
-        uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
-        uint32_t run = inc - s;
-#pragma unroll
-        for (int q = 0; q < PER; q++) {
-            int idx = lane * PER + q;
-            if (idx < NV)
-                es->cnt[idx] = run;
-            run += v[q];
-        }
-        uint64_t excl = lookback_warp(L.status, tile, total, L.epoch);
-        if (lane == 0) {
-            es->tile_off = (int64_t)excl;
-            if (tile == ntiles - 1)
-                *L.n_dev = (int64_t)(excl + total);
-        }
-    }
-    __syncthreads();
-    const int64_t base = es->tile_off;
-    for (int j = 0; j < P.nout; j++) {
-        const char *src = loc_ptr(P.out_loc[j], stage, scratch);
-        switch (P.out_w[j]) {
-        case 1: store_col<ITEMS, uint8_t>((uint8_t *)P.out_ptr[j], (const uint8_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
-        case 4: store_col<ITEMS, uint32_t>((uint32_t *)P.out_ptr[j], (const uint32_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
-        default: store_col<ITEMS, uint64_t>((uint64_t *)P.out_ptr[j], (const uint64_t *)src, mask, bal, es->cnt, base, P.out_capacity); break;
-        }
-    }
 }
 
 // ---------------------------------------------------------------------------
@@ -708,9 +640,12 @@ __device__ inline void reg_agg_reduce_warp(const ChainProg &P, RegAgg &R, unsign
 // Row loop of the register terminal: NAGG sums (W64: every sum column is 64-bit, so
 // no per-row type dispatch); the one-hot over the groups becomes a jump to the
 // row's group, whose partials take predicated-free adds.
+// Narrow sums (a < NN) accumulate in 32-bit partials whose flush period comes from the
+// caller-declared bounds; their values are OR-ed into `orv` so that a value outside
+// [0, 2^narrow_bits) is reported (err[2]) instead of silently wrapping a partial.
 template <int NT, int ITEMS, int NAGG, bool W64, int NN = 0>
 __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *at, const uint32_t *g, uint32_t ok,
-                                             RegAgg &R)
+                                             RegAgg &R, uint64_t &orv)
 {
     const int tid = threadIdx.x;
 #pragma unroll
@@ -721,6 +656,10 @@ __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *a
 #pragma unroll
         for (int a = 0; a < kRegA; a++)
             v[a] = a < NAGG ? (W64 ? ((const uint64_t *)ab[a])[r] : ld_ext(ab[a], at[a], r)) : 0ull;
+#pragma unroll
+        for (int a = 0; a < NN; a++)
+            if ((ok >> k) & 1u)
+                orv |= v[a];
 #pragma unroll
         for (int d = 0; d < kRegD; d++) {
             if (gk == (uint32_t)d) {
@@ -797,34 +736,36 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
             w64 = false;
     }
     // the sum count and the all-64-bit case are compile-time in the row loop
+    uint64_t orv = 0;
     if (NT == kNarrowNT) {
-        // the 544-thread instance is specialised (host-selected) for 5 all-64-bit sums of
+        // the 576-thread instance is specialised (host-selected) for 5 all-64-bit sums of
         // which the first 2 are narrow: only this row loop is compiled into it, which is
-        // what lets 17 compute warps fit the register file
-        agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R);
-        return;
-    }
-    if (w64 && P.agg_narrow) {
+        // what lets 18 compute warps fit the register file
+        agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R, orv);
+    } else if (w64 && P.agg_narrow) {
         switch (P.nagg * 4 + P.agg_narrow) {
-        case 3 * 4 + 1: agg_rows_reg<NT, ITEMS, 3, true, 1>(ab, at, g, ok, R); return;
-        case 3 * 4 + 2: agg_rows_reg<NT, ITEMS, 3, true, 2>(ab, at, g, ok, R); return;
-        case 4 * 4 + 1: agg_rows_reg<NT, ITEMS, 4, true, 1>(ab, at, g, ok, R); return;
-        case 4 * 4 + 2: agg_rows_reg<NT, ITEMS, 4, true, 2>(ab, at, g, ok, R); return;
-        case 5 * 4 + 1: agg_rows_reg<NT, ITEMS, 5, true, 1>(ab, at, g, ok, R); return;
-        default: agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R); return;
+        case 3 * 4 + 1: agg_rows_reg<NT, ITEMS, 3, true, 1>(ab, at, g, ok, R, orv); break;
+        case 3 * 4 + 2: agg_rows_reg<NT, ITEMS, 3, true, 2>(ab, at, g, ok, R, orv); break;
+        case 4 * 4 + 1: agg_rows_reg<NT, ITEMS, 4, true, 1>(ab, at, g, ok, R, orv); break;
+        case 4 * 4 + 2: agg_rows_reg<NT, ITEMS, 4, true, 2>(ab, at, g, ok, R, orv); break;
+        case 5 * 4 + 1: agg_rows_reg<NT, ITEMS, 5, true, 1>(ab, at, g, ok, R, orv); break;
+        default: agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R, orv); break;
         }
-    }
-    if (w64) {
+    } else if (w64) {
         switch (P.nagg) {
-        case 0: agg_rows_reg<NT, ITEMS, 0, true>(ab, at, g, ok, R); return;
-        case 1: agg_rows_reg<NT, ITEMS, 1, true>(ab, at, g, ok, R); return;
-        case 2: agg_rows_reg<NT, ITEMS, 2, true>(ab, at, g, ok, R); return;
-        case 3: agg_rows_reg<NT, ITEMS, 3, true>(ab, at, g, ok, R); return;
-        case 4: agg_rows_reg<NT, ITEMS, 4, true>(ab, at, g, ok, R); return;
-        default: agg_rows_reg<NT, ITEMS, kRegA, true>(ab, at, g, ok, R); return;
+        case 0: agg_rows_reg<NT, ITEMS, 0, true>(ab, at, g, ok, R, orv); break;
+        case 1: agg_rows_reg<NT, ITEMS, 1, true>(ab, at, g, ok, R, orv); break;
+        case 2: agg_rows_reg<NT, ITEMS, 2, true>(ab, at, g, ok, R, orv); break;
+        case 3: agg_rows_reg<NT, ITEMS, 3, true>(ab, at, g, ok, R, orv); break;
+        case 4: agg_rows_reg<NT, ITEMS, 4, true>(ab, at, g, ok, R, orv); break;
+        default: agg_rows_reg<NT, ITEMS, kRegA, true>(ab, at, g, ok, R, orv); break;
         }
+    } else {
+        agg_rows_reg<NT, ITEMS, kRegA, false>(ab, at, g, ok, R, orv);
     }
-    agg_rows_reg<NT, ITEMS, kRegA, false>(ab, at, g, ok, R);
+    // a narrow value outside its declared bounds: report (err[2]) rather than wrap
+    if (orv >> P.narrow_bits)
+        atomicAdd(err + 2, 1);
 }
 
 // End-of-kernel combine of the thread-private partials: one thread per (group,

@@ -94,6 +94,8 @@ struct ChainProg {
     int32_t agg_mode;                   // 0: thread-private partials in smem; 2: register one-hot (D <= kRegD, nagg <= kRegA)
     int32_t agg_narrow;                 // mode 2: the first agg_narrow sums are non-negative with |v| < 2^16 and
                                         // accumulate in 32-bit registers (flush_rows keeps them below 2^32)
+    int32_t narrow_bits;                // every narrow value is < 2^narrow_bits (declared bounds); the kernel ORs
+                                        // the narrow values of a tile and counts a violation into err[2]
     // input-dependence fusion (§4.4, Fig. 14(d)): nbranch chains over the same
     // staged tile, each with its own mask and compacted output.  Branch b runs ops
     // [br_op_end[b-1], br_op_end[b]) and writes output columns [br_out_end[b-1], br_out_end[b]).
@@ -101,6 +103,7 @@ struct ChainProg {
     uint8_t br_op_end[kMaxBranch];
     uint8_t br_out_end[kMaxBranch];
     int64_t br_cap[kMaxBranch];         // output capacity of branch b (b = 0: out_capacity)
+    uint8_t br_nw[kMaxBranch][3];       // output columns of branch b that are 1, 4 and 8 bytes wide
     uint32_t stage_bytes;               // bytes of one stage (all input slots, aligned)
     uint32_t scratch_bytes;             // bytes of scratch (computed slots)
 };
@@ -124,6 +127,9 @@ struct TileLaunch {
     int32_t *err;              // [0] domain errors
     int32_t dbg;               // diagnostics: 1 = skip look-back (offset = tile * T, uncompacted),
                                // 2 = stream tiles only, 4 = per-tile phase timestamps into dbg_ts
+    int32_t delay;             // emitting scan kernel: compute warps hold at most `delay` evaluated tiles
+                               // (in their input stages) waiting for their global offsets
+    uint32_t warp_buf;         // emitting scan kernel: bytes of each compute warp's compaction buffer
     uint64_t *dbg_ts;          // 12 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots, scattered, reserve start; join: records cached, gathered)
 };
 

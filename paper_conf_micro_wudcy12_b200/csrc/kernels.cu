@@ -23,19 +23,6 @@ namespace rw {
 
 static __host__ __device__ inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-__device__ inline void cta_exit_reset(uint32_t *ctrs)
-{
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        if (atomicAdd(&ctrs[1], 1u) == gridDim.x - 1) {
-            ctrs[0] = 0;
-            ctrs[1] = 0;
-            __threadfence();
-        }
-    }
-}
-
 // ===========================================================================
 // Fused scan chain, warp-specialised (kThreads compute threads + 3 warps):
 //   producer warp  : claims tiles in order (global atomic) and stages each live
@@ -755,6 +742,8 @@ __global__ void __launch_bounds__(kThreads) k_agg_finalize(const __grid_constant
         *F.n_dev = base;
         F.err[1] = F.err[0];
         F.err[0] = 0;
+        F.err[3] = F.err[2];
+        F.err[2] = 0;
     }
 }
 

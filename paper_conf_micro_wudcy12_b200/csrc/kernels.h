@@ -21,7 +21,7 @@ struct AggFinal {
     void *out[kMaxOut];
     int64_t capacity;
     int64_t *n_dev;
-    int32_t *err;                    // err[0] -> err[1], err[0] = 0
+    int32_t *err;                    // err[0] -> err[1], err[2] -> err[3], then err[0] = err[2] = 0
 };
 
 struct JoinRunsLaunch {
@@ -71,6 +71,7 @@ struct SetLaunch {
     int64_t *total;                  // device row count of the result
     uint64_t *status;                // non-null: single pass with decoupled look-back (nparts words)
     uint32_t epoch;
+    uint32_t *ctrs;                  // single pass: [0] partition counter, [1] exit counter (reset by the last CTA)
 };
 size_t set_op_smem(int ncols);
 int set_partition_rows();
@@ -90,5 +91,11 @@ int join_expand_tile();
 cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem, int grid,
                               cudaStream_t s);
 int scan_tile();
+
+// emitting scan kernel (scan_emit.cu): compacting SELECT / PROJECT chains, 1..4 branches
+size_t emit_ctl_bytes();
+int scan_emit_occupancy(int nt, int items, bool multi, size_t smem);
+cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, int items, size_t smem, int grid,
+                             cudaStream_t s);
 
 }  // namespace rw

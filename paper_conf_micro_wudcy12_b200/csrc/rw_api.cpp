@@ -100,6 +100,9 @@ struct Lowered {
     std::vector<uint32_t> out_off;
     size_t smem = 0;
     bool agg = false;
+    bool emit = false;            // compacting chain on the emitting scan kernel (scan_emit.cu)
+    int delay = 1;                // emit: evaluated tiles a compute warp may hold for their offsets
+    uint32_t warp_buf = 0;        // emit: per-warp compaction buffer bytes
     AggFinal F;
 };
 
@@ -117,7 +120,8 @@ struct rw_plan {
     int cnt_cap = 0;
     int64_t *jtot = nullptr;      // join totals: 2 int64 per join group
     int64_t *jtot_host = nullptr; // pinned mirror
-    int32_t *err = nullptr;       // [0] running domain errors, [1] last finalised
+    int32_t *err = nullptr;       // [0] running domain errors, [1] last finalised; [2] running
+                                  // declared-bound violations of narrow sums, [3] last finalised
     char *gring = nullptr;        // global compacted-tile rings (per CTA slices)
     size_t gring_cap = 0;
     std::map<int, unsigned long long *> agg_acc;
@@ -667,6 +671,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             }
         narrow_n = 0;
         narrow_flush = ((unsigned __int128)1) << 40;
+        int narrow_bits = 1;
         for (size_t q = 0; q < a.aggs.size(); q++)
             if (a.aggs[q].op != RW_SUM) {
                 L.F.req_is_sum[q] = 0;
@@ -687,14 +692,20 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 flush = std::min(flush, std::max<unsigned __int128>(1, lim / mx));
                 narrow_all64 = narrow_all64 && (slots[s].type == T_I64 || slots[s].type == T_U64);
                 if (b.lo >= 0 && b.hi < 65536) {
+                    // the device checks every narrow value against 2^narrow_bits (an OR per
+                    // row), so the flush period is taken from that power of two
+                    int bits = 1;
+                    while (((i128)1 << bits) <= b.hi) bits++;
+                    narrow_bits = std::max(narrow_bits, bits);
                     narrow_n++;
-                    narrow_flush = std::min(narrow_flush, (unsigned __int128)UINT32_MAX / mx);
+                    narrow_flush = std::min(narrow_flush, (unsigned __int128)UINT32_MAX / (((unsigned __int128)1 << narrow_bits) - 1));
                 }
                 L.F.req_is_sum[q] = 1;
                 L.F.req_acc[q] = (int16_t)(1 + ns);
                 ns++;
         }
         L.P.nagg = ns;
+        L.P.narrow_bits = narrow_bits;
         L.P.flush_rows = (int64_t)flush;
         L.F.D = a.D;
         L.F.NA = ns + 1;
@@ -937,6 +948,80 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             raise(RW_E_UNSUPPORTED, "join group exceeds the shared-memory budget");
         return;
     }
+    if (!L.agg && p->o.reserved[6] != 3) {
+        // Emitting scan kernel (scan_emit.cu): S input stages, each with its own scratch
+        // for computed columns (a stage holds its tile until the tile's offset resolves),
+        // per-thread hold words, and one compaction buffer per compute warp (resource
+        // budget, §4.3.3).  Variants: compute threads x rows per thread.
+        struct EVar { int nt, items; };
+        std::vector<EVar> vars;
+        if (p->o.reserved[4] == 3) vars.push_back({512, 8});
+        else if (p->o.reserved[4] == 2) vars.push_back({256, 4});
+        else if (p->o.reserved[4] == 4) vars.push_back({256, 8});
+        else if (p->o.reserved[4] == 5) vars.push_back({256, 16});
+        else if (nbr > 1) vars = {{256, 8}, {256, 4}};
+        else vars = {{256, 16}, {256, 8}, {256, 4}};
+        const int want_stages_e = p->o.stages > 0 ? std::min(std::max(p->o.stages, 2), 8) : 0;
+        bool direct_e = nbr == 1;
+        for (const HOp &h : ops)
+            if (h.kind == K_PRED) direct_e = false;
+        double best = -1;
+        const size_t want_ring_e = p->o.reserved[0] > 0 ? (size_t)p->o.reserved[0] * 1024 : 0;
+        for (const EVar &v : vars) {
+            const int T = v.nt * v.items;
+            layout(T);
+            const size_t SB = P.stage_bytes;
+            size_t W = 0;                     // largest compacted block (every row survives)
+            for (int b = 0; b < nbr && !direct_e; b++) {
+                size_t wb = 0;
+                for (int c = b ? P.br_out_end[b - 1] : 0; c < (int)P.br_out_end[b]; c++)
+                    wb += ((size_t)T * type_width(P.slot[P.out_slot[c]].type) + 15) / 16 * 16;
+                W = std::max(W, wb);
+            }
+            const size_t base = emit_ctl_bytes() + P.scratch_bytes;
+            for (int occ_t : {1, 2}) {
+                if (p->o.ctas_per_sm > 0 && occ_t != p->o.ctas_per_sm) continue;
+                const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
+                for (int S = 2; S <= 8; S++) {
+                    if (want_stages_e && S != want_stages_e) continue;
+                    if (base + (size_t)S * SB > per_cta) break;
+                    size_t Rb = direct_e ? 0 : (per_cta - base - (size_t)S * SB) / 128 * 128;
+                    if (want_ring_e && !direct_e) Rb = std::min(Rb, want_ring_e);
+                    if (!direct_e && Rb < W) continue;
+                    const size_t smem = base + (size_t)S * SB + Rb;
+                    if (scan_emit_occupancy(v.nt, v.items, nbr > 1, smem) < occ_t) continue;
+                    // compacted blocks the ring holds while their offsets resolve (>= 2
+                    // worst-case blocks wanted), then input bytes in flight per SM (capped:
+                    // ~64 KB per SM covers the HBM latency), then the larger tile
+                    const double q = direct_e ? 4.0 : (double)Rb / (double)W;
+                    const double inflight = std::min<double>((double)occ_t * S * SB, 160.0 * 1024);
+                    const double sc = (q >= 1.9 ? 1e9 : q * 1e8) + inflight + (double)T * 64 + S;
+                    if (sc > best) {
+                        best = sc;
+                        L.items = v.items;
+                        L.nt = v.nt;
+                        L.tile = T;
+                        L.stages = S;
+                        L.smem = smem;
+                        L.ctas = occ_t;
+                        L.out_bytes = (uint32_t)Rb;
+                    }
+                }
+            }
+        }
+        if (best < 0)
+            raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
+        layout(L.tile);
+        for (int b = 0; b < nbr; b++)
+            for (int c = b ? P.br_out_end[b - 1] : 0; c < (int)P.br_out_end[b]; c++) {
+                const int w = type_width(P.slot[P.out_slot[c]].type);
+                P.br_nw[b][w == 1 ? 0 : w == 4 ? 1 : 2]++;
+            }
+        L.emit = true;
+        L.direct = direct_e;
+        L.delay = 0;
+        return;
+    }
     // Scan kernel: S input stages (TMA ring), one scratch tile for computed
     // columns, and a byte ring of R bytes holding compacted tiles until their
     // global offset is resolved (resource budget, §4.3.3).
@@ -1078,6 +1163,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         P.agg_narrow = narrow_n;
         P.flush_rows = std::min<int64_t>(P.flush_rows, (int64_t)narrow_flush);
     }
+    // the kNarrowNT instance compiles only the 5-sum / 2-narrow / all-64-bit row loop
+    if (L.agg && L.nt == kNarrowNT && !(P.nagg == 5 && P.agg_narrow == 2 && all64 && P.agg_mode == 2))
+        raise(RW_E_STATE, "internal: Q1-specialised aggregate instance selected for another plan shape");
     if (global_ring && !L.direct) {
         size_t W = 0;
         for (int c = 0; c < P.nout; c++)
@@ -1261,7 +1349,13 @@ void run_group(ExecCtx &X, int gi)
                 L.P.out_ptr[c] = outp[c];
             L.P.out_capacity = capacity;
             TL.n_dev = n_dev;
-            cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
+            if (L.emit) {
+                TL.delay = L.delay;
+                TL.warp_buf = L.warp_buf;
+                cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream), "k_scan_emit");
+            } else {
+                cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
+            }
             p->launches++;
         }
     } else if (g.kind == G_SET) {
@@ -1293,6 +1387,7 @@ void run_group(ExecCtx &X, int gi)
             ensure_status(p, S.nparts + 1);
             S.status = p->status;
             S.epoch = next_epoch(p);
+            S.ctrs = p->ctrs;
         }
         cuda_check(set_op_launch(S, p->sms, p->stream), "k_set_op");
         p->launches += S.status ? (S.nparts > 0 ? 2 : 1) : (S.nparts > 0 ? 4 : 2);
@@ -1397,6 +1492,17 @@ void run_group(ExecCtx &X, int gi)
 
 std::vector<int> &schema_types(rw_plan *p, int node) { return p->nodes[node].types; }
 
+// errors an aggregate finalisation recorded (err[1], err[3] copied to jtot_host + 8)
+void raise_agg_errors(rw_plan *p)
+{
+    const int32_t *e = (const int32_t *)(p->jtot_host + 8);
+    if (e[1])
+        raise(RW_E_DOMAIN, std::to_string(e[1]) + " rows had a group value outside its domain");
+    if (e[3])
+        raise(RW_E_DOMAIN, std::to_string(e[3]) + " tiles held a summed value outside its declared [lo, hi] "
+                                                  "bounds (rw_plan_add_input): the 32-bit partials are not exact");
+}
+
 void check_inputs(rw_plan *p, const rw_relation_in *in, int nin)
 {
     if (nin != (int)p->inputs.size())
@@ -1446,12 +1552,10 @@ void execute(rw_plan *p, const rw_relation_in *in, int nin, int out_node, rw_rel
     out->n = -1;
     if (!out->n_dev) {
         cuda_check(cudaMemcpyAsync(p->jtot_host + 2, X.final_n_dev, 8, cudaMemcpyDeviceToHost, p->stream), "copy n");
-        cuda_check(cudaMemcpyAsync(p->jtot_host + 3, p->err + 1, 4, cudaMemcpyDeviceToHost, p->stream), "copy err");
+        cuda_check(cudaMemcpyAsync(p->jtot_host + 8, p->err, 16, cudaMemcpyDeviceToHost, p->stream), "copy err");
         cuda_check(cudaStreamSynchronize(p->stream), "sync");
         out->n = p->jtot_host[2];
-        const int32_t derr = ((int32_t *)(p->jtot_host + 3))[0];
-        if (derr)
-            raise(RW_E_DOMAIN, std::to_string(derr) + " rows had a group value outside its domain");
+        raise_agg_errors(p);
         if (out->n > out->capacity)
             raise(RW_E_CAPACITY, "output needs " + std::to_string(out->n) + " rows, capacity " +
                                      std::to_string(out->capacity));
@@ -1556,7 +1660,13 @@ void execute_multi(rw_plan *p, const rw_relation_in *in, int nin, const int32_t 
         if (k == 0) TL.n_dev = nd;
         else TL.br_n_dev[k] = nd;
     }
-    cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain<multi>");
+    if (L.emit) {
+        TL.delay = L.delay;
+        TL.warp_buf = L.warp_buf;
+        cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream), "k_scan_emit<multi>");
+    } else {
+        cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain<multi>");
+    }
     p->launches++;
     bool any_sync = false;
     for (int k = 0; k < nout; k++)
@@ -1704,10 +1814,8 @@ bool execute_host_streamed(rw_plan *p, const rw_relation_in *in, int nin, int ou
         cuda_check(cudaStreamSynchronize(sd), "sync");
         cuda_check(cudaStreamSynchronize(p->stream), "sync");
         if (agg) {
-            cuda_check(cudaMemcpy(p->jtot_host + 3, p->err + 1, 4, cudaMemcpyDeviceToHost), "copy err");
-            const int32_t derr = ((int32_t *)(p->jtot_host + 3))[0];
-            if (derr)
-                raise(RW_E_DOMAIN, std::to_string(derr) + " rows had a group value outside its domain");
+            cuda_check(cudaMemcpy(p->jtot_host + 8, p->err, 16, cudaMemcpyDeviceToHost), "copy err");
+            raise_agg_errors(p);
         }
         out->n = total;
         p->launches = launches;
@@ -1781,6 +1889,9 @@ std::string explain(rw_plan *p, int out_node)
             Lowered L;
             std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
             lower(p, g, st, L);
+            if (L.emit)
+                s << " | emitting kernel k_scan_emit<" << L.nt << "," << L.items << ">"
+                  << (L.direct ? ", direct (no SELECT)" : "");
             s << " | tile " << L.tile << " rows (" << L.items << "/thread), stages " << L.stages << ", out ring " << L.out_bytes << " B"
               << ", smem " << L.smem
               << " B, CTAs/SM " << L.ctas << ", slots " << L.P.nslots << " (" << L.P.nin << " loaded), ops "
@@ -1882,7 +1993,7 @@ rw_status rw_plan_create(rw_plan **out, const rw_plan_opts *opts)
         p->jtot = (int64_t *)dev_alloc(p, 64);
         p->err = (int32_t *)dev_alloc(p, 64);
         cuda_check(cudaMemsetAsync(p->err, 0, 64, p->stream), "memset");
-        cuda_check(cudaMallocHost(&p->jtot_host, 64), "cudaMallocHost");
+        cuda_check(cudaMallocHost(&p->jtot_host, 128), "cudaMallocHost");
         ensure_status(p, 4096);
         cuda_check(cudaStreamSynchronize(p->stream), "sync");
     } catch (...) {

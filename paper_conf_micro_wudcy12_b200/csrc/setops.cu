@@ -132,9 +132,24 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
     __shared__ int32_t wcnt[kThreads / 32 + 1];
     __shared__ int32_t nbr[4];                            // has_pred, pred_is_x, has_succ, succ_is_x
     __shared__ int64_t pbase;                             // single pass: the partition's output offset
+    __shared__ int64_t pclaim;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     constexpr int nc = NC;
-    for (int64_t p = blockIdx.x; p < S.nparts; p += gridDim.x) {
+    // single pass (look-back): partitions are claimed in order with a global atomic, so
+    // every partition a CTA waits for has been claimed by a running CTA (no assumption
+    // that the whole grid is resident); the count pass walks them statically
+    const bool claim = WRITE && S.status != nullptr;
+    for (int64_t it = 0;; ++it) {
+        int64_t p = (int64_t)blockIdx.x + it * gridDim.x;
+        if (claim) {
+            __syncthreads();
+            if (tid == 0)
+                pclaim = (int64_t)atomicAdd(&S.ctrs[0], 1u);
+            __syncthreads();
+            p = pclaim;
+        }
+        if (p >= S.nparts)
+            break;
         const int64_t d0 = p * kSetT, d1 = min(d0 + kSetT, S.nx + S.ny);
         const int64_t i0 = S.split[p], i1 = S.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
         const int nX = (int)(i1 - i0), nY = (int)(j1 - j0), m = (int)(d1 - d0);
@@ -248,9 +263,7 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
         }
         int64_t o;
         if (S.status) {
-            // single pass: decoupled look-back over the partitions (every CTA of the
-            // grid is resident and walks its partitions in increasing order, so the
-            // predecessors a partition waits for always make progress)
+            // single pass: decoupled look-back over the partitions (claimed in order)
             if (warp == 0) {
                 const uint64_t excl = lookback_warp(S.status, p, (uint64_t)tot, S.epoch);
                 if (lane == 0) {
@@ -277,6 +290,8 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
             o++;
         }
     }
+    if (claim)
+        cta_exit_reset(S.ctrs);
 }
 
 // exclusive scan of the per-partition counts (one CTA) and the total
