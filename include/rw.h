@@ -140,7 +140,13 @@ void rw_plan_destroy(rw_plan *plan);
 /* Declare an input relation: ncols attribute types; nkey_sorted = number of leading
  * columns the data is sorted on (lexicographic, ascending in each type; 0 = unsorted;
  * A6).  lo/hi (optional, NULL = full type range): caller-promised inclusive value
- * bounds per column, used by interval analysis (aggregate flush period, strict mode). */
+ * bounds per column, used by interval analysis (aggregate flush period, strict mode).
+ * The bounds are a correctness precondition of the aggregate terminal: sums of columns
+ * declared within [0, 2^16) accumulate in 32-bit partials flushed on a period derived
+ * from the bounds.  A summed narrow value outside [0, 2^b) (b = bits of the declared
+ * upper bound) is detected and reported as RW_E_DOMAIN by the execute that finalises
+ * the aggregate; wide sums keep 64-bit partials flushed before they could overflow
+ * under the declared bounds (undefined sums if data exceed them by orders of magnitude). */
 rw_status rw_plan_add_input(rw_plan *plan, int32_t ncols, const int32_t *types, int32_t nkey_sorted,
                             const int64_t *lo, const int64_t *hi, int32_t *node);
 

@@ -1395,6 +1395,10 @@ void run_group(ExecCtx &X, int gi)
         const Node &jn = p->nodes[g.join];
         Rel lr = rel_of(X, g.jl >= 0 ? g.jl : jn.left), rr = rel_of(X, g.jr >= 0 ? g.jr : jn.right);
         const int64_t nl = host_count(X, lr), nr = host_count(X, rr);
+        // run records and the expansion cache hold 32-bit row indices: a materialised
+        // intermediate above 2^32 rows must be sharded across ranks
+        if (nl > (int64_t)UINT32_MAX || nr > (int64_t)UINT32_MAX)
+            raise(RW_E_UNSUPPORTED, "join input above 2^32 rows per GPU (materialised intermediate): shard across ranks");
         const int kt = lr.types[0];
         // phase 1: run records
         const int64_t T1 = 2048;

@@ -101,7 +101,8 @@ def choose_splitters(local_keys: Sequence[Tuple[torch.Tensor, str]], world: int,
             pos = torch.linspace(0, n - 1, min(samples, n)).round().to(torch.int64).to(keys.device)
             parts.append(key_values(keys.index_select(0, pos), kt))
     mine = torch.cat(parts) if parts else torch.zeros(0, dtype=torch.int64, device=local_keys[0][0].device)
-    # pad to a fixed size so all_gather shapes agree; -1 marks padding (keys are >= 0 here)
+    # fixed-size buffer so all_gather shapes agree: buf[0] = number of samples, then the
+    # samples (key values as int64; i32/i64 keys may be negative), the rest unused
     width = samples * len(local_keys)
     buf = torch.full((width + 1,), 0, dtype=torch.int64, device=mine.device)
     buf[0] = mine.numel()

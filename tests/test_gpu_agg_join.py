@@ -232,3 +232,22 @@ def test_n2_signed_keys():
     got, plan = run_gpu(spec, ins, capacity=2_000_000)
     assert_same(got, run_oracle(spec, ins))
     assert "key SELECT" in plan.explain(plan.out_id)
+
+
+def test_q1_declared_bound_violation_is_reported():
+    """A summed narrow column (disc, declared in [0, 10]) holding a value outside its
+    declared bounds: the 32-bit partials could be inexact, so the execute reports
+    RW_E_DOMAIN instead of returning silently wrong sums (rw.h, rw_plan_add_input)."""
+    from paper_conf_micro_wudcy12_b200 import rw
+    spec = workloads.c4_spec()
+    ins = workloads.c4_inputs(50_001, device=DEV, cfg=0x95)
+    ins["lineitem"][3][12345] = 1000          # disc far above its declared hi = 10
+    with pytest.raises(rw.RwError) as e:
+        run_gpu(spec, ins, capacity=6)
+    assert "declared" in str(e.value)
+    # the same data with the bound not declared narrow: exact, no error
+    spec2 = workloads.c4_spec()
+    spec2["inputs"]["lineitem"]["hi"] = list(spec2["inputs"]["lineitem"]["hi"])
+    spec2["inputs"]["lineitem"]["hi"][3] = 1 << 40
+    got, _ = run_gpu(spec2, ins, capacity=6)
+    assert_same(got, run_oracle(spec2, ins))
