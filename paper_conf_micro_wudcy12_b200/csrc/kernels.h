@@ -92,6 +92,61 @@ cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const Joi
                               cudaStream_t s);
 int scan_tile();
 
+// ---- join2.cu: run matching (single pass) and the fused expansion ----
+struct KeySrc {                      // order-preserving image of the leading nkey (<= 2) key columns
+    const void *col[2];
+    uint8_t type[2];
+    int32_t ncol;
+    const void *img;                 // non-null: precomputed images (uint32 / uint64 array)
+};
+
+struct MatchLaunch {
+    KeySrc A, B;
+    int64_t nA, nB, nparts;          // nparts: launched partitions (an upper bound when nA_dev is set)
+    const int64_t *nA_dev;           // chained match: A's row count on the device (else null: nA)
+    int64_t *split;                  // nparts + 1 merge-path splits
+    const uint64_t *wA;              // chained match: weight of every A element (first-level run), else null
+    // chained (3-input) composition: A element ga = first-level run, whose (s0, s1, len1) are copied
+    int32_t chain1;
+    const uint32_t *c_s0, *c_s1, *c_len1;
+    // outputs: one record per matched key, in key order (capacity cap_runs + 8 padded)
+    uint32_t *s0, *s1, *len1, *s2, *len2, *len0;
+    void *key_out;                   // optional key images of the runs (chaining)
+    uint64_t *w_out;                 // optional lenA * lenB per run (chaining)
+    uint64_t *off;                   // exclusive prefix of the runs' candidate counts
+    int64_t cap_runs;
+    uint64_t *st_runs, *st_cands;    // look-back status words, nparts each
+    uint32_t ep_runs, ep_cands;
+    uint32_t *ctrs;
+    int64_t *totals;                 // [0] runs, [1] candidates
+    int32_t nkpred;                  // fused key SELECT atoms (N2): on the key image
+    uint8_t kop[kMaxKeyPreds];
+    uint64_t kpk[kMaxKeyPreds];
+};
+
+struct JoinEmit {
+    const int64_t *tile_run;         // first run of every tile (+ entry ntiles = nruns - 1)
+    const uint64_t *off;
+    const uint32_t *s0, *s1, *len1, *s2, *len2;
+    uint32_t rec_cap4, rec_stage_bytes;
+    int32_t ncols;                   // live join columns gathered into input slots 0..ncols-1
+    const void *src[kMaxSlots];
+    uint8_t w[kMaxSlots];
+    uint8_t side[kMaxSlots];         // 0: first input (row s0 + i), 1: second (s1 + j), 2: third (s2 + k)
+    int32_t regpath;                 // gathers through registers (<= 4 live columns, all 1 or 4 bytes)
+};
+
+int match_partition();
+cudaError_t match_launch(const MatchLaunch &M, bool wide, cudaStream_t st);
+cudaError_t jtiles_launch(const uint64_t *off, const int64_t *totals, int64_t T, int64_t cap_tiles, int64_t *tile_run,
+                          int32_t *overflow, int sms, cudaStream_t st);
+uint32_t join_rec_cap4(int T);
+size_t join_rec_stage_bytes(int ways, int T);
+size_t join_emit_ctl_bytes();
+int join_emit_occupancy(int items, int ways, size_t smem);
+cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int items, int ways, size_t smem,
+                             int grid, cudaStream_t s);
+
 // emitting scan kernel (scan_emit.cu): compacting SELECT / PROJECT chains, 1..4 branches
 size_t emit_ctl_bytes();
 int scan_emit_occupancy(int nt, int items, bool multi, size_t smem);

@@ -55,6 +55,9 @@ struct Group {
     // join then reads their source relations (jl, jr) directly
     std::vector<int> pre;            // absorbed SELECT nodes
     int jl = -1, jr = -1;            // relations feeding the join (after absorption)
+    // 3-input group (JOIN -> JOIN on the same key, Fig. 14(b)): join_in = the inner JOIN
+    // (inputs jl, jr), `join` the outer one (inner output, jc)
+    int join_in = -1, jc = -1;
 };
 
 Interval type_range(int t);

@@ -115,6 +115,7 @@ struct rw_plan {
     // persistent scratch
     uint64_t *status = nullptr;
     int64_t status_cap = 0;
+    int64_t status_used = 0;      // join groups: words handed out of `status` in this group
     uint32_t *ctrs = nullptr;     // 2 counters
     int64_t *cnt = nullptr;       // per-group row counts (grown)
     int cnt_cap = 0;
@@ -304,9 +305,9 @@ int dep_group(const rw_plan *p, int id, Grouping &G)
 // SELECTs on the key column only, directly upstream of a JOIN input (single consumer):
 // they keep or drop whole key runs, so the join's run matching applies them and the
 // join reads their source relation (CTA dependence fused, Fig. 13; N2).
-int absorb_key_selects(const rw_plan *p, int nd, const Grouping &G, Group &g, int &npred)
+int absorb_key_selects(const rw_plan *p, int nd, const Grouping &G, Group &g, int &npred, int nkey)
 {
-    if (!p->o.fuse)
+    if (!p->o.fuse || nkey != 1)
         return nd;
     while (p->nodes[nd].kind == N_SELECT && G.consumers[nd] == 1) {
         const Node &sn = p->nodes[nd];
@@ -320,6 +321,34 @@ int absorb_key_selects(const rw_plan *p, int nd, const Grouping &G, Group &g, in
         nd = sn.in;
     }
     return nd;
+}
+
+// A JOIN group (§4.3.2): key SELECTs on its inputs are absorbed into the
+// run matching (N2), and a left input that is itself a single-consumer JOIN on the same
+// key (CTA dependence, Fig. 8(b); pattern (b) of Fig. 14) is absorbed too: the
+// group then joins three inputs in one expansion (mixed radix (i, j, k)).
+void setup_join(const rw_plan *p, int jid, Grouping &G, Group &g)
+{
+    g.kind = G_JOIN;
+    g.join = jid;
+    const Node &j = p->nodes[jid];
+    int np = 0;
+    const int left = j.left;
+    const Node &ln = p->nodes[left];
+    if (p->o.fuse && ln.kind == N_JOIN && G.consumers[left] == 1 && ln.nkey == j.nkey && p->o.reserved[6] != 5) {
+        g.join_in = left;
+        g.jl = absorb_key_selects(p, ln.left, G, g, np, j.nkey);
+        g.jr = absorb_key_selects(p, ln.right, G, g, np, j.nkey);
+        g.jc = absorb_key_selects(p, j.right, G, g, np, j.nkey);
+    } else {
+        g.jl = absorb_key_selects(p, left, G, g, np, j.nkey);
+        g.jr = absorb_key_selects(p, j.right, G, g, np, j.nkey);
+    }
+    for (int src : {g.jl, g.jr, g.jc}) {
+        if (src < 0) continue;
+        const int d = dep_group(p, src, G);
+        if (d >= 0) g.deps.push_back(d);
+    }
 }
 
 int make_group(const rw_plan *p, int id, Grouping &G)
@@ -356,14 +385,7 @@ int make_group(const rw_plan *p, int id, Grouping &G)
         return G.produced_by[id] = (int)G.groups.size() - 1;
     }
     if (n.kind == N_JOIN) {
-        g.kind = G_JOIN;
-        g.join = id;
-        int np = 0;
-        g.jl = absorb_key_selects(p, n.left, G, g, np);
-        g.jr = absorb_key_selects(p, n.right, G, g, np);
-        int a = dep_group(p, g.jl, G), b = dep_group(p, g.jr, G);
-        if (a >= 0) g.deps.push_back(a);
-        if (b >= 0) g.deps.push_back(b);
+        setup_join(p, id, G, g);
         G.groups.push_back(g);
         return G.produced_by[id] = (int)G.groups.size() - 1;
     }
@@ -393,15 +415,7 @@ int make_group(const rw_plan *p, int id, Grouping &G)
     g.chain = chain;
     if (fuse && p->nodes[src].kind == N_JOIN && G.consumers[src] == 1) {
         // JOIN -> SELECT/PROJECT: fused into the join expansion (CTA dependence)
-        g.kind = G_JOIN;
-        g.join = src;
-        const Node &j = p->nodes[src];
-        int np = 0;
-        g.jl = absorb_key_selects(p, j.left, G, g, np);
-        g.jr = absorb_key_selects(p, j.right, G, g, np);
-        int a = dep_group(p, g.jl, G), b = dep_group(p, g.jr, G);
-        if (a >= 0) g.deps.push_back(a);
-        if (b >= 0) g.deps.push_back(b);
+        setup_join(p, src, G, g);
     } else {
         g.kind = G_SCAN;
         g.source = src;
@@ -916,36 +930,53 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         raise(RW_E_UNSUPPORTED, "aggregate needs more than 4096 accumulators");
 
     if (g.kind == G_JOIN) {
-        // join expansion runs inside the warp-specialised chain kernel: one stage (the
-        // compute warps fill it themselves), the run-record cache, and the output ring
-        const int T = join_expand_tile();
-        layout(T);
-        size_t W = 0;
-        for (int c = 0; c < P.nout; c++)
-            W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
-        const size_t base = scan_ctl_bytes() + P.scratch_bytes + join_run_cache_bytes() + P.stage_bytes;
+        // join expansion (join2.cu k_join_emit): S stages of run records (TMA), two
+        // gathered tiles (parity), scratch, and the compacted-output ring (resource
+        // budget, §4.3.3)
+        const int ways = g.join_in >= 0 ? 3 : 2;
         bool found = false;
-        for (int occ_t : {2, 1}) {
-            if (p->o.ctas_per_sm > 0 && occ_t != p->o.ctas_per_sm) continue;
-            const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
-            if (base + W > per_cta) continue;
-            size_t Rb = (per_cta - base) / 128 * 128;
-            if (p->o.reserved[0] > 0) Rb = std::min(Rb, (size_t)p->o.reserved[0] * 1024);
-            if (Rb < W || (occ_t == 2 && Rb < W * 19 / 10)) continue;
-            const size_t smem = base + Rb;
-            if (chain_occupancy(2, kThreads, kJoinItems, smem) < occ_t) continue;
-            L.items = kJoinItems;
-            L.nt = kThreads;
-            L.tile = T;
-            L.stages = 1;
-            L.out_bytes = (uint32_t)Rb;
-            L.smem = smem;
-            L.ctas = occ_t;
-            found = true;
-            break;
+        double best = -1;
+        for (int items : {8, 4}) {
+            if (p->o.reserved[5] > 0 && items != p->o.reserved[5]) continue;
+            const int T = kThreads * items;
+            layout(T);
+            size_t W = 0;
+            for (int c = 0; c < P.nout; c++)
+                W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+            const size_t RS = join_rec_stage_bytes(ways, T);
+            const size_t base = join_emit_ctl_bytes() + 2 * (size_t)P.stage_bytes + (size_t)ways * T * 4 +
+                                (size_t)T * 2 + P.scratch_bytes;
+            for (int S = 2; S <= 3; S++) {
+                if (p->o.stages > 0 && S != p->o.stages) continue;
+                const size_t per_cta = kSmemLimit;
+                if (base + S * RS + W > per_cta) continue;
+                size_t Rb = (per_cta - base - S * RS) / 128 * 128;
+                if (p->o.reserved[0] > 0) Rb = std::min(Rb, (size_t)p->o.reserved[0] * 1024);
+                if (Rb < W) continue;
+                const size_t smem = base + S * RS + Rb;
+                if (join_emit_occupancy(items, ways, smem) < 1) continue;
+                const double q = (double)Rb / (double)W;
+                const double sc = (q >= 2.0 ? 1e9 : q * 1e8) + T * 1e3 + S;
+                if (sc > best) {
+                    best = sc;
+                    L.items = items;
+                    L.nt = kThreads;
+                    L.tile = T;
+                    L.stages = S;
+                    L.out_bytes = (uint32_t)Rb;
+                    L.smem = smem;
+                    L.ctas = 1;
+                    found = true;
+                }
+            }
         }
         if (!found)
             raise(RW_E_UNSUPPORTED, "join group exceeds the shared-memory budget");
+        layout(L.tile);
+        for (int c = 0; c < P.nout; c++) {
+            const int w = type_width(P.slot[P.out_slot[c]].type);
+            P.br_nw[0][w == 1 ? 0 : w == 4 ? 1 : 2]++;
+        }
         return;
     }
     if (!L.agg && p->o.reserved[6] != 3) {
@@ -1254,6 +1285,217 @@ unsigned long long *agg_buffer(rw_plan *p, int node, size_t words)
     return b;
 }
 
+// order-preserving key images of a relation's leading nkey columns (join2.cu KeySrc)
+KeySrc key_src(const Rel &r, int nkey)
+{
+    KeySrc k{};
+    k.ncol = nkey;
+    for (int c = 0; c < nkey; c++) {
+        k.col[c] = r.cols[c];
+        k.type[c] = (uint8_t)r.types[c];
+    }
+    return k;
+}
+
+// image of a key constant (for key SELECTs fused into the matching): as col_img
+uint64_t key_const_img(int type, int64_t v)
+{
+    const uint64_t u = (uint64_t)wrap_to(type, v);
+    switch (type) {
+    case T_I32: return (uint32_t)u ^ 0x80000000u;
+    case T_U32: return (uint32_t)u;
+    case T_I64: return u ^ 0x8000000000000000ull;
+    case T_U64: return u;
+    default: return (uint8_t)u;
+    }
+}
+
+// JOIN group (2 or 3 inputs): single-pass run matching (chained for 3 inputs), tile
+// index, fused expansion.  No host synchronisation when the group writes the caller's
+// output (its capacity is given); a materialised join intermediate reads its row count.
+void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void *> &outp, int64_t &capacity,
+                    int64_t *&n_dev)
+{
+    rw_plan *p = X.p;
+    const Node &jn = p->nodes[g.join];
+    const Node &outn = p->nodes[g.out];
+    const bool three = g.join_in >= 0;
+    const int nkey = jn.nkey;
+    Rel ra = rel_of(X, g.jl), rb = rel_of(X, g.jr);
+    Rel rc;
+    if (three) rc = rel_of(X, g.jc);
+    const int64_t na = host_count(X, ra), nb = host_count(X, rb), nc = three ? host_count(X, rc) : 0;
+    // run records and the expansion hold 32-bit row indices
+    if (na > (int64_t)UINT32_MAX || nb > (int64_t)UINT32_MAX || nc > (int64_t)UINT32_MAX)
+        raise(RW_E_UNSUPPORTED, "join input above 2^32 rows per GPU (materialised intermediate): shard across ranks");
+    int kbytes = 0;
+    for (int c = 0; c < nkey; c++)
+        kbytes += type_width(ra.types[c]) == 8 ? 8 : 4;
+    if (kbytes > 8)
+        raise(RW_E_UNSUPPORTED, "join keys wider than 8 bytes (nkey = 2 needs 32-bit key columns)");
+    const bool wide = kbytes > 4;
+    const int mt = match_partition();
+    // ---- run matching ----
+    auto status_at = [&](int64_t words) {
+        uint64_t *st = p->status + p->status_used;
+        p->status_used += words;
+        return st;
+    };
+    const int64_t nparts1 = (na + nb + mt - 1) / mt;
+    const int64_t cap1 = std::max<int64_t>(1, std::min(na, nb));
+    const int64_t nparts2 = three ? (cap1 + nc + mt - 1) / mt : 0;
+    const int64_t cap2 = three ? std::max<int64_t>(1, std::min(cap1, nc)) : 0;
+    const int T = 0;   // set below from the lowering
+    (void)T;
+    Lowered L;
+    lower(p, g, jn.types, L);
+    const int64_t T2 = L.tile;
+    const double maxc = three ? (double)na * (double)nb * (double)nc : (double)na * (double)nb;
+    // tile index capacity: every candidate when that is below 2^34 (no host sync), else
+    // the exact count after a synchronisation
+    const bool exact_tiles = maxc > 17179869184.0;
+    p->status_used = 0;
+    int64_t status_need = 2 * (nparts1 + 1) + 2 * (nparts2 + 1) + 16;
+    int64_t cap_tiles = exact_tiles ? 0 : (int64_t)(maxc / (double)T2) + 2;
+    ensure_status(p, status_need + cap_tiles + 1);
+    auto mk_u32 = [&](int64_t n) { return (uint32_t *)temp_alloc(p, (size_t)(n + 8) * 4); };
+    auto mk_u64 = [&](int64_t n) { return (uint64_t *)temp_alloc(p, (size_t)(n + 8) * 8); };
+    int64_t *tot1 = p->jtot, *tot2 = p->jtot + 2;
+    cuda_check(cudaMemsetAsync(p->jtot, 0, 32, p->stream), "memset totals");
+    MatchLaunch M{};
+    M.A = key_src(ra, nkey);
+    M.B = key_src(rb, nkey);
+    M.nA = na;
+    M.nB = nb;
+    M.nparts = nparts1;
+    M.split = (int64_t *)temp_alloc(p, (size_t)(nparts1 + 1) * 8);
+    M.cap_runs = cap1;
+    M.s0 = mk_u32(cap1);
+    M.s1 = mk_u32(cap1);
+    M.len1 = mk_u32(cap1);
+    M.off = mk_u64(cap1);
+    if (three) {
+        M.key_out = temp_alloc(p, (size_t)(cap1 + 8) * (wide ? 8 : 4));
+        M.w_out = mk_u64(cap1);
+    }
+    M.st_runs = status_at(nparts1 + 1);
+    M.st_cands = status_at(nparts1 + 1);
+    M.ep_runs = next_epoch(p);
+    M.ep_cands = next_epoch(p);
+    M.ctrs = p->ctrs;
+    M.totals = tot1;
+    for (int sid : g.pre)
+        for (const rw_pred &a : p->nodes[sid].preds) {
+            if (nkey != 1)
+                raise(RW_E_STATE, "internal: key SELECT fused into a multi-column key");
+            M.kop[M.nkpred] = (uint8_t)a.op;
+            M.kpk[M.nkpred] = key_const_img(ra.types[0], a.rhs_const);
+            M.nkpred++;
+        }
+    cuda_check(match_launch(M, wide, p->stream), "k_jmatch");
+    p->launches += nparts1 > 0 ? 2 : 1;
+    JoinEmit XJ{};
+    const int64_t *totals = tot1;
+    if (three) {
+        MatchLaunch M2{};
+        M2.A.img = M.key_out;
+        M2.A.ncol = 1;
+        M2.B = key_src(rc, nkey);
+        M2.nA = cap1;
+        M2.nA_dev = tot1;                    // first-level runs (device)
+        M2.nB = nc;
+        M2.nparts = nparts2;
+        M2.split = (int64_t *)temp_alloc(p, (size_t)(nparts2 + 1) * 8);
+        M2.wA = M.w_out;
+        M2.chain1 = 1;
+        M2.c_s0 = M.s0;
+        M2.c_s1 = M.s1;
+        M2.c_len1 = M.len1;
+        M2.cap_runs = cap2;
+        M2.s0 = mk_u32(cap2);
+        M2.s1 = mk_u32(cap2);
+        M2.len1 = mk_u32(cap2);
+        M2.s2 = mk_u32(cap2);
+        M2.len2 = mk_u32(cap2);
+        M2.off = mk_u64(cap2);
+        M2.st_runs = status_at(nparts2 + 1);
+        M2.st_cands = status_at(nparts2 + 1);
+        M2.ep_runs = next_epoch(p);
+        M2.ep_cands = next_epoch(p);
+        M2.ctrs = p->ctrs;
+        M2.totals = tot2;
+        cuda_check(match_launch(M2, wide, p->stream), "k_jmatch (chained)");
+        p->launches += nparts2 > 0 ? 2 : 1;
+        XJ.off = M2.off;
+        XJ.s0 = M2.s0;
+        XJ.s1 = M2.s1;
+        XJ.len1 = M2.len1;
+        XJ.s2 = M2.s2;
+        XJ.len2 = M2.len2;
+        totals = tot2;
+    } else {
+        XJ.off = M.off;
+        XJ.s0 = M.s0;
+        XJ.s1 = M.s1;
+        XJ.len1 = M.len1;
+    }
+    // ---- output: the caller's (capacity given) or a materialised intermediate ----
+    int64_t total_host = -1;
+    if (gi != X.final_group || exact_tiles) {
+        cuda_check(cudaMemcpyAsync(p->jtot_host, totals, 16, cudaMemcpyDeviceToHost, p->stream), "copy totals");
+        cuda_check(cudaStreamSynchronize(p->stream), "sync after join runs");
+        total_host = p->jtot_host[1];
+        if (exact_tiles)
+            cap_tiles = (total_host + T2 - 1) / T2 + 2;
+    }
+    if (exact_tiles)
+        ensure_status(p, p->status_used + cap_tiles + 1);
+    make_output(X, gi, outn.types, gi == X.final_group ? X.out->capacity : total_host, o, outp, capacity, n_dev);
+    // ---- tile index ----
+    int64_t *tile_run = (int64_t *)temp_alloc(p, (size_t)std::max<int64_t>(cap_tiles, 2) * 8);
+    int32_t *ovf = (int32_t *)(p->err + 8);
+    cuda_check(jtiles_launch(XJ.off, totals, T2, cap_tiles, tile_run, ovf, p->sms, p->stream), "k_jtiles");
+    p->launches++;
+    // ---- expansion fused with the downstream chain ----
+    XJ.tile_run = tile_run;
+    XJ.rec_cap4 = join_rec_cap4((int)T2);
+    XJ.rec_stage_bytes = (uint32_t)join_rec_stage_bytes(three ? 3 : 2, (int)T2);
+    // join output column -> (input, column): (key, A rest, B rest[, C rest])
+    const int nac = (int)ra.types.size(), nbc = (int)rb.types.size();
+    XJ.ncols = L.P.nin;
+    for (int i = 0; i < L.P.nin; i++) {
+        const int c = L.in_src[i];
+        int side, col;
+        if (c < nac) { side = 0; col = c; }
+        else if (c < nac + nbc - nkey) { side = 1; col = c - nac + nkey; }
+        else { side = 2; col = c - (nac + nbc - nkey) + nkey; }
+        const Rel &src = side == 0 ? ra : side == 1 ? rb : rc;
+        XJ.src[i] = src.cols[col];
+        XJ.side[i] = (uint8_t)side;
+        XJ.w[i] = (uint8_t)type_width(src.types[col]);
+    }
+    XJ.regpath = XJ.ncols <= 4;
+    for (int i = 0; i < XJ.ncols; i++)
+        if (XJ.w[i] == 8) XJ.regpath = 0;
+    if (p->o.reserved[6] == 6) XJ.regpath = 0;        // diagnostics: cp.async gathers
+    for (size_t c = 0; c < outp.size(); c++)
+        L.P.out_ptr[c] = outp[c];
+    L.P.out_capacity = capacity;
+    TileLaunch TL{};
+    TL.n_ptr = totals + 1;
+    TL.stages = L.stages;
+    TL.epoch = next_epoch(p);
+    TL.status = status_at(cap_tiles + 1);
+    TL.ctrs = p->ctrs;
+    TL.n_dev = n_dev;
+    TL.err = p->err;
+    TL.out_bytes = L.out_bytes;
+    TL.dbg = p->o.reserved[1];
+    const int grid = p->sms * L.ctas;
+    cuda_check(join_emit_launch(L.P, TL, XJ, L.items, three ? 3 : 2, L.smem, grid, p->stream), "k_join_emit");
+    p->launches++;
+}
+
 void run_group(ExecCtx &X, int gi)
 {
     if (X.done[gi])
@@ -1392,103 +1634,7 @@ void run_group(ExecCtx &X, int gi)
         cuda_check(set_op_launch(S, p->sms, p->stream), "k_set_op");
         p->launches += S.status ? (S.nparts > 0 ? 2 : 1) : (S.nparts > 0 ? 4 : 2);
     } else {
-        const Node &jn = p->nodes[g.join];
-        Rel lr = rel_of(X, g.jl >= 0 ? g.jl : jn.left), rr = rel_of(X, g.jr >= 0 ? g.jr : jn.right);
-        const int64_t nl = host_count(X, lr), nr = host_count(X, rr);
-        // run records and the expansion cache hold 32-bit row indices: a materialised
-        // intermediate above 2^32 rows must be sharded across ranks
-        if (nl > (int64_t)UINT32_MAX || nr > (int64_t)UINT32_MAX)
-            raise(RW_E_UNSUPPORTED, "join input above 2^32 rows per GPU (materialised intermediate): shard across ranks");
-        const int kt = lr.types[0];
-        // phase 1: run records
-        const int64_t T1 = 2048;
-        const int64_t nparts = (nl + nr + T1 - 1) / T1;
-        const int64_t cap_runs = std::max<int64_t>(1, std::min(nl, nr));
-        JoinRunsLaunch J{};
-        J.lkey = lr.cols[0];
-        J.rkey = rr.cols[0];
-        J.nl = nl;
-        J.nr = nr;
-        J.nparts = nparts;
-        J.s = (uint32_t *)temp_alloc(p, cap_runs * 4);
-        J.lenL = (uint32_t *)temp_alloc(p, cap_runs * 4);
-        J.lo = (uint32_t *)temp_alloc(p, cap_runs * 4);
-        J.lenR = (uint32_t *)temp_alloc(p, cap_runs * 4);
-        J.off = (uint64_t *)temp_alloc(p, cap_runs * 8);
-        J.cap_runs = cap_runs;
-        ensure_status(p, 2 * nparts + 2);
-        J.status_runs = p->status;
-        J.status_outs = p->status + nparts + 1;
-        J.epoch_runs = next_epoch(p);
-        J.epoch_outs = next_epoch(p);
-        J.ctrs = p->ctrs;
-        J.totals = p->jtot;
-        J.split = (int64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
-        J.pruns = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
-        J.pouts = (uint64_t *)temp_alloc(p, (size_t)(nparts + 1) * 8);
-        J.nkpred = 0;
-        for (int sid : g.pre)
-            for (const rw_pred &a : p->nodes[sid].preds) {
-                J.kop[J.nkpred] = (uint8_t)a.op;
-                J.kpk[J.nkpred] = (int64_t)wrap_to(kt, a.rhs_const);
-                J.nkpred++;
-            }
-        const size_t smem1 = join_runs_smem(kt);
-        const int occ1 = std::max(1, chain_occupancy(3, kThreads, 8, smem1));
-        const int grid1 = (int)std::max<int64_t>(1, std::min<int64_t>(nparts, (int64_t)p->sms * occ1));
-        cuda_check(join_runs_launch(J, kt, smem1, grid1, p->stream), "k_join_runs");
-        p->launches += 4;
-        cuda_check(cudaMemcpyAsync(p->jtot_host, p->jtot, 16, cudaMemcpyDeviceToHost, p->stream), "copy totals");
-        cuda_check(cudaStreamSynchronize(p->stream), "sync after join runs");
-        const int64_t nruns = p->jtot_host[0], total = p->jtot_host[1];
-        // phase 2: expansion fused with the downstream chain
-        std::vector<int> jtypes = jn.types;
-        Lowered L;
-        lower(p, g, jtypes, L);
-        make_output(X, gi, outn.types, total, o, outp, capacity, n_dev);
-        const int64_t T2 = join_expand_tile();
-        const int64_t ntiles = (total + T2 - 1) / T2;
-        int64_t *tile_run = (int64_t *)temp_alloc(p, (size_t)std::max<int64_t>(ntiles, 1) * 8);
-        cuda_check(tile_runs_launch(J.off, nruns, ntiles, T2, tile_run, p->stream), "k_tile_runs");
-        if (ntiles > 0) p->launches++;
-        JoinExpand XJ{};
-        XJ.s = J.s;
-        XJ.lo = J.lo;
-        XJ.lenR = J.lenR;
-        XJ.off = J.off;
-        XJ.tile_run = tile_run;
-        XJ.nruns = nruns;
-        const int nlc = (int)lr.types.size();
-        XJ.ncols = L.P.nin;
-        for (int i = 0; i < L.P.nin; i++) {
-            const int c = L.in_src[i];
-            if (c < nlc) {
-                XJ.src[i] = lr.cols[c];
-                XJ.from_right[i] = 0;
-            } else {
-                XJ.src[i] = rr.cols[c - nlc + jn.nkey];
-                XJ.from_right[i] = 1;
-            }
-            XJ.dst_slot[i] = (int16_t)i;
-        }
-        for (size_t c = 0; c < outp.size(); c++)
-            L.P.out_ptr[c] = outp[c];
-        L.P.out_capacity = capacity;
-        ensure_status(p, ntiles + 1);
-        TileLaunch TL{};
-        TL.n = total;
-        TL.stages = 1;
-        TL.epoch = next_epoch(p);
-        TL.status = p->status;
-        TL.ctrs = p->ctrs;
-        TL.n_dev = n_dev;
-        TL.err = p->err;
-        TL.out_bytes = L.out_bytes;
-        TL.dbg = p->o.reserved[1];
-        TL.dbg_ts = (uint64_t *)(((uint64_t)(uint32_t)p->o.reserved[3] << 32) | (uint32_t)p->o.reserved[2]);
-        const int grid2 = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (int64_t)p->sms * L.ctas));
-        cuda_check(join_chain_launch(L.P, TL, XJ, L.smem, grid2, p->stream), "k_scan_chain<join>");
-        p->launches++;
+        run_join_group(X, gi, g, o, outp, capacity, n_dev);
     }
     X.rels[gi] = o;
     X.done[gi] = 1;
@@ -1851,7 +1997,7 @@ std::string explain(rw_plan *p, int out_node)
             int gc = -3;
             for (size_t q = 0; q < G.groups.size(); q++) {
                 const Group &g = G.groups[q];
-                if (g.out == (int)i || g.join == (int)i || g.agg == (int)i ||
+                if (g.out == (int)i || g.join == (int)i || g.join_in == (int)i || g.agg == (int)i ||
                     std::find(g.chain.begin(), g.chain.end(), (int)i) != g.chain.end() ||
                     std::find(g.pre.begin(), g.pre.end(), (int)i) != g.pre.end())
                     gc = (int)q;
@@ -1859,7 +2005,8 @@ std::string explain(rw_plan *p, int out_node)
             bool fused = false;
             if (gc >= 0) {
                 const Group &g = G.groups[gc];
-                fused = pr == g.join || std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end() ||
+                fused = pr == g.join || (g.join_in >= 0 && pr == g.join_in) ||
+                        std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end() ||
                         std::find(g.pre.begin(), g.pre.end(), pr) != g.pre.end();
             }
             (void)gp;
@@ -1874,11 +2021,13 @@ std::string explain(rw_plan *p, int out_node)
         s << "  group " << q << ": "
           << (g.kind == G_SCAN ? "k_scan_chain"
                                : g.kind == G_SET ? "k_set_splits+k_set_op+k_set_scan+k_set_op<write>"
-                                                 : "k_merge_splits+k_join_runs+k_tile_runs+k_scan_chain<join>");
+                                                 : (g.join_in >= 0 ? "k_jsplit+k_jmatch x2 (chained)+k_jtiles+k_join_emit<3-input>"
+                                                                   : "k_jsplit+k_jmatch+k_jtiles+k_join_emit<2-input>"));
         if (g.agg >= 0) s << "<agg>+k_agg_finalize";
         s << " nodes [";
         if (g.kind == G_SCAN) s << "src " << g.source;
         else if (g.kind == G_SET) s << "setop " << g.join;
+        else if (g.join_in >= 0) s << "joins " << g.join_in << " -> " << g.join << " (3 inputs, mixed-radix expansion)";
         else s << "join " << g.join;
         for (int c : g.pre) s << ", key SELECT " << c << " (fused into the run matching)";
         for (int c : g.chain) s << ", " << kn[p->nodes[c].kind] << " " << c;
@@ -2172,11 +2321,13 @@ rw_status rw_plan_add_join(rw_plan *p, int32_t left, int32_t right, int32_t nkey
     const Node &R = node_at(p, right);
     if (nkey < 1 || nkey > (int)L.types.size() || nkey > (int)R.types.size())
         raise(RW_E_ARG, "bad nkey");
-    if (nkey != 1)
-        raise(RW_E_UNSUPPORTED, "this build joins on a single key column");
     for (int c = 0; c < nkey; c++)
         if (L.types[c] != R.types[c])
             raise(RW_E_TYPE, "join key types differ");
+    // keys are matched on one order-preserving image of at most 8 bytes: one column of
+    // any type, or two columns of at most 4 bytes each (lexicographic, A7)
+    if (nkey > 2 || (nkey == 2 && (type_width(L.types[0]) == 8 || type_width(L.types[1]) == 8)))
+        raise(RW_E_UNSUPPORTED, "join keys: one column, or two columns of at most 4 bytes each");
     if (L.nkey_sorted < nkey || R.nkey_sorted < nkey)
         raise(RW_E_UNSORTED, "join inputs must be sorted on the key (kernel dependence: sort first)");
     if (L.kind == N_AGG || R.kind == N_AGG)

@@ -241,7 +241,9 @@ def test_q1_declared_bound_violation_is_reported():
     from paper_conf_micro_wudcy12_b200 import rw
     spec = workloads.c4_spec()
     ins = workloads.c4_inputs(50_001, device=DEV, cfg=0x95)
-    ins["lineitem"][3][12345] = 1000          # disc far above its declared hi = 10
+    import rwgen
+    ins["lineitem"][0][12345] = rwgen.D_1998_09_02 - 10   # passes the SELECT
+    ins["lineitem"][3][12345] = 70_000        # disc far above its declared hi = 10 (and above 2^16)
     with pytest.raises(rw.RwError) as e:
         run_gpu(spec, ins, capacity=6)
     assert "declared" in str(e.value)
