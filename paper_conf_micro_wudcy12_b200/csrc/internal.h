@@ -26,8 +26,6 @@ constexpr int kMaxGroupCols = 8;
 constexpr int kMaxAggs = 16;
 constexpr int kThreads = 256;        // threads per CTA for every chain kernel
 constexpr int kScanItems = 8;        // rows per thread per tile in the scan kernel (T = 2048)
-constexpr int kJoinItems = 9;        // outputs per thread per tile in the join expansion (T = 2304,
-                                     // odd stride -> conflict-free thread-contiguous smem writes)
 constexpr int kMaxAggSlots = 4096;
 constexpr int kMaxBranch = 4;        // input-dependence fusion: SELECT/PROJECT chains sharing one scan
 constexpr int kRegD = 6;             // register aggregate terminal: groups x sums held per thread
@@ -131,29 +129,6 @@ struct TileLaunch {
                                // (in their input stages) waiting for their global offsets
     uint32_t warp_buf;         // emitting scan kernel: bytes of each compute warp's compaction buffer
     uint64_t *dbg_ts;          // 12 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots, scattered, reserve start; join: records cached, gathered)
-};
-
-// Join expansion inputs (run records written by k_join_runs).
-struct JoinRuns {
-    const uint32_t *s;         // first L row of the run
-    const uint32_t *lenL;
-    const uint32_t *lo;        // first matching R row
-    const uint32_t *lenR;
-    const uint64_t *off;       // exclusive output offset of the run
-    int64_t nruns;
-    int64_t total;             // total join candidates
-    // gather sources: output column j of the join = L col (j < nl) else R col (nkey + j - nl)
-    int32_t ncols;             // number of join output columns that are live (gathered)
-    const void *src[kMaxSlots];
-    uint8_t from_right[kMaxSlots];
-    int16_t dst_slot[kMaxSlots];
-};
-
-struct JoinKeys {
-    const void *lkey;
-    const void *rkey;
-    int32_t key_type;
-    int64_t nl, nr;
 };
 
 }  // namespace rw

@@ -5,12 +5,9 @@
 //                             compacted store or group-by aggregate (a9).
 //   k_agg_finalize            128-bit accumulators -> output relation (groups with
 //                             count > 0, ascending code).
-//   k_join_runs<K>            merge-path partitioned sorted-key JOIN, phase 1:
-//                             matched key runs + output offsets (a7).
-//   k_tile_runs               first run of every expansion tile.
-//   k_scan_chain<..., JOIN>   JOIN phase 2: output-balanced expansion (join_fill)
-//                             fused with the downstream SELECT / PROJECT chain (a8),
-//                             same warp-specialised pipeline as the scan chain.
+//   (the compacting scan chains run on scan_emit.cu, the JOIN path on join2.cu;
+//    this kernel carries the aggregate terminal and, opts.reserved[6] == 3, the
+//    earlier L2-ring scan for comparison)
 //
 // Every persistent kernel claims tiles with a global atomic counter (so the
 // decoupled look-back always has forward progress) and the last CTA to leave
@@ -136,110 +133,9 @@ __device__ __forceinline__ void group_copy_out(T *dst, const T *src, int64_t bas
         d[j] = ld_ring(src + j, gring);
 }
 
-// Join expansion into a tile (§8(a) a8): candidates [t*T, t*T + rows) of the
-// join output are mapped to (left row, right row) through the tile's run records
-// (cached in smem) and the live join columns are gathered into the tile's slots.
-// Thread `tid` expands candidates [tid*ITEMS, tid*ITEMS + ITEMS): one binary search,
-// then a forward walk; ITEMS odd makes the thread-contiguous smem writes conflict-free.
-template <int NT, int ITEMS>
-__device__ inline void join_fill(const ChainProg &P, const JoinExpand &X, int64_t t, int64_t ntiles, int rows,
-                                 char *st, char *rcache, const TileLaunch &L)
-{
-    constexpr int T = NT * ITEMS;
-    const int tid = threadIdx.x;
-    uint64_t *c_off = (uint64_t *)rcache;
-    uint32_t *c_s = (uint32_t *)(c_off + (T + 1));
-    uint32_t *c_lo = c_s + (T + 1);
-    uint32_t *c_lenR = c_lo + (T + 1);
-    const int64_t o0 = t * T;
-    const int64_t r0 = X.tile_run[t];
-    const int64_t r1 = (t + 1 < ntiles) ? X.tile_run[t + 1] : X.nruns - 1;
-    const int nr = (int)(r1 - r0 + 1);
-    for (int q = tid; q < nr; q += NT) {
-        cp_async8(c_off + q, X.off + r0 + q);
-        cp_async4(c_s + q, X.s + r0 + q);
-        cp_async4(c_lo + q, X.lo + r0 + q);
-        cp_async4(c_lenR + q, X.lenR + r0 + q);
-    }
-    cp_async_wait_all();
-    bar_sync(kComputeBar, NT);
-    if ((L.dbg & 4) && tid == 0)
-        L.dbg_ts[12 * t + 10] = globaltimer();
-    const int first = tid * ITEMS;
-    if (first < rows) {
-        uint32_t ii[ITEMS], jj[ITEMS];
-        const uint64_t o = (uint64_t)(o0 + first);
-        int lo = 0, hi = nr;
-        while (lo < hi) {
-            const int mid = (lo + hi) >> 1;
-            if (c_off[mid] <= o) lo = mid + 1;
-            else hi = mid;
-        }
-        int r = lo - 1;
-        // (i, j) of the first candidate by division, the rest by a carry walk: every
-        // run has >= 1 candidate, so a step that leaves run r lands on the first
-        // candidate (0, 0) of run r + 1
-        const uint64_t d = o - c_off[r];
-        uint32_t lr = c_lenR[r];
-        uint32_t qi, qj;
-        if (d == 0) {
-            qi = qj = 0;
-        } else if (d <= 0xffffffffull) {
-            qi = (uint32_t)d / lr;
-            qj = (uint32_t)d - qi * lr;
-        } else {
-            qi = (uint32_t)(d / lr);
-            qj = (uint32_t)(d - (uint64_t)qi * lr);
-        }
-#pragma unroll
-        for (int k = 0; k < ITEMS; k++) {
-            ii[k] = jj[k] = 0;
-            if (first + k < rows) {
-                const uint64_t oo = o + k;
-                if (r + 1 < nr && c_off[r + 1] <= oo) {
-                    r++;
-                    lr = c_lenR[r];
-                    qi = qj = 0;
-                }
-                ii[k] = c_s[r] + qi;
-                jj[k] = c_lo[r] + qj;
-                if (++qj == lr) {
-                    qj = 0;
-                    ++qi;
-                }
-            }
-        }
-        // every gather of every live column is issued as an async copy before any
-        // completes (one round trip per tile instead of one per column)
-        for (int c = 0; c < X.ncols; c++) {
-            char *dst = st + P.slot[X.dst_slot[c]].off;
-            const int w = type_width(P.slot[X.dst_slot[c]].type);
-            const char *src = (const char *)X.src[c];
-            const bool right = X.from_right[c];
-#pragma unroll
-            for (int k = 0; k < ITEMS; k++) {
-                if (first + k < rows) {
-                    const size_t row = right ? jj[k] : ii[k];
-                    if (w == 4)
-                        cp_async4((uint32_t *)dst + first + k, (const uint32_t *)src + row);
-                    else if (w == 8)
-                        cp_async8((uint64_t *)dst + first + k, (const uint64_t *)src + row);
-                    else
-                        ((uint8_t *)dst)[first + k] = ((const uint8_t *)src)[row];
-                }
-            }
-        }
-        cp_async_wait_all();
-    }
-    if ((L.dbg & 4) && tid == 0)
-        L.dbg_ts[12 * t + 11] = globaltimer();
-    bar_sync(kComputeBar, NT);
-}
-
-template <int NT, int ITEMS, bool AGG, bool JOIN, bool MULTI = false>
+template <int NT, int ITEMS, bool AGG, bool MULTI = false>
 __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_chain(const __grid_constant__ ChainProg P,
-                                                                     const __grid_constant__ TileLaunch L,
-                                                                     const __grid_constant__ JoinExpand X)
+                                                                     const __grid_constant__ TileLaunch L)
 {
     constexpr int T = NT * ITEMS;
     constexpr int NW = NT / 32;             // compute warps
@@ -262,14 +158,13 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
     // accumulators
     const size_t part_words = AGG ? (P.agg_mode == 0 ? (size_t)P.D * NA * NT : 0) : 0;
     unsigned long long *cta_acc = part + part_words;
-    char *rcache = sm_after;                // join: run-record cache for the current tile
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
     const int64_t ntiles = (n + T - 1) / T;
     const bool emit = !AGG && !(L.dbg & 2) && !L.direct;
     // input-dependence branches: only the MULTI instance carries the branch loop, so
     // the single-chain instances compile with NB == 1
-    const int NB = (AGG || JOIN || !MULTI) ? 1 : P.nbranch;
+    const int NB = (AGG || !MULTI) ? 1 : P.nbranch;
 
     if (tid == 0) {
         for (int s = 0; s < S; s++) {
@@ -310,7 +205,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 ctl->in[s].tile = t;
                 if ((L.dbg & 4) && t < ntiles)
                     L.dbg_ts[12 * t + 0] = globaltimer();
-                if (!JOIN && t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
+                if (t < ntiles && L.use_tma && (t + 1) * (int64_t)T <= n) {
                     char *st = stages + (size_t)s * P.stage_bytes;
                     fence_proxy_async_smem();
                     mbar_arrive_expect_tx(&ctl->in[s].full, tx_bytes);
@@ -446,9 +341,7 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                 release_stage();
                 continue;
             }
-            if (JOIN) {
-                join_fill<NT, ITEMS>(P, X, t, ntiles, rows, st, rcache, L);
-            } else if (!(L.use_tma && rows == T)) {
+            if (!(L.use_tma && rows == T)) {
                 // ragged last tile or unaligned column bases: each thread loads its own rows
                 for (int c = 0; c < P.nin; c++) {
                     const int w = type_width(P.slot[c].type);
@@ -748,496 +641,10 @@ __global__ void __launch_bounds__(kThreads) k_agg_finalize(const __grid_constant
 }
 
 // ===========================================================================
-// JOIN phase 1 — merge-path partitions of the merged key sequence (L before R on
-// ties, §4.3.2 binary-search partitioning).  For every L element that
-// starts a key run inside the partition: R range [lo, hi) by binary search in
-// the partition's smem copy of R (lo always lies inside it), galloping past the
-// partition end for long runs; L run length likewise.  Runs with a match are
-// compacted (ballot + look-back) into run records with their output offsets.
-// ===========================================================================
-constexpr int kRunItems = 8;
-constexpr int kRunT = kThreads * kRunItems;
-constexpr int kRunExt = 512;     // extra L / R elements staged past the partition end
-
-template <typename K>
-__device__ __forceinline__ int64_t merge_path(const K *L, int64_t nl, const K *R, int64_t nr, int64_t d)
-{
-    int64_t lo = d > nr ? d - nr : 0;
-    int64_t hi = d < nl ? d : nl;
-    while (lo < hi) {
-        int64_t mid = (lo + hi) >> 1;
-        if (L[mid] <= R[d - mid - 1])
-            lo = mid + 1;
-        else
-            hi = mid;
-    }
-    return lo;
-}
-
-template <typename K>
-__device__ __forceinline__ int lower_bound_smem(const K *a, int n, K key)
-{
-    int lo = 0, hi = n;
-    while (lo < hi) {
-        int mid = (lo + hi) >> 1;
-        if (a[mid] < key) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
-template <typename K>
-__device__ __forceinline__ int upper_bound_smem(const K *a, int n, K key)
-{
-    int lo = 0, hi = n;
-    while (lo < hi) {
-        int mid = (lo + hi) >> 1;
-        if (a[mid] <= key) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
-// first index >= start with A[idx] > key (A[start..] sorted, A[start-1] <= key)
-template <typename K>
-__device__ int64_t gallop_upper(const K *A, int64_t start, int64_t n, K key)
-{
-    int64_t lo = start, hi = n, step = 1;
-    while (true) {
-        int64_t probe = lo + step - 1;
-        if (probe >= n) { hi = n; break; }
-        if (A[probe] > key) { hi = probe; break; }
-        lo = probe + 1;
-        step <<= 1;
-    }
-    while (lo < hi) {
-        int64_t mid = (lo + hi) >> 1;
-        if (A[mid] <= key) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
-// exclusive block scan of per-(item, thread) 64-bit values in (k, warp, lane) order
-template <int ITEMS>
-__device__ inline void block_scan_u64(uint64_t (&v)[ITEMS], uint64_t *wtot /* ITEMS*kWarps */, uint64_t &total)
-{
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++) {
-        uint64_t x = v[k], inc = x;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o)
-                inc += y;
-        }
-        v[k] = inc - x;   // exclusive within the warp
-        if (lane == 31)
-            wtot[k * kWarps + warp] = inc;
-    }
-    __syncthreads();
-    if (warp == 0) {
-        constexpr int NV = ITEMS * kWarps;
-        constexpr int PER = (NV + 31) / 32;
-        uint64_t a[PER];
-        uint64_t s = 0;
-#pragma unroll
-        for (int q = 0; q < PER; q++) {
-            int idx = lane * PER + q;
-            a[q] = idx < NV ? wtot[idx] : 0;
-            s += a[q];
-        }
-        uint64_t inc = s;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o)
-                inc += y;
-        }
-        uint64_t run = inc - s;
-#pragma unroll
-        for (int q = 0; q < PER; q++) {
-            int idx = lane * PER + q;
-            if (idx < NV)
-                wtot[idx] = run;
-            run += a[q];
-        }
-        if (lane == 31)
-            wtot[NV] = inc;
-    }
-    __syncthreads();
-    total = wtot[ITEMS * kWarps];
-#pragma unroll
-    for (int k = 0; k < ITEMS; k++)
-        v[k] += wtot[k * kWarps + warp];
-}
-
-// merge-path split of every partition boundary d = p * kRunT (p = 0..nparts)
-template <typename K>
-__global__ void k_merge_splits(const __grid_constant__ JoinRunsLaunch J)
-{
-    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (p > J.nparts)
-        return;
-    const int64_t d = min(p * kRunT, J.nl + J.nr);
-    J.split[p] = merge_path((const K *)J.lkey, J.nl, (const K *)J.rkey, J.nr, d);
-}
-
-// first index in [start, n) of a sorted smem array with a[idx] > key (a[start-1] <= key)
-template <typename K>
-__device__ __forceinline__ int gallop_smem(const K *a, int start, int n, K key)
-{
-    int lo = start, hi = n, step = 1;
-    while (true) {
-        const int probe = lo + step - 1;
-        if (probe >= n) { hi = n; break; }
-        if (a[probe] > key) { hi = probe; break; }
-        lo = probe + 1;
-        step <<= 1;
-    }
-    while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (a[mid] <= key) lo = mid + 1;
-        else hi = mid;
-    }
-    return lo;
-}
-
-// fused upstream SELECT on the join key (N2): every atom must hold for the run's key
-template <typename K>
-__device__ __forceinline__ bool key_pass(const JoinRunsLaunch &J, K key)
-{
-    bool ok = true;
-    for (int i = 0; i < J.nkpred; i++) {
-        const K c = (K)J.kpk[i];
-        switch (J.kop[i]) {
-        case C_LT: ok = ok && key < c; break;
-        case C_LE: ok = ok && key <= c; break;
-        case C_GT: ok = ok && key > c; break;
-        case C_GE: ok = ok && key >= c; break;
-        case C_EQ: ok = ok && key == c; break;
-        default: ok = ok && key != c; break;
-        }
-    }
-    return ok;
-}
-
-// Two streaming passes (no look-back on the critical path): WRITE = false counts
-// the matched runs and join candidates of every partition; k_scan_parts turns the
-// counts into exclusive offsets; WRITE = true recomputes the partition (identical
-// arithmetic) and writes the run records at their offsets.
-//
-// In the merged order (L before R on equal keys, P:196 binary-search partitioning)
-// every key forms one contiguous segment [its L rows][its R rows].  A segment HEAD is
-// a merged element whose key differs from its predecessor's; at a head the walk's
-// (L index, R index) are the key's first L row and its R lower bound, and the next
-// head's indices end both runs.  So a partition needs no per-run searches:
-//   1. each thread merges its 8 positions (one diagonal search) and records heads;
-//   2. a block scan places the heads in smem in merged order;
-//   3. head k's run lengths are head k+1's indices minus its own; only the
-//      partition's last head looks past the partition end (galloping in smem, then
-//      in HBM for hot keys whose segment spans later partitions);
-//   4. matched heads (lenL > 0 and lenR > 0) are compacted into run records.
-template <typename K, bool WRITE>
-__global__ void __launch_bounds__(kThreads, 3) k_join_runs(const __grid_constant__ JoinRunsLaunch J)
-{
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    uint64_t *wtot = (uint64_t *)smem_raw;                        // 2 * kWarps, then head counts
-    int32_t *hcount = (int32_t *)(wtot + 2 * kWarps);             // kWarps
-    K *sL = (K *)(smem_raw + align_up((kRunItems * kWarps + 1) * 8, 128));   // kRunT + kRunExt
-    K *sR = sL + kRunT + kRunExt;                                 // kRunT + kRunExt
-    int32_t *hL = (int32_t *)(sR + kRunT + kRunExt);              // kRunT heads (local L index)
-    int32_t *hR = hL + kRunT;                                     // kRunT heads (local R index)
-    K *hK = (K *)align_up((size_t)(hR + kRunT), 16);              // kRunT head keys
-    const K *L = (const K *)J.lkey;
-    const K *R = (const K *)J.rkey;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int64_t ntot = J.nl + J.nr;
-
-    // software pipeline: the keys of the CTA's next partition are loaded into
-    // registers while the current one is processed
-    constexpr int PF = (kRunT + kRunExt + kThreads - 1) / kThreads;
-    K pfL[PF], pfR[PF];
-    auto fetch = [&](int64_t pp) {
-        const int64_t a0 = J.split[pp], a1 = J.split[pp + 1];
-        const int64_t e0 = min(pp * kRunT, ntot);
-        const int64_t b0 = e0 - a0, b1 = min(e0 + kRunT, ntot) - a1;
-        const int nle = (int)(min(a1 + kRunExt, J.nl) - a0), nre = (int)(min(b1 + kRunExt, J.nr) - b0);
-#pragma unroll
-        for (int q = 0; q < PF; q++) {
-            const int idx = tid + q * kThreads;
-            pfL[q] = idx < nle ? L[a0 + idx] : K(0);
-            pfR[q] = idx < nre ? R[b0 + idx] : K(0);
-        }
-    };
-    if ((int64_t)blockIdx.x < J.nparts)
-        fetch(blockIdx.x);
-    for (int64_t p = blockIdx.x; p < J.nparts; p += gridDim.x) {
-        const int64_t d0 = p * kRunT, d1 = min(d0 + kRunT, ntot);
-        const int64_t i0 = J.split[p], i1 = J.split[p + 1], j0 = d0 - i0, j1 = d1 - i1;
-        const int nL = (int)(i1 - i0), nR = (int)(j1 - j0), m = (int)(d1 - d0);
-        const int nLe = (int)(min(i1 + kRunExt, J.nl) - i0), nRe = (int)(min(j1 + kRunExt, J.nr) - j0);
-        __syncthreads();
-#pragma unroll
-        for (int q = 0; q < PF; q++) {
-            const int idx = tid + q * kThreads;
-            if (idx < nLe) sL[idx] = pfL[q];
-            if (idx < nRe) sR[idx] = pfR[q];
-        }
-        __syncthreads();
-        if (p + gridDim.x < J.nparts)
-            fetch(p + gridDim.x);
-
-        // 1. merge walk over the thread's positions: bit q of hmask = position dt+q is a
-        //    segment head, bit q of tmask = it is an L element (so its L index is lo0 +
-        //    popc(tmask below q) and its R index the merged position minus that)
-        uint32_t hmask = 0, tmask = 0;
-        int lo0 = 0;
-        const int dt = tid * kRunItems;
-        if (dt < m) {
-            int lo = dt > nR ? dt - nR : 0, hi = dt < nL ? dt : nL;
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (sL[mid] <= sR[dt - mid - 1]) lo = mid + 1;
-                else hi = mid;
-            }
-            lo0 = lo;
-            int li = lo, rj = dt - lo;
-            // predecessor of the first position in merged order: the larger of the
-            // preceding L and R elements (global ones at the partition start)
-            const bool pl_ok = (i0 + li) > 0, pr_ok = (j0 + rj) > 0;
-            bool has_prev = pl_ok || pr_ok;
-            K prev = K(0);
-            if (has_prev) {
-                const K pl = pl_ok ? (li > 0 ? sL[li - 1] : L[i0 - 1]) : K(0);
-                const K pr = pr_ok ? (rj > 0 ? sR[rj - 1] : R[j0 - 1]) : K(0);
-                prev = !pl_ok ? pr : (!pr_ok ? pl : (pl < pr ? pr : pl));
-            }
-#pragma unroll
-            for (int q = 0; q < kRunItems; q++) {
-                if (dt + q < m) {
-                    const bool takeL = rj >= nR || (li < nL && sL[li] <= sR[rj]);
-                    const K key = takeL ? sL[li] : sR[rj];
-                    hmask |= (uint32_t)(!has_prev || key != prev) << q;
-                    tmask |= (uint32_t)takeL << q;
-                    has_prev = true;
-                    prev = key;
-                    li += takeL ? 1 : 0;
-                    rj += takeL ? 0 : 1;
-                }
-            }
-        }
-        const int nh = __popc(hmask);
-        // 2. heads in merged order into smem
-        int hinc = nh;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(0xffffffffu, hinc, o);
-            if (lane >= o) hinc += y;
-        }
-        if (lane == 31)
-            hcount[warp] = hinc;
-        __syncthreads();
-        int hbase = 0, H = 0;
-        for (int w = 0; w < kWarps; w++) {
-            if (w < warp) hbase += hcount[w];
-            H += hcount[w];
-        }
-        hbase += hinc - nh;
-        for (uint32_t hm = hmask; hm; hm &= hm - 1) {
-            const int q = __ffs(hm) - 1;
-            const int li = lo0 + __popc(tmask & ((1u << q) - 1u));
-            const int rj = dt + q - li;
-            hL[hbase] = li;
-            hR[hbase] = rj;
-            hK[hbase] = ((tmask >> q) & 1u) ? sL[li] : sR[rj];
-            hbase++;
-        }
-        __syncthreads();
-        // 3. run lengths; the last head's segment may continue past the partition
-        const int k0 = tid * kRunItems;
-        int64_t tailL = 0, tailR = 0;
-        if (k0 < H && k0 + kRunItems >= H) {
-            const K key = hK[H - 1];
-            int e = nL;
-            if (nL < nLe && sL[nL] == key)
-                e = gallop_smem(sL, nL + 1, nLe, key);
-            tailL = i0 + e;
-            if (e == nLe && i0 + e < J.nl && L[i0 + e] == key)
-                tailL = gallop_upper(L, i0 + e, J.nl, key);
-            int f = nR;
-            if (nR < nRe && sR[nR] == key)
-                f = gallop_smem(sR, nR + 1, nRe, key);
-            tailR = j0 + f;
-            if (f == nRe && j0 + f < J.nr && R[j0 + f] == key)
-                tailR = gallop_upper(R, j0 + f, J.nr, key);
-        }
-        int nrun = 0;
-        uint64_t outs = 0;
-        uint32_t matched = 0;
-        uint64_t cnt[kRunItems];
-        int64_t lenl[kRunItems], lenr[kRunItems];
-#pragma unroll
-        for (int q = 0; q < kRunItems; q++) {
-            const int k = k0 + q;
-            cnt[q] = 0;
-            lenl[q] = lenr[q] = 0;
-            if (k < H) {
-                const int64_t nl_ = k + 1 < H ? i0 + hL[k + 1] : tailL;
-                const int64_t nr_ = k + 1 < H ? j0 + hR[k + 1] : tailR;
-                lenl[q] = nl_ - (i0 + hL[k]);
-                lenr[q] = nr_ - (j0 + hR[k]);
-                if (lenl[q] > 0 && lenr[q] > 0 && key_pass<K>(J, hK[k])) {
-                    matched |= 1u << q;
-                    cnt[q] = (uint64_t)lenl[q] * (uint64_t)lenr[q];
-                    nrun++;
-                    outs += cnt[q];
-                }
-            }
-        }
-        // 4. block exclusive scan of (runs, outputs) over threads (thread order = merge order)
-        uint64_t ir = (uint64_t)nrun, io = outs;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint64_t yr = __shfl_up_sync(0xffffffffu, ir, o), yo = __shfl_up_sync(0xffffffffu, io, o);
-            if (lane >= o) {
-                ir += yr;
-                io += yo;
-            }
-        }
-        if (lane == 31) {
-            wtot[warp] = ir;
-            wtot[kWarps + warp] = io;
-        }
-        __syncthreads();
-        uint64_t br = 0, bo = 0, tr = 0, to = 0;
-        for (int w = 0; w < kWarps; w++) {
-            if (w < warp) {
-                br += wtot[w];
-                bo += wtot[kWarps + w];
-            }
-            tr += wtot[w];
-            to += wtot[kWarps + w];
-        }
-        br += ir - (uint64_t)nrun;
-        bo += io - outs;
-        if (!WRITE) {
-            if (tid == 0) {
-                J.pruns[p] = tr;
-                J.pouts[p] = to;
-            }
-            continue;
-        }
-        int64_t r = (int64_t)J.pruns[p] + (int64_t)br;
-        uint64_t off = J.pouts[p] + bo;
-#pragma unroll
-        for (int q = 0; q < kRunItems; q++) {
-            if ((matched >> q) & 1u) {
-                const int k = k0 + q;
-                if (r < J.cap_runs) {
-                    J.s[r] = (uint32_t)(i0 + hL[k]);
-                    J.lenL[r] = (uint32_t)lenl[q];
-                    J.lo[r] = (uint32_t)(j0 + hR[k]);
-                    J.lenR[r] = (uint32_t)lenr[q];
-                    J.off[r] = off;
-                }
-                r++;
-                off += cnt[q];
-            }
-        }
-    }
-}
-
-// exclusive scan of the per-partition counts (one CTA; nparts is ~ rows / 2048)
-__global__ void __launch_bounds__(1024) k_scan_parts(const __grid_constant__ JoinRunsLaunch J)
-{
-    __shared__ uint64_t wr[32], wo[32];
-    __shared__ uint64_t carry_r, carry_o;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0)
-        carry_r = carry_o = 0;
-    __syncthreads();
-    for (int64_t b0 = 0; b0 < J.nparts; b0 += 1024) {
-        const int64_t p = b0 + tid;
-        const uint64_t r = p < J.nparts ? J.pruns[p] : 0, o = p < J.nparts ? J.pouts[p] : 0;
-        uint64_t ir = r, io = o;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint64_t yr = __shfl_up_sync(0xffffffffu, ir, d), yo = __shfl_up_sync(0xffffffffu, io, d);
-            if (lane >= d) {
-                ir += yr;
-                io += yo;
-            }
-        }
-        if (lane == 31) {
-            wr[warp] = ir;
-            wo[warp] = io;
-        }
-        __syncthreads();
-        if (warp == 0) {
-            uint64_t xr = wr[lane], xo = wo[lane];
-#pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint64_t yr = __shfl_up_sync(0xffffffffu, xr, d), yo = __shfl_up_sync(0xffffffffu, xo, d);
-                if (lane >= d) {
-                    xr += yr;
-                    xo += yo;
-                }
-            }
-            wr[lane] = xr;
-            wo[lane] = xo;
-        }
-        __syncthreads();
-        const uint64_t er = carry_r + (warp ? wr[warp - 1] : 0) + ir - r;
-        const uint64_t eo = carry_o + (warp ? wo[warp - 1] : 0) + io - o;
-        if (p < J.nparts) {
-            J.pruns[p] = er;
-            J.pouts[p] = eo;
-        }
-        __syncthreads();
-        if (tid == 0) {
-            carry_r += wr[31];
-            carry_o += wo[31];
-        }
-        __syncthreads();
-    }
-    if (tid == 0) {
-        J.totals[0] = (int64_t)carry_r;
-        J.totals[1] = (int64_t)carry_o;
-    }
-}
-
-// first run of every expansion tile: tile_run[t] = upper_bound(off, t*T) - 1
-__global__ void k_tile_runs(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run)
-{
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= ntiles)
-        return;
-    const uint64_t o = (uint64_t)(t * T);
-    int64_t lo = 0, hi = nruns;
-    while (lo < hi) {
-        int64_t mid = (lo + hi) >> 1;
-        if (off[mid] <= o) lo = mid + 1;
-        else hi = mid;
-    }
-    tile_run[t] = lo - 1;
-}
-
-// ===========================================================================
 // Host launchers
 // ===========================================================================
 size_t scan_ctl_bytes() { return align_up(sizeof(ScanCtl<512, 8>), 128); }   // >= every (NT, ITEMS) variant
-size_t join_run_cache_bytes() { return align_up((size_t)(kThreads * kJoinItems + 1) * 20, 128); }
 int scan_tile() { return kThreads * kScanItems; }
-int join_expand_tile() { return kThreads * kJoinItems; }
-
-size_t join_runs_smem(int key_type)
-{
-    const size_t w = type_width(key_type);
-    return align_up((kRunItems * kWarps + 1) * 8, 128) + 2 * (size_t)(kRunT + kRunExt) * w + 2 * (size_t)kRunT * 4 +
-           16 + (size_t)kRunT * w;
-}
 
 template <typename F>
 static int occ(F f, size_t smem, int threads = kThreads)
@@ -1253,46 +660,35 @@ int chain_occupancy(int which, int nt, int items, size_t smem)
 {
     switch (which) {
     case 0:
-        if (nt == 512) return items == 8 ? occ(k_scan_chain<512, 8, false, false>, smem, 512 + kAuxThreads)
-                                         : occ(k_scan_chain<512, 4, false, false>, smem, 512 + kAuxThreads);
+        if (nt == 512) return items == 8 ? occ(k_scan_chain<512, 8, false>, smem, 512 + kAuxThreads)
+                                         : occ(k_scan_chain<512, 4, false>, smem, 512 + kAuxThreads);
         switch (items) {
-        case 4: return occ(k_scan_chain<256, 4, false, false>, smem, 256 + kAuxThreads);
-        case 5: return occ(k_scan_chain<256, 5, false, false>, smem, 256 + kAuxThreads);
-        case 6: return occ(k_scan_chain<256, 6, false, false>, smem, 256 + kAuxThreads);
-        default: return occ(k_scan_chain<256, 8, false, false>, smem, 256 + kAuxThreads);
+        case 4: return occ(k_scan_chain<256, 4, false>, smem, 256 + kAuxThreads);
+        case 5: return occ(k_scan_chain<256, 5, false>, smem, 256 + kAuxThreads);
+        case 6: return occ(k_scan_chain<256, 6, false>, smem, 256 + kAuxThreads);
+        default: return occ(k_scan_chain<256, 8, false>, smem, 256 + kAuxThreads);
         }
     case 4:   // input-dependence branches
-        return items == 4 ? occ(k_scan_chain<256, 4, false, false, true>, smem, 256 + kAuxThreads)
-                          : occ(k_scan_chain<256, 8, false, false, true>, smem, 256 + kAuxThreads);
+        return items == 4 ? occ(k_scan_chain<256, 4, false, true>, smem, 256 + kAuxThreads)
+                          : occ(k_scan_chain<256, 8, false, true>, smem, 256 + kAuxThreads);
     case 1:
-        if (nt == 128) return occ(k_scan_chain<128, 16, true, false>, smem, 128 + 32);
-        if (nt == 384) return occ(k_scan_chain<384, 5, true, false>, smem, 384 + 32);
-        if (nt == 448) return occ(k_scan_chain<448, 4, true, false>, smem, 448 + 32);
-        if (nt == 480) return occ(k_scan_chain<480, 4, true, false>, smem, 480 + 32);
-        if (nt == kNarrowNT) return occ(k_scan_chain<kNarrowNT, kNarrowItems, true, false>, smem, kNarrowNT + 32);
-        return items == 4 ? occ(k_scan_chain<256, 4, true, false>, smem, 256 + 32)
-                          : occ(k_scan_chain<256, 8, true, false>, smem, 256 + 32);
-    case 2: return occ(k_scan_chain<kThreads, kJoinItems, false, true>, smem, kThreads + kAuxThreads);
-    default: return occ(k_join_runs<uint64_t, true>, smem);
+        if (nt == 128) return occ(k_scan_chain<128, 16, true>, smem, 128 + 32);
+        if (nt == 384) return occ(k_scan_chain<384, 5, true>, smem, 384 + 32);
+        if (nt == 448) return occ(k_scan_chain<448, 4, true>, smem, 448 + 32);
+        if (nt == 480) return occ(k_scan_chain<480, 4, true>, smem, 480 + 32);
+        if (nt == kNarrowNT) return occ(k_scan_chain<kNarrowNT, kNarrowItems, true>, smem, kNarrowNT + 32);
+        return items == 4 ? occ(k_scan_chain<256, 4, true>, smem, 256 + 32)
+                          : occ(k_scan_chain<256, 8, true>, smem, 256 + 32);
+    default: return 0;
     }
 }
 
 template <int NT, int ITEMS, bool AGG, bool MULTI = false>
 static cudaError_t sc(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
-    JoinExpand X{};
-    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, false, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_scan_chain<NT, ITEMS, AGG, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)smem);
-    k_scan_chain<NT, ITEMS, AGG, false, MULTI><<<grid, NT + aux_threads(AGG), smem, s>>>(P, L, X);
-    return cudaGetLastError();
-}
-
-cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem, int grid,
-                              cudaStream_t s)
-{
-    cudaFuncSetAttribute(k_scan_chain<kThreads, kJoinItems, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)smem);
-    k_scan_chain<kThreads, kJoinItems, false, true><<<grid, kThreads + kAuxThreads, smem, s>>>(P, L, X);
+    k_scan_chain<NT, ITEMS, AGG, MULTI><<<grid, NT + aux_threads(AGG), smem, s>>>(P, L);
     return cudaGetLastError();
 }
 
@@ -1327,41 +723,6 @@ cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg,
 cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s)
 {
     k_agg_finalize<<<1, kThreads, 0, s>>>(F);
-    return cudaGetLastError();
-}
-
-template <typename K>
-static cudaError_t jr(const JoinRunsLaunch &J, size_t smem, int grid, cudaStream_t s)
-{
-    k_merge_splits<K><<<(unsigned)((J.nparts + 1 + 255) / 256), 256, 0, s>>>(J);
-    cudaFuncSetAttribute(k_join_runs<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(k_join_runs<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (J.nparts > 0) {
-        k_join_runs<K, false><<<grid, kThreads, smem, s>>>(J);
-        k_scan_parts<<<1, 1024, 0, s>>>(J);
-        k_join_runs<K, true><<<grid, kThreads, smem, s>>>(J);
-    } else {
-        k_scan_parts<<<1, 1024, 0, s>>>(J);
-    }
-    return cudaGetLastError();
-}
-
-cudaError_t join_runs_launch(const JoinRunsLaunch &J, int key_type, size_t smem, int grid, cudaStream_t s)
-{
-    switch (key_type) {
-    case T_I32: return jr<int32_t>(J, smem, grid, s);
-    case T_U32: return jr<uint32_t>(J, smem, grid, s);
-    case T_I64: return jr<int64_t>(J, smem, grid, s);
-    case T_U64: return jr<uint64_t>(J, smem, grid, s);
-    default: return jr<uint8_t>(J, smem, grid, s);
-    }
-}
-
-cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run,
-                             cudaStream_t s)
-{
-    if (ntiles > 0)
-        k_tile_runs<<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(off, nruns, ntiles, T, tile_run);
     return cudaGetLastError();
 }
 

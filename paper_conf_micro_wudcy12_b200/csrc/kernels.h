@@ -24,38 +24,6 @@ struct AggFinal {
     int32_t *err;                    // err[0] -> err[1], err[2] -> err[3], then err[0] = err[2] = 0
 };
 
-struct JoinRunsLaunch {
-    const void *lkey, *rkey;
-    int64_t nl, nr;
-    int64_t nparts;
-    uint32_t *s, *lenL, *lo, *lenR;
-    uint64_t *off;
-    int64_t cap_runs;
-    uint64_t *status_runs, *status_outs;
-    uint32_t epoch_runs, epoch_outs;
-    uint32_t *ctrs;
-    int64_t *totals;                 // [0] runs, [1] join candidates
-    int64_t *split;                  // nparts + 1 merge-path splits (k_merge_splits)
-    uint64_t *pruns, *pouts;         // per-partition counts, then exclusive offsets
-    // SELECTs on the join key fused into the run matching (SURVEY §8(f) N2
-    // Fig. 13): a run is matched only if its key passes every atom (key op kpk[i]),
-    // compared in the key type; a key predicate keeps or drops whole runs
-    int32_t nkpred;
-    uint8_t kop[kMaxKeyPreds];
-    int64_t kpk[kMaxKeyPreds];
-};
-
-struct JoinExpand {
-    const uint32_t *s, *lo, *lenR;
-    const uint64_t *off;
-    const int64_t *tile_run;
-    int64_t nruns;
-    int32_t ncols;                   // gathered (live) join output columns
-    const void *src[kMaxSlots];
-    uint8_t from_right[kMaxSlots];
-    int16_t dst_slot[kMaxSlots];
-};
-
 // set operators (setops.cu): inputs sorted on every column, identical schemas
 constexpr int kMaxSetCols = 4;
 struct SetLaunch {
@@ -78,18 +46,12 @@ int set_partition_rows();
 cudaError_t set_op_launch(const SetLaunch &S, int sms, cudaStream_t st);   // 2 launches (look-back) or 4
 
 size_t scan_ctl_bytes();
-size_t join_run_cache_bytes();
-int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 2 join expand, 3 join runs, 4 scan branches
+int chain_occupancy(int which, int nt, int items, size_t smem);   // which: 0 scan, 1 scan+agg, 4 scan branches
 cudaError_t scan_chain_launch(const ChainProg &P, const TileLaunch &L, bool agg, int nt, int items, size_t smem, int grid,
                               cudaStream_t s);
 cudaError_t agg_finalize_launch(const AggFinal &F, cudaStream_t s);
-cudaError_t join_runs_launch(const JoinRunsLaunch &J, int key_type, size_t smem, int grid, cudaStream_t s);
-size_t join_runs_smem(int key_type);
-cudaError_t tile_runs_launch(const uint64_t *off, int64_t nruns, int64_t ntiles, int64_t T, int64_t *tile_run,
-                             cudaStream_t s);
-int join_expand_tile();
-cudaError_t join_chain_launch(const ChainProg &P, const TileLaunch &L, const JoinExpand &X, size_t smem, int grid,
-                              cudaStream_t s);
+
+
 int scan_tile();
 
 // ---- join2.cu: run matching (single pass) and the fused expansion ----
