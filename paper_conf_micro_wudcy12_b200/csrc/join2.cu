@@ -1032,8 +1032,10 @@ static int jocc(size_t smem)
     return n;
 }
 
-int join_emit_occupancy(int items, int ways, size_t smem)
+int join_emit_occupancy(int nt, int items, int ways, size_t smem)
 {
+    if (nt == 512)
+        return ways == 3 ? jocc<512, 4, 3>(smem) : jocc<512, 4, 2>(smem);
     if (ways == 3)
         return items == 4 ? jocc<256, 4, 3>(smem) : jocc<256, 8, 3>(smem);
     return items == 4 ? jocc<256, 4, 2>(smem) : jocc<256, 8, 2>(smem);
@@ -1047,9 +1049,11 @@ static cudaError_t jgo(const ChainProg &P, const TileLaunch &L, const JoinEmit &
     return cudaGetLastError();
 }
 
-cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int items, int ways, size_t smem,
-                             int grid, cudaStream_t s)
+cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int nt, int items, int ways,
+                             size_t smem, int grid, cudaStream_t s)
 {
+    if (nt == 512)
+        return ways == 3 ? jgo<512, 4, 3>(P, L, X, smem, grid, s) : jgo<512, 4, 2>(P, L, X, smem, grid, s);
     if (ways == 3)
         return items == 4 ? jgo<256, 4, 3>(P, L, X, smem, grid, s) : jgo<256, 8, 3>(P, L, X, smem, grid, s);
     return items == 4 ? jgo<256, 4, 2>(P, L, X, smem, grid, s) : jgo<256, 8, 2>(P, L, X, smem, grid, s);

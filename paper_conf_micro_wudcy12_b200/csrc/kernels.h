@@ -105,9 +105,9 @@ cudaError_t jtiles_launch(const uint64_t *off, const int64_t *totals, int64_t T,
 uint32_t join_rec_cap4(int T);
 size_t join_rec_stage_bytes(int ways, int T);
 size_t join_emit_ctl_bytes();
-int join_emit_occupancy(int items, int ways, size_t smem);
-cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int items, int ways, size_t smem,
-                             int grid, cudaStream_t s);
+int join_emit_occupancy(int nt, int items, int ways, size_t smem);
+cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int nt, int items, int ways,
+                             size_t smem, int grid, cudaStream_t s);
 
 // emitting scan kernel (scan_emit.cu): compacting SELECT / PROJECT chains, 1..4 branches
 size_t emit_ctl_bytes();

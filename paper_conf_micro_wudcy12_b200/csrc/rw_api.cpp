@@ -936,9 +936,12 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         const int ways = g.join_in >= 0 ? 3 : 2;
         bool found = false;
         double best = -1;
-        for (int items : {8, 4}) {
+        struct JV { int nt, items; };
+        for (JV jv : {JV{256, 8}, JV{512, 4}, JV{256, 4}}) {
+            const int items = jv.items, ntj = jv.nt;
             if (p->o.reserved[5] > 0 && items != p->o.reserved[5]) continue;
-            const int T = kThreads * items;
+            if (p->o.reserved[4] == 7 ? ntj != 512 : (p->o.reserved[4] == 8 && ntj != 256)) continue;
+            const int T = ntj * items;
             layout(T);
             size_t W = 0;
             for (int c = 0; c < P.nout; c++)
@@ -946,28 +949,31 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             const size_t RS = join_rec_stage_bytes(ways, T);
             const size_t base = join_emit_ctl_bytes() + 2 * (size_t)P.stage_bytes + (size_t)ways * T * 4 +
                                 (size_t)T * 2 + P.scratch_bytes;
-            for (int S = 2; S <= 3; S++) {
+            for (int occ_t : {1, 2}) {
+              if (p->o.ctas_per_sm > 0 ? occ_t != p->o.ctas_per_sm : occ_t != 1) continue;
+              for (int S = 2; S <= 3; S++) {
                 if (p->o.stages > 0 && S != p->o.stages) continue;
-                const size_t per_cta = kSmemLimit;
+                const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
                 if (base + S * RS + W > per_cta) continue;
                 size_t Rb = (per_cta - base - S * RS) / 128 * 128;
                 if (p->o.reserved[0] > 0) Rb = std::min(Rb, (size_t)p->o.reserved[0] * 1024);
                 if (Rb < W) continue;
                 const size_t smem = base + S * RS + Rb;
-                if (join_emit_occupancy(items, ways, smem) < 1) continue;
+                if (join_emit_occupancy(ntj, items, ways, smem) < occ_t) continue;
                 const double q = (double)Rb / (double)W;
-                const double sc = (q >= 2.0 ? 1e9 : q * 1e8) + T * 1e3 + S;
+                const double sc = (q >= 2.0 ? 1e9 : q * 1e8) + T * 1e3 + ntj + S;
                 if (sc > best) {
                     best = sc;
                     L.items = items;
-                    L.nt = kThreads;
+                    L.nt = ntj;
                     L.tile = T;
                     L.stages = S;
                     L.out_bytes = (uint32_t)Rb;
                     L.smem = smem;
-                    L.ctas = 1;
+                    L.ctas = occ_t;
                     found = true;
                 }
+              }
             }
         }
         if (!found)
@@ -1492,7 +1498,7 @@ void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void
     TL.out_bytes = L.out_bytes;
     TL.dbg = p->o.reserved[1];
     const int grid = p->sms * L.ctas;
-    cuda_check(join_emit_launch(L.P, TL, XJ, L.items, three ? 3 : 2, L.smem, grid, p->stream), "k_join_emit");
+    cuda_check(join_emit_launch(L.P, TL, XJ, L.nt, L.items, three ? 3 : 2, L.smem, grid, p->stream), "k_join_emit");
     p->launches++;
 }
 
