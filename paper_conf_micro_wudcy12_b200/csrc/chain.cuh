@@ -408,9 +408,17 @@ __device__ inline void agg_tile_rowwise(const ChainProg &P, const char *stage, c
     }
 }
 
+// Row of mask bit k: the scan kernels' k*NT + tid, or (R4) the 4-row vector layout of
+// chain4.cuh, ((k/4)*NT + tid)*4 + k%4 (the join expansion's aggregate terminal).
+template <int NT, bool R4>
+__device__ __forceinline__ int arow(int k)
+{
+    return R4 ? (((k >> 2) * NT + (int)threadIdx.x) << 2) + (k & 3) : k * NT + (int)threadIdx.x;
+}
+
 // Global-atomic terminal (agg_mode 3) for group-bys too large for per-thread
 // partials in shared memory: every row adds into the global 128-bit accumulators.
-template <int NT, int ITEMS>
+template <int NT, int ITEMS, bool R4 = false>
 __device__ inline void agg_tile_global(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
                                        unsigned long long *acc, int32_t *err)
 {
@@ -420,7 +428,7 @@ __device__ inline void agg_tile_global(const ChainProg &P, const char *stage, co
     for (int k = 0; k < ITEMS; k++) {
         if (!((mask >> k) & 1u))
             continue;
-        const int r = k * NT + tid;
+        const int r = arow<NT, R4>(k);
         int g = 0;
         bool ok = true;
         for (int c = 0; c < P.ngc; c++) {
@@ -643,7 +651,7 @@ __device__ inline void reg_agg_reduce_warp(const ChainProg &P, RegAgg &R, unsign
 // Narrow sums (a < NN) accumulate in 32-bit partials whose flush period comes from the
 // caller-declared bounds; their values are OR-ed into `orv` so that a value outside
 // [0, 2^narrow_bits) is reported (err[2]) instead of silently wrapping a partial.
-template <int NT, int ITEMS, int NAGG, bool W64, int NN = 0>
+template <int NT, int ITEMS, int NAGG, bool W64, int NN = 0, bool R4 = false>
 __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *at, const uint32_t *g, uint32_t ok,
                                              RegAgg &R, uint64_t &orv)
 {
@@ -651,7 +659,7 @@ __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *a
 #pragma unroll
     for (int k = 0; k < ITEMS; k++) {
         const uint32_t gk = ((ok >> k) & 1u) ? g[k] : 0xffffffffu;   // failing rows match no group
-        const int r = k * NT + tid;
+        const int r = arow<NT, R4>(k);
         uint64_t v[kRegA];
 #pragma unroll
         for (int a = 0; a < kRegA; a++)
@@ -676,7 +684,7 @@ __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *a
     }
 }
 
-template <int NT, int ITEMS>
+template <int NT, int ITEMS, bool R4 = false>
 __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const char *scratch, uint32_t mask,
                                     RegAgg &R, unsigned long long *cta_acc, int64_t &since_flush, int32_t *err)
 {
@@ -693,7 +701,7 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
         case T_U8:
 #pragma unroll
             for (int k = 0; k < ITEMS; k++) {
-                const uint32_t v = ((const uint8_t *)b)[k * NT + tid];
+                const uint32_t v = ((const uint8_t *)b)[arow<NT, R4>(k)];
                 if (v >= dom) ok &= ~(1u << k);
                 g[k] = g[k] * dom + v;
             }
@@ -702,7 +710,7 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
         case T_U32:
 #pragma unroll
             for (int k = 0; k < ITEMS; k++) {
-                const uint32_t v = ((const uint32_t *)b)[k * NT + tid];   // negative i32 -> huge
+                const uint32_t v = ((const uint32_t *)b)[arow<NT, R4>(k)];   // negative i32 -> huge
                 if (v >= dom) ok &= ~(1u << k);
                 g[k] = g[k] * dom + v;
             }
@@ -710,7 +718,7 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
         default:
 #pragma unroll
             for (int k = 0; k < ITEMS; k++) {
-                const uint64_t v = ((const uint64_t *)b)[k * NT + tid];
+                const uint64_t v = ((const uint64_t *)b)[arow<NT, R4>(k)];
                 if (v >= dom) ok &= ~(1u << k);
                 g[k] = g[k] * dom + (uint32_t)v;
             }
@@ -741,27 +749,27 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
         // the 576-thread instance is specialised (host-selected) for 5 all-64-bit sums of
         // which the first 2 are narrow: only this row loop is compiled into it, which is
         // what lets 18 compute warps fit the register file
-        agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R, orv);
+        agg_rows_reg<NT, ITEMS, 5, true, 2, R4>(ab, at, g, ok, R, orv);
     } else if (w64 && P.agg_narrow) {
         switch (P.nagg * 4 + P.agg_narrow) {
-        case 3 * 4 + 1: agg_rows_reg<NT, ITEMS, 3, true, 1>(ab, at, g, ok, R, orv); break;
-        case 3 * 4 + 2: agg_rows_reg<NT, ITEMS, 3, true, 2>(ab, at, g, ok, R, orv); break;
-        case 4 * 4 + 1: agg_rows_reg<NT, ITEMS, 4, true, 1>(ab, at, g, ok, R, orv); break;
-        case 4 * 4 + 2: agg_rows_reg<NT, ITEMS, 4, true, 2>(ab, at, g, ok, R, orv); break;
-        case 5 * 4 + 1: agg_rows_reg<NT, ITEMS, 5, true, 1>(ab, at, g, ok, R, orv); break;
-        default: agg_rows_reg<NT, ITEMS, 5, true, 2>(ab, at, g, ok, R, orv); break;
+        case 3 * 4 + 1: agg_rows_reg<NT, ITEMS, 3, true, 1, R4>(ab, at, g, ok, R, orv); break;
+        case 3 * 4 + 2: agg_rows_reg<NT, ITEMS, 3, true, 2, R4>(ab, at, g, ok, R, orv); break;
+        case 4 * 4 + 1: agg_rows_reg<NT, ITEMS, 4, true, 1, R4>(ab, at, g, ok, R, orv); break;
+        case 4 * 4 + 2: agg_rows_reg<NT, ITEMS, 4, true, 2, R4>(ab, at, g, ok, R, orv); break;
+        case 5 * 4 + 1: agg_rows_reg<NT, ITEMS, 5, true, 1, R4>(ab, at, g, ok, R, orv); break;
+        default: agg_rows_reg<NT, ITEMS, 5, true, 2, R4>(ab, at, g, ok, R, orv); break;
         }
     } else if (w64) {
         switch (P.nagg) {
-        case 0: agg_rows_reg<NT, ITEMS, 0, true>(ab, at, g, ok, R, orv); break;
-        case 1: agg_rows_reg<NT, ITEMS, 1, true>(ab, at, g, ok, R, orv); break;
-        case 2: agg_rows_reg<NT, ITEMS, 2, true>(ab, at, g, ok, R, orv); break;
-        case 3: agg_rows_reg<NT, ITEMS, 3, true>(ab, at, g, ok, R, orv); break;
-        case 4: agg_rows_reg<NT, ITEMS, 4, true>(ab, at, g, ok, R, orv); break;
-        default: agg_rows_reg<NT, ITEMS, kRegA, true>(ab, at, g, ok, R, orv); break;
+        case 0: agg_rows_reg<NT, ITEMS, 0, true, 0, R4>(ab, at, g, ok, R, orv); break;
+        case 1: agg_rows_reg<NT, ITEMS, 1, true, 0, R4>(ab, at, g, ok, R, orv); break;
+        case 2: agg_rows_reg<NT, ITEMS, 2, true, 0, R4>(ab, at, g, ok, R, orv); break;
+        case 3: agg_rows_reg<NT, ITEMS, 3, true, 0, R4>(ab, at, g, ok, R, orv); break;
+        case 4: agg_rows_reg<NT, ITEMS, 4, true, 0, R4>(ab, at, g, ok, R, orv); break;
+        default: agg_rows_reg<NT, ITEMS, kRegA, true, 0, R4>(ab, at, g, ok, R, orv); break;
         }
     } else {
-        agg_rows_reg<NT, ITEMS, kRegA, false>(ab, at, g, ok, R, orv);
+        agg_rows_reg<NT, ITEMS, kRegA, false, 0, R4>(ab, at, g, ok, R, orv);
     }
     // a narrow value outside its declared bounds: report (err[2]) rather than wrap
     if (orv >> P.narrow_bits)

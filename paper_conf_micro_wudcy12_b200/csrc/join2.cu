@@ -501,7 +501,7 @@ __device__ __forceinline__ uint32_t fastdiv(uint32_t d, uint2 mg)
     return (hi + ((d - hi) >> 1)) >> mg.y;
 }
 
-template <int NT, int ITEMS, int WAYS>
+template <int NT, int ITEMS, int WAYS, bool AGG = false>
 __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_constant__ ChainProg P,
                                                            const __grid_constant__ TileLaunch L,
                                                            const __grid_constant__ JoinEmit X)
@@ -519,6 +519,8 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
     uint32_t *rowbuf = (uint32_t *)(tbuf + 2 * (size_t)P.stage_bytes);   // candidate rows per side
     uint16_t *runidx = (uint16_t *)(rowbuf + (size_t)(WAYS == 3 ? 3 : 2) * T);   // candidate -> run
     char *scratch = (char *)(runidx + T);
+    // aggregate terminal (JOIN -> chain -> AGG): the CTA's 128-bit accumulators instead of a ring
+    unsigned long long *cta_acc = (unsigned long long *)(scratch + P.scratch_bytes);
     char *ring = scratch + P.scratch_bytes;
     const uint32_t R = L.out_bytes;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -543,6 +545,9 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
         ctl->tail = 0;
         fence_mbar_init();
     }
+    if (AGG && P.agg_mode == 2)          // (global-atomic terminal: no CTA accumulators)
+        for (int q = tid; q < P.D * (P.nagg + 1) * 2; q += blockDim.x)
+            cta_acc[q] = 0;
     __syncthreads();
 
     if (warp == NW) {
@@ -629,6 +634,10 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
         int s = 0;
         uint32_t fph = 0;
         uint32_t gv[kJRegCols][ITEMS];                  // register-gathered values of the next tile
+        RegAgg racc;                                    // aggregate terminal: register partials
+        int64_t since_flush = 0;
+        if (AGG)
+            reg_agg_zero(racc);
         char *pend_st = tbuf;
         int pend_rows = 0;
         auto fill = [&](uint32_t idx, int64_t &t) -> bool {
@@ -863,6 +872,18 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                     if (row4<NT>(g) + q < rows)
                         mask0 |= 1u << (g * 4 + q);
             const uint32_t m = run_ops4<NT, G>(P, 0, P.nops, st, scratch, mask0);
+            if constexpr (AGG) {
+                // aggregate terminal: every surviving candidate adds into the partials
+                if (P.agg_mode == 2)
+                    agg_tile_reg<NT, ITEMS, true>(P, st, scratch, m, racc, cta_acc, since_flush, L.err);
+                else
+                    agg_tile_global<NT, ITEMS, true>(P, st, scratch, m, L.agg_acc, L.err);
+                int64_t tn;
+                const bool next = fill(i + 1, tn);
+                t = tn;
+                have = next;
+                continue;
+            }
             uint32_t pk = 0;
 #pragma unroll
             for (int g = 0; g < G; g++)
@@ -975,6 +996,8 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             t = tn;
             have = next;
         }
+        if (AGG && P.agg_mode == 2)
+            reg_agg_reduce_warp(P, racc, cta_acc);   // warp-reduced, 128-bit exact
         if (tid == 0) {
             for (uint32_t u = ublk; u < ublk + kJWriters; ++u) {
                 const int ju = (int)(u % kJSlots);
@@ -986,8 +1009,16 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
         }
     }
     __syncthreads();
-    if (blockIdx.x == 0 && tid == 0 && ntiles == 0)
+    if (AGG) {
+        if (P.agg_mode == 2)
+            for (int q = tid; q < P.D * (P.nagg + 1); q += blockDim.x) {
+                const unsigned long long lo = cta_acc[2 * q], hi = cta_acc[2 * q + 1];
+                if (lo | hi)
+                    atomic_add128(&L.agg_acc[2 * q], &L.agg_acc[2 * q + 1], lo, hi);
+            }
+    } else if (blockIdx.x == 0 && tid == 0 && ntiles == 0) {
         *L.n_dev = 0;
+    }
     cta_exit_reset(L.ctrs);
 }
 
@@ -1021,10 +1052,10 @@ cudaError_t jtiles_launch(const uint64_t *off, const int64_t *totals, int64_t T,
     return cudaGetLastError();
 }
 
-template <int NT, int ITEMS, int WAYS>
+template <int NT, int ITEMS, int WAYS, bool AGG = false>
 static int jocc(size_t smem)
 {
-    auto f = k_join_emit<NT, ITEMS, WAYS>;
+    auto f = k_join_emit<NT, ITEMS, WAYS, AGG>;
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int n = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, NT + kJAux, smem) != cudaSuccess)
@@ -1032,8 +1063,10 @@ static int jocc(size_t smem)
     return n;
 }
 
-int join_emit_occupancy(int nt, int items, int ways, size_t smem)
+int join_emit_occupancy(int nt, int items, int ways, size_t smem, bool agg)
 {
+    if (agg)
+        return ways == 3 ? jocc<256, 8, 3, true>(smem) : jocc<256, 8, 2, true>(smem);
     if (nt == 512)
         return ways == 3 ? jocc<512, 4, 3>(smem) : jocc<512, 4, 2>(smem);
     if (ways == 3)
@@ -1041,17 +1074,19 @@ int join_emit_occupancy(int nt, int items, int ways, size_t smem)
     return items == 4 ? jocc<256, 4, 2>(smem) : jocc<256, 8, 2>(smem);
 }
 
-template <int NT, int ITEMS, int WAYS>
+template <int NT, int ITEMS, int WAYS, bool AGG = false>
 static cudaError_t jgo(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, size_t smem, int grid, cudaStream_t s)
 {
-    cudaFuncSetAttribute(k_join_emit<NT, ITEMS, WAYS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_join_emit<NT, ITEMS, WAYS><<<grid, NT + kJAux, smem, s>>>(P, L, X);
+    cudaFuncSetAttribute(k_join_emit<NT, ITEMS, WAYS, AGG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_join_emit<NT, ITEMS, WAYS, AGG><<<grid, NT + kJAux, smem, s>>>(P, L, X);
     return cudaGetLastError();
 }
 
 cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int nt, int items, int ways,
                              size_t smem, int grid, cudaStream_t s)
 {
+    if (P.is_agg)
+        return ways == 3 ? jgo<256, 8, 3, true>(P, L, X, smem, grid, s) : jgo<256, 8, 2, true>(P, L, X, smem, grid, s);
     if (nt == 512)
         return ways == 3 ? jgo<512, 4, 3>(P, L, X, smem, grid, s) : jgo<512, 4, 2>(P, L, X, smem, grid, s);
     if (ways == 3)

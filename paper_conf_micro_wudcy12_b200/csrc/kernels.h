@@ -105,7 +105,7 @@ cudaError_t jtiles_launch(const uint64_t *off, const int64_t *totals, int64_t T,
 uint32_t join_rec_cap4(int T);
 size_t join_rec_stage_bytes(int ways, int T);
 size_t join_emit_ctl_bytes();
-int join_emit_occupancy(int nt, int items, int ways, size_t smem);
+int join_emit_occupancy(int nt, int items, int ways, size_t smem, bool agg);
 cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const JoinEmit &X, int nt, int items, int ways,
                              size_t smem, int grid, cudaStream_t s);
 

@@ -58,6 +58,9 @@ struct Group {
     // 3-input group (JOIN -> JOIN on the same key, Fig. 14(b)): join_in = the inner JOIN
     // (inputs jl, jr), `join` the outer one (inner output, jc)
     int join_in = -1, jc = -1;
+    // per input (A, B, C): SELECT / key-preserving PROJECT nodes upstream of the JOIN fused
+    // into the expansion (source-to-join order); jl / jr / jc are then their raw sources
+    std::vector<int> prechain[3];
 };
 
 Interval type_range(int t);

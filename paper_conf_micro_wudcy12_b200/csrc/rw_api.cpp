@@ -335,14 +335,25 @@ void setup_join(const rw_plan *p, int jid, Grouping &G, Group &g)
     int np = 0;
     const int left = j.left;
     const Node &ln = p->nodes[left];
+    // an input's upstream SELECT / PROJECT chain (single consumers): key SELECTs go to the
+    // run matching; the rest becomes the side's pre-chain, evaluated on the gathered rows
+    auto side_src = [&](int start, int side) {
+        int nd = absorb_key_selects(p, start, G, g, np, j.nkey);
+        while (p->o.fuse && p->o.reserved[6] != 7 && is_unary_chain(p->nodes[nd].kind) && G.consumers[nd] == 1 &&
+               p->nodes[nd].nkey_sorted >= j.nkey) {
+            g.prechain[side].insert(g.prechain[side].begin(), nd);
+            nd = absorb_key_selects(p, p->nodes[nd].in, G, g, np, j.nkey);
+        }
+        return nd;
+    };
     if (p->o.fuse && ln.kind == N_JOIN && G.consumers[left] == 1 && ln.nkey == j.nkey && p->o.reserved[6] != 5) {
         g.join_in = left;
-        g.jl = absorb_key_selects(p, ln.left, G, g, np, j.nkey);
-        g.jr = absorb_key_selects(p, ln.right, G, g, np, j.nkey);
-        g.jc = absorb_key_selects(p, j.right, G, g, np, j.nkey);
+        g.jl = side_src(ln.left, 0);
+        g.jr = side_src(ln.right, 1);
+        g.jc = side_src(j.right, 2);
     } else {
-        g.jl = absorb_key_selects(p, left, G, g, np, j.nkey);
-        g.jr = absorb_key_selects(p, j.right, G, g, np, j.nkey);
+        g.jl = side_src(left, 0);
+        g.jr = side_src(j.right, 1);
     }
     for (int src : {g.jl, g.jr, g.jc}) {
         if (src < 0) continue;
@@ -364,6 +375,12 @@ int make_group(const rw_plan *p, int id, Grouping &G)
     if (n.kind == N_AGG) {
         g.agg = id;
         cur = n.in;
+        if (fuse && p->nodes[cur].kind == N_JOIN && G.consumers[cur] == 1) {
+            // JOIN -> AGG: the aggregate is the join expansion's terminal (CTA dependence)
+            setup_join(p, cur, G, g);
+            G.groups.push_back(g);
+            return G.produced_by[id] = (int)G.groups.size() - 1;
+        }
         if (!fuse || !is_unary_chain(p->nodes[cur].kind) || G.consumers[cur] != 1) {
             // AGG directly over a relation (or operator-at-a-time mode)
             g.kind = G_SCAN;
@@ -402,16 +419,9 @@ int make_group(const rw_plan *p, int id, Grouping &G)
         chain.assign(1, cur);
         src = p->nodes[cur].in;
     }
-    if (g.agg >= 0 && fuse && p->nodes[src].kind == N_JOIN && G.consumers[src] == 1) {
-        // JOIN -> chain -> AGG: the join expansion materialises the chain's output and
-        // the aggregate scans it (the expansion kernel has no aggregate terminal yet)
-        const int mid = chain.back();
-        g.kind = G_SCAN;
-        g.source = mid;
-        g.deps.push_back(make_group(p, mid, G));
-        G.groups.push_back(g);
-        return G.produced_by[id] = (int)G.groups.size() - 1;
-    }
+    // JOIN -> chain -> AGG: the join expansion's aggregate terminal (X -> AGG is CTA
+    // dependence: block reduction + one global atomic stage), handled below with the
+    // other JOIN -> SELECT / PROJECT groups
     g.chain = chain;
     if (fuse && p->nodes[src].kind == N_JOIN && G.consumers[src] == 1) {
         // JOIN -> SELECT/PROJECT: fused into the join expansion (CTA dependence)
@@ -424,6 +434,16 @@ int make_group(const rw_plan *p, int id, Grouping &G)
     }
     G.groups.push_back(g);
     return G.produced_by[id] = (int)G.groups.size() - 1;
+}
+
+// raw column types of a join group's inputs, side by side (its input slot space)
+std::vector<int> join_src_types(const rw_plan *p, const Group &g)
+{
+    std::vector<int> t;
+    for (int src : {g.jl, g.jr, g.jc})
+        if (src >= 0)
+            for (int ty : p->nodes[src].types) t.push_back(ty);
+    return t;
 }
 
 Grouping build_groups(const rw_plan *p, int out_node)
@@ -527,7 +547,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     cur.resize(src_types.size());
     for (size_t c = 0; c < src_types.size(); c++)
         cur[c] = -1 - (int)c;
-    for (int nid : chain_b) {
+    // one SELECT / PROJECT node applied to the column references `cur` (slot ids, or
+    // -1-c for source column c not yet loaded)
+    auto apply = [&](int nid, std::vector<int> &cur) {
         const Node &nd = p->nodes[nid];
         if (nd.kind == N_SELECT) {
             for (const rw_pred &a : nd.preds) {
@@ -642,7 +664,34 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             }
             cur = next;
         }
+        };
+    if (g.kind == G_JOIN) {
+        // join group: the input slots are the raw columns of the join inputs side by side
+        // (A, B[, C]); each side's pre-chain (SELECT / key-preserving PROJECT fused
+        // upstream of the JOIN, Fig. 13) runs on its own columns: a predicate of
+        // a side holds for a candidate iff it holds for that side's row (bag semantics,
+        // order kept), so it is evaluated on the gathered candidate.  Then the join output
+        // (key, A rest, B rest[, C rest]) is assembled and the downstream chain follows.
+        const int nk = p->nodes[g.join].nkey;
+        const int sides = g.join_in >= 0 ? 3 : 2;
+        const int srcn[3] = {g.jl, g.jr, g.jc};
+        std::vector<int> out;
+        int base = 0;
+        for (int sd = 0; sd < sides; sd++) {
+            const int nc = (int)p->nodes[srcn[sd]].types.size();
+            std::vector<int> cs(nc);
+            for (int c = 0; c < nc; c++)
+                cs[c] = -1 - (base + c);
+            for (int nid : g.prechain[sd])
+                apply(nid, cs);
+            for (size_t c = sd == 0 ? 0 : nk; c < cs.size(); c++)
+                out.push_back(cs[c]);
+            base += nc;
+        }
+        cur = out;
     }
+    for (int nid : chain_b)
+        apply(nid, cur);
     if (nbr > 1) {
         for (int v : cur)
             term.push_back(resolve(v));
@@ -937,7 +986,14 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         bool found = false;
         double best = -1;
         struct JV { int nt, items; };
+        if (L.agg) {
+            // register one-hot partials for small group-bys, else per-row global atomics;
+            // the narrow 32-bit partials are a scan-kernel specialisation (not used here)
+            P.agg_mode = (P.D <= kRegD && P.nagg <= kRegA && P.flush_rows >= (1 << 16)) ? 2 : 3;
+            P.agg_narrow = 0;
+        }
         for (JV jv : {JV{256, 8}, JV{512, 4}, JV{256, 4}}) {
+            if (L.agg && !(jv.nt == 256 && jv.items == 8)) continue;
             const int items = jv.items, ntj = jv.nt;
             if (p->o.reserved[5] > 0 && items != p->o.reserved[5]) continue;
             if (p->o.reserved[4] == 7 ? ntj != 512 : (p->o.reserved[4] == 8 && ntj != 256)) continue;
@@ -946,6 +1002,8 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             size_t W = 0;
             for (int c = 0; c < P.nout; c++)
                 W += (((size_t)T * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
+            if (L.agg)
+                W = P.agg_mode == 2 ? al128((size_t)P.D * (P.nagg + 1) * 16) : 128;   // CTA accumulators, no ring
             const size_t RS = join_rec_stage_bytes(ways, T);
             const size_t base = join_emit_ctl_bytes() + 2 * (size_t)P.stage_bytes + (size_t)ways * T * 4 +
                                 (size_t)T * 2 + P.scratch_bytes;
@@ -957,9 +1015,10 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 if (base + S * RS + W > per_cta) continue;
                 size_t Rb = (per_cta - base - S * RS) / 128 * 128;
                 if (p->o.reserved[0] > 0) Rb = std::min(Rb, (size_t)p->o.reserved[0] * 1024);
+                if (L.agg) Rb = W;
                 if (Rb < W) continue;
                 const size_t smem = base + S * RS + Rb;
-                if (join_emit_occupancy(ntj, items, ways, smem) < occ_t) continue;
+                if (join_emit_occupancy(ntj, items, ways, smem, L.agg) < occ_t) continue;
                 const double q = (double)Rb / (double)W;
                 const double sc = (q >= 2.0 ? 1e9 : q * 1e8) + T * 1e3 + ntj + S;
                 if (sc > best) {
@@ -1354,7 +1413,7 @@ void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void
     const int T = 0;   // set below from the lowering
     (void)T;
     Lowered L;
-    lower(p, g, jn.types, L);
+    lower(p, g, join_src_types(p, g), L);
     const int64_t T2 = L.tile;
     const double maxc = three ? (double)na * (double)nb * (double)nc : (double)na * (double)nb;
     // tile index capacity: every candidate when that is below 2^34 (no host sync), else
@@ -1456,7 +1515,8 @@ void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void
     }
     if (exact_tiles)
         ensure_status(p, p->status_used + cap_tiles + 1);
-    make_output(X, gi, outn.types, gi == X.final_group ? X.out->capacity : total_host, o, outp, capacity, n_dev);
+    make_output(X, gi, outn.types, gi == X.final_group ? X.out->capacity : (L.agg ? p->nodes[g.agg].D : total_host), o,
+                outp, capacity, n_dev);
     // ---- tile index ----
     int64_t *tile_run = (int64_t *)temp_alloc(p, (size_t)std::max<int64_t>(cap_tiles, 2) * 8);
     int32_t *ovf = (int32_t *)(p->err + 8);
@@ -1466,15 +1526,15 @@ void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void
     XJ.tile_run = tile_run;
     XJ.rec_cap4 = join_rec_cap4((int)T2);
     XJ.rec_stage_bytes = (uint32_t)join_rec_stage_bytes(three ? 3 : 2, (int)T2);
-    // join output column -> (input, column): (key, A rest, B rest[, C rest])
+    // input slot -> (input, raw column): the slot space is A's, B's[, C's] columns side by side
     const int nac = (int)ra.types.size(), nbc = (int)rb.types.size();
     XJ.ncols = L.P.nin;
     for (int i = 0; i < L.P.nin; i++) {
         const int c = L.in_src[i];
         int side, col;
         if (c < nac) { side = 0; col = c; }
-        else if (c < nac + nbc - nkey) { side = 1; col = c - nac + nkey; }
-        else { side = 2; col = c - (nac + nbc - nkey) + nkey; }
+        else if (c < nac + nbc) { side = 1; col = c - nac; }
+        else { side = 2; col = c - nac - nbc; }
         const Rel &src = side == 0 ? ra : side == 1 ? rb : rc;
         XJ.src[i] = src.cols[col];
         XJ.side[i] = (uint8_t)side;
@@ -1498,8 +1558,25 @@ void run_join_group(ExecCtx &X, int gi, const Group &g, Rel &o, std::vector<void
     TL.out_bytes = L.out_bytes;
     TL.dbg = p->o.reserved[1];
     const int grid = p->sms * L.ctas;
+    unsigned long long *acc = nullptr;
+    if (L.agg) {
+        const size_t words = (size_t)p->nodes[g.agg].D * (L.P.nagg + 1) * 2;
+        acc = agg_buffer(p, g.agg, words);
+        TL.agg_acc = acc;
+    }
     cuda_check(join_emit_launch(L.P, TL, XJ, L.nt, L.items, three ? 3 : 2, L.smem, grid, p->stream), "k_join_emit");
     p->launches++;
+    if (L.agg) {
+        L.F.acc = acc;
+        L.F.acc_w = acc;
+        for (size_t c = 0; c < outp.size(); c++)
+            L.F.out[c] = outp[c];
+        L.F.capacity = capacity;
+        L.F.n_dev = n_dev;
+        L.F.err = p->err;
+        cuda_check(agg_finalize_launch(L.F, p->stream), "k_agg_finalize");
+        p->launches++;
+    }
 }
 
 void run_group(ExecCtx &X, int gi)
@@ -2005,7 +2082,10 @@ std::string explain(rw_plan *p, int out_node)
                 const Group &g = G.groups[q];
                 if (g.out == (int)i || g.join == (int)i || g.join_in == (int)i || g.agg == (int)i ||
                     std::find(g.chain.begin(), g.chain.end(), (int)i) != g.chain.end() ||
-                    std::find(g.pre.begin(), g.pre.end(), (int)i) != g.pre.end())
+                    std::find(g.pre.begin(), g.pre.end(), (int)i) != g.pre.end() ||
+                    std::find(g.prechain[0].begin(), g.prechain[0].end(), (int)i) != g.prechain[0].end() ||
+                    std::find(g.prechain[1].begin(), g.prechain[1].end(), (int)i) != g.prechain[1].end() ||
+                    std::find(g.prechain[2].begin(), g.prechain[2].end(), (int)i) != g.prechain[2].end())
                     gc = (int)q;
             }
             bool fused = false;
@@ -2013,7 +2093,10 @@ std::string explain(rw_plan *p, int out_node)
                 const Group &g = G.groups[gc];
                 fused = pr == g.join || (g.join_in >= 0 && pr == g.join_in) ||
                         std::find(g.chain.begin(), g.chain.end(), pr) != g.chain.end() ||
-                        std::find(g.pre.begin(), g.pre.end(), pr) != g.pre.end();
+                        std::find(g.pre.begin(), g.pre.end(), pr) != g.pre.end() ||
+                        std::find(g.prechain[0].begin(), g.prechain[0].end(), pr) != g.prechain[0].end() ||
+                        std::find(g.prechain[1].begin(), g.prechain[1].end(), pr) != g.prechain[1].end() ||
+                        std::find(g.prechain[2].begin(), g.prechain[2].end(), pr) != g.prechain[2].end();
             }
             (void)gp;
             s << "  " << pr << "(" << kn[p->nodes[pr].kind] << ") -> " << i << "(" << kn[n.kind]
@@ -2036,6 +2119,10 @@ std::string explain(rw_plan *p, int out_node)
         else if (g.join_in >= 0) s << "joins " << g.join_in << " -> " << g.join << " (3 inputs, mixed-radix expansion)";
         else s << "join " << g.join;
         for (int c : g.pre) s << ", key SELECT " << c << " (fused into the run matching)";
+        for (int sd = 0; sd < 3; sd++)
+            for (int c : g.prechain[sd])
+                s << ", " << kn[p->nodes[c].kind] << " " << c << " (upstream of the join, input " << sd
+                  << ", fused into the expansion)";
         for (int c : g.chain) s << ", " << kn[p->nodes[c].kind] << " " << c;
         if (g.agg >= 0) s << ", AGG " << g.agg;
         s << "] -> node " << g.out;
@@ -2046,7 +2133,7 @@ std::string explain(rw_plan *p, int out_node)
         }
         try {
             Lowered L;
-            std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : p->nodes[g.join].types;
+            std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : join_src_types(p, g);
             lower(p, g, st, L);
             if (L.emit)
                 s << " | emitting kernel k_scan_emit<" << L.nt << "," << L.items << ">"

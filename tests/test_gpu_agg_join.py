@@ -171,8 +171,8 @@ def test_join_then_aggregate():
 
 def test_pattern_c_selects_upstream_of_join():
     """Fig. 14(c) shape: SELECTs on both JOIN inputs, then the join and a
-    downstream SELECT + PROJECT.  The upstream SELECTs keep key order (their outputs
-    stay join-able); they run as their own materialised groups (N2 not fused)."""
+    downstream SELECT + PROJECT.  The upstream value SELECTs are fused into the join's
+    expansion (N2, Fig. 13): one kernel group."""
     spec = workloads.c3_spec()
     spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(1, "<", workloads.thr_u32(0.6))]},
                      {"id": "fr", "op": "select", "in": "R", "preds": [(1, ">=", workloads.thr_u32(0.3))]},
@@ -180,7 +180,8 @@ def test_pattern_c_selects_upstream_of_join():
     ins = workloads.c3_inputs(30_000, device=DEV, cfg=0x96)
     got, plan = run_gpu(spec, ins, capacity=400_000)
     assert_same(got, run_oracle(spec, ins))
-    assert "materialised" in plan.explain(plan.out_id)
+    ex = plan.explain(plan.out_id)
+    assert "group 1" not in ex and ex.count("fused into the expansion") == 2, ex
 
 
 @pytest.mark.parametrize("n", [0, 1000, 30_000, 200_000])
@@ -204,7 +205,8 @@ def test_n2_key_selects_fused_into_join(n, fuse):
 
 
 def test_n2_mixed_key_and_value_selects():
-    """A key SELECT on L is fused; a value SELECT on R stays a materialised group."""
+    """A key SELECT on L is fused into the run matching; a value SELECT on R is fused into
+    the expansion (evaluated on the gathered R row of every candidate): one group."""
     spec = workloads.c3_spec()
     spec["nodes"] = [{"id": "fl", "op": "select", "in": "L", "preds": [(0, ">", workloads.thr_u32(0.1))]},
                      {"id": "fr", "op": "select", "in": "R", "preds": [(1, "<", workloads.thr_u32(0.5))]},
@@ -213,7 +215,7 @@ def test_n2_mixed_key_and_value_selects():
     got, plan = run_gpu(spec, ins, capacity=500_000)
     assert_same(got, run_oracle(spec, ins))
     ex = plan.explain(plan.out_id)
-    assert ex.count("key SELECT") == 1 and "group 1" in ex
+    assert ex.count("key SELECT") == 1 and "group 1" not in ex and "upstream of the join, input 1" in ex, ex
 
 
 def test_n2_signed_keys():
