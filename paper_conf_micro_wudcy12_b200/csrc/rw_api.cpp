@@ -276,6 +276,7 @@ Interval expr_interval(const Node &in, const std::vector<rw_expr> &e, int i, std
 // ---------------------------------------------------------------------------
 struct Grouping {
     std::vector<Group> groups;
+    std::vector<int> cuts;              // nodes split at by the resource budget (Algorithm 2)
     std::map<int, int> produced_by;     // node -> group index
     std::vector<int> consumers;         // within the reachable sub-DAG
     std::vector<char> reach;
@@ -446,12 +447,17 @@ std::vector<int> join_src_types(const rw_plan *p, const Group &g)
     return t;
 }
 
-Grouping build_groups(const rw_plan *p, int out_node)
+Grouping build_groups_once(const rw_plan *p, int out_node, const std::vector<int> &cuts)
 {
     Grouping G;
     G.consumers.assign(p->nodes.size(), 0);
     G.reach.assign(p->nodes.size(), 0);
     mark_reach(p, out_node, G);
+    // nodes Algorithm 2 split at (resource budget): their output is materialised, so
+    // they count as having a further consumer
+    for (int c : cuts)
+        G.consumers[c] += 1;
+    G.cuts = cuts;
     for (size_t i = 0; i < p->nodes.size(); i++) {
         if (!G.reach[i]) continue;
         const Node &n = p->nodes[i];
@@ -1268,6 +1274,81 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
             W += (((size_t)L.tile * type_width(P.slot[P.out_slot[c]].type)) + 15) / 16 * 16;
         L.gring_bytes = (uint32_t)std::max<size_t>(want_ring ? want_ring : 128 * 1024, 4 * W);
         L.out_bytes = L.gring_bytes;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Algorithm 2 analogue (§4.2, §4.3.3; reading A20): operators are
+// fused greedily, earliest first, while the group's kernel fits its resource budget
+// (micro-ops, tile columns, shared memory); a group that does not fit is split after
+// its longest fitting prefix, whose output is then materialised, and the grouping is
+// rebuilt.  A single operator that does not fit is an error (RW_E_UNSUPPORTED).
+// ---------------------------------------------------------------------------
+bool lowers(rw_plan *p, const Group &g)
+{
+    try {
+        Lowered L;
+        lower(p, g, g.kind == G_SCAN ? p->nodes[g.source].types : join_src_types(p, g), L);
+        return true;
+    } catch (const RwError &e) {
+        if (e.s != RW_E_UNSUPPORTED)
+            throw;
+        return false;
+    }
+}
+
+Grouping build_groups(const rw_plan *p_, int out_node)
+{
+    rw_plan *p = const_cast<rw_plan *>(p_);
+    std::vector<int> cuts;
+    for (int iter = 0;; iter++) {
+        Grouping G = build_groups_once(p, out_node, cuts);
+        if (!p->o.fuse || iter > (int)p->nodes.size())
+            return G;
+        int cut = -1;
+        for (const Group &g : G.groups) {
+            if (g.kind == G_SET || lowers(p, g))
+                continue;
+            const std::vector<int> &c = g.chain;
+            const int k = (int)c.size();
+            if (g.kind == G_SCAN) {
+                for (int m = k; m >= 1 && cut < 0; m--) {
+                    Group h = g;
+                    h.chain.assign(c.begin(), c.begin() + m);
+                    h.agg = -1;
+                    h.out = c[m - 1];
+                    if (lowers(p, h))
+                        cut = c[m - 1];
+                }
+            } else {
+                for (int m = k; m >= 0 && cut < 0; m--) {
+                    Group h = g;
+                    h.chain.assign(c.begin(), c.begin() + m);
+                    h.agg = -1;
+                    h.out = m > 0 ? c[m - 1] : g.join;
+                    if (lowers(p, h))
+                        cut = m > 0 ? c[m - 1] : g.join;
+                }
+                if (cut < 0) {
+                    // the expansion alone does not fit: materialise an upstream pre-chain, else
+                    // the inner JOIN of a 3-input group
+                    int best = -1;
+                    for (int sd = 0; sd < 3; sd++)
+                        if (!g.prechain[sd].empty() && (best < 0 || g.prechain[sd].size() > g.prechain[best].size()))
+                            best = sd;
+                    if (best >= 0) cut = g.prechain[best].back();
+                    else if (g.join_in >= 0) cut = g.join_in;
+                }
+            }
+            if (cut < 0 || std::find(cuts.begin(), cuts.end(), cut) != cuts.end()) {
+                Lowered L;   // rethrows the budget error of the group that cannot be split
+                lower(p, g, g.kind == G_SCAN ? p->nodes[g.source].types : join_src_types(p, g), L);
+            }
+            break;
+        }
+        if (cut < 0)
+            return G;
+        cuts.push_back(cut);
     }
 }
 
@@ -2104,6 +2185,9 @@ std::string explain(rw_plan *p, int out_node)
               << (fused ? "fused" : "materialised") << "\n";
         }
     }
+    for (int c : G.cuts)
+        s << "split by the resource budget (Algorithm 2, P:167-171): node " << c << "(" << kn[p->nodes[c].kind]
+          << ") materialised\n";
     s << "groups:\n";
     for (size_t q = 0; q < G.groups.size(); q++) {
         const Group &g = G.groups[q];

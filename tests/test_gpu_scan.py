@@ -190,3 +190,47 @@ def test_explain_reports_fused_thread_dependence():
     assert txt.count("group ") == 1
     plan0, ids0 = build_gpu_plan(spec, fuse=False)
     assert plan0.explain(ids0["s2"]).count("group ") == 3
+
+
+def _long_chain_spec(nproj, per):
+    """nproj PROJECT nodes over (i64 x 3), each computing `per` wrapping sums and keeping
+    three columns, then a SELECT: too many micro-ops for one fused group when long."""
+    nodes, src = [], "R"
+    for k in range(nproj):
+        ex = [("col", 0, "i64"), ("col", 1, "i64"), ("col", 2, "i64")]
+        acc = 1
+        for q in range(per):
+            ex.append(("add", acc, q % 3, "i64"))
+            acc = len(ex) - 1
+        nodes.append({"id": f"p{k}", "op": "project", "in": src, "exprs": ex, "roots": [0, acc, 2]})
+        src = f"p{k}"
+    nodes.append({"id": "s", "op": "select", "in": src, "preds": [(1, "<", 0)]})
+    return {"inputs": {"R": {"types": ["i64"] * 3, "nkey_sorted": 0}}, "nodes": nodes, "out": "s"}
+
+
+@pytest.mark.parametrize("n", [1, 5000, 100_003])
+def test_algorithm2_splits_over_budget_groups(n):
+    """Algorithm 2: a chain whose fused kernel would exceed the micro-op
+    budget is split greedily (longest fitting prefix first), the prefix materialised;
+    result identical to the oracle and to operator-at-a-time."""
+    import torch
+    spec = _long_chain_spec(8, 9)
+    g = torch.Generator().manual_seed(n)
+    ins = {"R": [torch.randint(-(2**40), 2**40, (n,), dtype=torch.int64, generator=g).to(DEV) for _ in range(3)]}
+    ref = run_oracle(spec, ins)
+    got, plan = run_gpu(spec, ins, capacity=max(n, 1))
+    assert_same(got, ref)
+    ex = plan.explain(plan.out_id)
+    assert "Algorithm 2" in ex and "group 1" in ex, ex
+    got0, _ = run_gpu(spec, ins, capacity=max(n, 1), fuse=False)
+    assert_same(got0, ref)
+
+
+def test_single_operator_over_budget_is_an_error():
+    from paper_conf_micro_wudcy12_b200 import rw
+    spec = _long_chain_spec(1, 60)
+    import torch
+    ins = {"R": [torch.zeros(10, dtype=torch.int64, device=DEV) for _ in range(3)]}
+    with pytest.raises(rw.RwError) as e:
+        run_gpu(spec, ins)
+    assert "RW_E_UNSUPPORTED" in str(e.value)
