@@ -55,6 +55,10 @@ def parse():
     ap.add_argument("--no-unfused", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-rows", type=int, default=0)
+    ap.add_argument("--cpu-worker", action="store_true", help=argparse.SUPPRESS)
+    ap.add_argument("--cpu-start", type=int, default=0, help=argparse.SUPPRESS)
+    ap.add_argument("--cpu-core", type=int, default=0, help=argparse.SUPPRESS)
+    ap.add_argument("--no-sweep", action="store_true", help="skip the selectivity / size sweeps")
     ap.add_argument("--stages", type=int, default=0, help="TMA stages per CTA (0 = auto)")
     ap.add_argument("--ctas", type=int, default=0, help="CTAs per SM cap (0 = auto)")
     ap.add_argument("--defer", type=int, default=0, help="scan store delay in tiles (0 = auto)")
@@ -153,6 +157,9 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+NOMINAL_HBM_GBS = 8000.0     # BASELINE.json "about 8 TB/s HBM3e" (DGX B200 figure; 7.7 TB/s HGX)
+
+
 def measured_peak():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -173,15 +180,25 @@ def ncu_traffic(cfg: str):
         return None
 
 
-def cpu_oracle_sample(cfg: str, rows: int, sample_rows: int):
-    """Time the oracle (single thread) on a bounded prefix sample of the same workload."""
+ROW_SHARDABLE = ("c1", "c2", "c4", "cd")
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def cpu_oracle_sample(cfg: str, rows: int, sample_rows: int, start: int = 0):
+    """Time the oracle (single thread) on a bounded sample (rows [start, start + m)) of
+    the same workload."""
     import oracle
-    from tests.planspec import run_oracle
     m = min(rows, sample_rows)
-    if cfg == "c3":
-        spec, ins = spec_and_inputs(cfg, m, 0, "cpu")
-    else:
-        spec, ins = spec_and_inputs(cfg, m, 0, "cpu")
+    spec, ins = spec_and_inputs(cfg, m, start, "cpu")
     rels = {}
     import numpy as np
     npt = {"i32": np.int32, "u32": np.uint32, "i64": np.int64, "u64": np.uint64, "u8": np.uint8}
@@ -194,6 +211,59 @@ def cpu_oracle_sample(cfg: str, rows: int, sample_rows: int):
     return n_in / dt, dt, n_in
 
 
+def cpu_worker(args):
+    """Child process of the CPU legs: pinned to one core, one oracle evaluation over its
+    rows; prints {"n_in", "seconds"}."""
+    try:
+        os.sched_setaffinity(0, {args.cpu_core})
+    except (AttributeError, OSError):
+        pass
+    os.environ["OMP_NUM_THREADS"] = "1"
+    v, dt, n_in = cpu_oracle_sample(args.config, args.cpu_rows, args.cpu_rows, args.cpu_start)
+    print(json.dumps({"n_in": n_in, "seconds": dt}), flush=True)
+    return 0
+
+
+def cpu_legs(cfg: str, rows: int, sample: int, multi: bool = True):
+    """The oracle on the box's host cores: one process pinned to one core (sched_setaffinity)
+    over a bounded sample, and for row-shardable chains N independent pinned processes over
+    N row shards of the same size (N = the cores this process may run on).  Returns the
+    cpu_baseline object."""
+    import subprocess
+    import oracle
+    oracle.build()
+    cores = sorted(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else [0]
+    base = [sys.executable, os.path.abspath(__file__), "--config", cfg, "--cpu-worker"]
+    if cfg == "cd":
+        base += ["--branches", str(BRANCHES)]
+    if cfg == "cs":
+        base += ["--setop", SETOP]
+    m = min(rows, sample)
+
+    def launch(core, start):
+        return subprocess.Popen(base + ["--cpu-rows", str(m), "--cpu-start", str(start), "--cpu-core", str(core)],
+                                stdout=subprocess.PIPE, text=True)
+
+    def result(pr):
+        out, _ = pr.communicate()
+        return json.loads([l for l in out.splitlines() if l.startswith("{")][-1])
+
+    one = result(launch(cores[0], 0))
+    v1 = one["n_in"] / one["seconds"]
+    out = {"value": v1, "unit": "tuples/s", "cores": 1, "kind": "oracle", "pinned": f"core {cores[0]} (sched_setaffinity)",
+           "sample": f"input tuples [0, {one['n_in']}) of the same workload, one pinned process ({one['seconds']:.2f} s)",
+           "cpu_model": cpu_model()}
+    if multi and cfg in ROW_SHARDABLE and len(cores) > 1 and m == sample:
+        prs = [launch(c, k * m) for k, c in enumerate(cores)]
+        res = [result(pr) for pr in prs]
+        wall = max(r["seconds"] for r in res)
+        n_all = sum(r["n_in"] for r in res)
+        out["all_cores"] = {"value": n_all / wall, "unit": "tuples/s", "cores": len(cores),
+                            "sample": f"{len(cores)} independent pinned processes, row shards of {m} rows each "
+                                      f"(slowest {wall:.2f} s)"}
+    return out
+
+
 def run_reference(args):
     rank, world, local = dist_env()
     if rank != 0:
@@ -203,6 +273,10 @@ def run_reference(args):
     sample = args.cpu_rows or {"c1": rows, "c2": 1 << 24, "c3": 1 << 21, "c4": 1 << 23, "c5": 1 << 21, "cd": 1 << 24, "cs": 1 << 21, "cc": 1 << 21}[cfg]
     import oracle
     oracle.build()
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})   # one pinned host core
+    except (AttributeError, OSError):
+        pass
     vals = []
     for i in range(args.warmup + args.steps):
         v, dt, n_in = cpu_oracle_sample(cfg, rows, sample)
@@ -217,10 +291,75 @@ def run_reference(args):
             "config": {"workload": CONFIGS[cfg]["name"], "sample_rows": vals[0][2],
                        "note": "reference arm = the CPU oracle (single thread) on a bounded prefix sample"},
             "cpu_baseline": {"value": value, "unit": "tuples/s", "cores": 1, "kind": "oracle",
-                             "sample": f"first {vals[0][2]} input tuples of {cfg}"},
+                             "sample": f"first {vals[0][2]} input tuples of {cfg}, one pinned core",
+                             "cpu_model": cpu_model()},
             "e2e": {"value": value, "unit": "tuples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+def sweeps(cfg, local, stream, dev, args):
+    """Selectivity sweep s in {0.1, 0.5, 0.9} for both SELECTs (Fig. 20) on C1 and C2,
+    and the C1 size sweep 2^20 .. 2^30 tuples (Fig. 4): fused vs operator-at-a-time
+    per point, CUDA events, L2 flushed before each step when the input fits in L2."""
+    import torch
+    from tests.planspec import build_gpu_plan
+    dtn = {"i32": torch.int32, "u32": torch.int32, "i64": torch.int64, "u64": torch.int64, "u8": torch.uint8}
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    out = {}
+
+    def point(spec, ins, steps=5):
+        n = int(next(iter(ins.values()))[0].numel())
+        inputs = [(n, ins[k]) for k in spec["inputs"]]
+        nb = workloads.input_bytes(spec, {k: n for k in spec["inputs"]})
+        res = {}
+        for fuse in (True, False):
+            plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse)
+            node = ids[spec["out"]]
+            types = plan.node_schema(node)
+            outs = [torch.empty(n, dtype=dtn[t], device=dev) for t in types]
+            nd = torch.zeros(1, dtype=torch.int64, device=dev)
+            for _ in range(2):
+                plan.execute(inputs, node, outs, n, n_dev=nd)
+            ts = []
+            for _ in range(steps):
+                if nb < (512 << 20):
+                    flush.zero_()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                plan.execute(inputs, node, outs, n, n_dev=nd)
+                e1.record(stream)
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ms = statistics.median(ts)
+            res["fused_ms" if fuse else "unfused_ms"] = ms
+            if fuse:
+                res["tuples_per_s"] = n / (ms / 1e3)
+                res["out_rows"] = int(nd.item())
+            del outs, plan
+        res["speedup"] = res["unfused_ms"] / res["fused_ms"]
+        return res
+
+    sel = {}
+    for sv in (0.1, 0.5, 0.9):
+        if cfg == "c1":
+            spec, ins = workloads.c1_spec(sv, sv), workloads.c1_inputs(workloads.C1_ROWS, 0, dev)
+        else:
+            spec, ins = workloads.c2_spec(sv, sv), workloads.c2_inputs(workloads.C2_ROWS, 0, dev)
+        sel[str(sv)] = point(spec, ins)
+        del ins
+        torch.cuda.empty_cache()
+    out["selectivity"] = sel
+    if cfg == "c1":
+        size = {}
+        for lg in range(20, 31, 2):
+            ins = workloads.c1_inputs(1 << lg, 0, dev)
+            size[f"2^{lg}"] = point(workloads.c1_spec(), ins)
+            del ins
+            torch.cuda.empty_cache()
+        out["size"] = size
+    out["note"] = "median of 5 CUDA-event steps per point; speedup = operator-at-a-time / fused time"
+    return out
 
 
 def main():
@@ -228,6 +367,8 @@ def main():
     global BRANCHES, SETOP
     BRANCHES = args.branches
     SETOP = args.setop
+    if args.cpu_worker:
+        return cpu_worker(args)
     if args.impl == "reference":
         return run_reference(args)
     import torch
@@ -367,6 +508,7 @@ def main():
     kname = {"c3": "k_join_runs + k_join_expand", "cc": "k_join_runs (key SELECTs fused) + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand",
              "cs": "k_set_splits + k_set_op x2 + k_set_scan"}.get(cfg, "k_scan_chain")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "frac_nominal": achieved / NOMINAL_HBM_GBS, "nominal_peak": NOMINAL_HBM_GBS,
                 "traffic": ncu_traffic(cfg), "kernel": kname,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src,
                 "note": "achieved = (input bytes + compacted output bytes) / CUDA-event time per step; "
@@ -375,7 +517,8 @@ def main():
     par = {"c5": f"key-range shard x{world} (all_to_all)", "cs": f"key-range shard x{world} (all_to_all)",
            "c4": f"row-shard x{world} + limb all-reduce"}
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
+            "ms_median": statistics.median(per), "ms_min": min(per), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs", "cc") else "i32"),
             "data": "synthetic (rwgen seeded SplitMix64 generators, generated on device)",
             "config": {"workload": CONFIGS[cfg]["name"], "rows_per_gpu": nrows, "output_rows_per_gpu": n_out,
@@ -393,8 +536,25 @@ def main():
         uv = n_in * world / (ut / 1e3 / us)
         line["unfused"] = {"value": uv, "ms_per_step": ut / us, "gpu_launches_per_step": ul / us,
                            "speedup_fused_vs_unfused": value / uv,
-                           "roofline_frac_same_numerator": alg_bytes / (ut / us / 1e3) / 1e9 / peak}
+                           "roofline_frac_same_numerator": alg_bytes / (ut / us / 1e3) / 1e9 / peak,
+                           "note": "operator at a time: every intermediate relation materialised (PROJECT copies its columns)"}
         del uouts, uplan
+        torch.cuda.empty_cache()
+        # stricter baseline: a PROJECT of plain column references aliases its input columns
+        zplan, zids = build_gpu_plan(spec, device=local, stream=stream, fuse=False, zero_copy_project=True)
+        zcap = cap
+        zouts = [torch.empty(zcap, dtype=dtn[t], device=dev) for t in out_types] if "outs" not in spec else None
+        if zouts is not None:
+            zt, _, zl, _ = timed(make_step(zplan, zids, zouts, zcap), us, 2)
+            zv = n_in * world / (zt / 1e3 / us)
+            line["unfused_zero_copy"] = {"value": zv, "ms_per_step": zt / us, "gpu_launches_per_step": zl / us,
+                                         "speedup_fused_vs_unfused": value / zv,
+                                         "note": "operator at a time with zero-copy PROJECT (column aliases)"}
+        del zouts, zplan
+        torch.cuda.empty_cache()
+
+    if not args.no_sweep and cfg in ("c1", "c2") and world == 1 and not args.rows:
+        line["sweeps"] = sweeps(cfg, local, stream, dev, args)
         torch.cuda.empty_cache()
 
     if not args.no_e2e and cfg in ("c1", "c2", "c4"):
@@ -427,10 +587,8 @@ def main():
         del host_in, host_out
 
     if rank == 0 and not args.no_cpu:
-        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 26, "c3": 1 << 22, "c4": 1 << 24, "c5": 1 << 22, "cd": 1 << 26, "cs": 1 << 22, "cc": 1 << 22}[cfg]
-        v, dt, n_s = cpu_oracle_sample(cfg, rows, sample)
-        line["cpu_baseline"] = {"value": v, "unit": "tuples/s", "cores": 1, "kind": "oracle",
-                                "sample": f"first {n_s} input tuples of the same workload ({dt:.2f} s, 1 thread)"}
+        sample = args.cpu_rows or {"c1": rows, "c2": 1 << 25, "c3": 1 << 22, "c4": 1 << 23, "c5": 1 << 22, "cd": 1 << 25, "cs": 1 << 22, "cc": 1 << 22}[cfg]
+        line["cpu_baseline"] = cpu_legs(cfg, rows, sample)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if pg:

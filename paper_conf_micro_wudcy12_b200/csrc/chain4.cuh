@@ -211,4 +211,29 @@ __device__ __forceinline__ uint32_t run_ops4(const ChainProg &P, int op0, int op
     return mask;
 }
 
+// Compacted-store slow path of the emitting kernels: the survivors of the thread's
+// groups (positions sp) of one column, into a circular ring whose segment for this
+// column starts at byte `so` and wraps at R.
+template <int NT, int G>
+__device__ __forceinline__ void wrap_scatter(char *ring, uint32_t R, uint32_t so, int w, const char *src, uint32_t m,
+                                          const uint32_t (&sp)[G][4])
+{
+    for (int g = 0; g < G; g++) {
+        const uint32_t m4 = (m >> (4 * g)) & 15u;
+        if (!m4)
+            continue;
+        const int r0 = row4<NT>(g);
+        for (int q = 0; q < 4; q++) {
+            if (!((m4 >> q) & 1u))
+                continue;
+            uint32_t b = so + sp[g][q] * (uint32_t)w;
+            if (b >= R)
+                b -= R;
+            if (w == 4) *(uint32_t *)(ring + b) = ((const uint32_t *)src)[r0 + q];
+            else if (w == 8) *(uint64_t *)(ring + b) = ((const uint64_t *)src)[r0 + q];
+            else ring[b] = src[r0 + q];
+        }
+    }
+}
+
 }  // namespace rw

@@ -127,7 +127,7 @@ struct TileLaunch {
                                // 2 = stream tiles only, 4 = per-tile phase timestamps into dbg_ts
     int32_t delay;             // emitting scan kernel: compute warps hold at most `delay` evaluated tiles
                                // (in their input stages) waiting for their global offsets
-    uint32_t warp_buf;         // emitting scan kernel: bytes of each compute warp's compaction buffer
+    uint32_t gring_bytes;      // emitting scan kernel: bytes of each CTA's L2 ring slice (gring != nullptr)
     uint64_t *dbg_ts;          // 12 globaltimer stamps per tile (claim, data, evaluated, offset, stored, writer start, ops, ballots, scattered, reserve start; join: records cached, gathered)
 };
 

@@ -602,15 +602,24 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             const int64_t excl = (int64_t)lookback_warp(L.status, t, tot, L.epoch, /*aggregate_published=*/true);
             if (lane == 0 && t == ntiles - 1)
                 *L.n_dev = excl + (int64_t)tot;
-            const char *blk = ring + ctl->blk[j].roff;
+            const uint32_t roff = ctl->blk[j].roff;
             uint32_t coff = 0;
             for (int c = 0; c < P.nout; c++) {
                 const int w = P.out_w[c];
-                const char *src = blk + coff;
+                // the ring is circular: a column's segment may wrap at R (16-byte aligned,
+                // so no vector straddles the end) -> copied in two pieces
+                const uint32_t so = (roff + coff) % R;
                 coff += al16j(tot * w);
-                if (w == 4) emit_copy_j<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, tot, P.out_capacity, lane);
-                else if (w == 8) emit_copy_j<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, tot, P.out_capacity, lane);
-                else emit_copy_j<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, tot, P.out_capacity, lane);
+                const uint32_t n1 = min(tot, (R - so) / (uint32_t)w);
+                for (int piece = 0; piece < 2; piece++) {
+                    const char *src = piece ? ring : ring + so;
+                    const int64_t at = piece ? excl + n1 : excl;
+                    const uint32_t cnt = piece ? tot - n1 : n1;
+                    if (cnt == 0) continue;
+                    if (w == 4) emit_copy_j<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, at, cnt, P.out_capacity, lane);
+                    else if (w == 8) emit_copy_j<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, at, cnt, P.out_capacity, lane);
+                    else emit_copy_j<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, at, cnt, P.out_capacity, lane);
+                }
             }
             __syncwarp();
             if (lane == 0) {
@@ -919,29 +928,20 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             int64_t tn;
             const bool next = fill(i + 1, tn);
             const uint32_t need = P.br_nw[0][0] * al16j(tot) + P.br_nw[0][1] * al16j(tot * 4u) + P.br_nw[0][2] * al16j(tot * 8u);
-            uint32_t pos = hpos, used = need;
-            bool drain = false;
-            if (pos + need > R) {
-                used += R - pos;
-                pos = 0;
-                if (used > R) {
-                    used = need;
-                    drain = true;
-                }
-            }
+            // circular ring: a block may wrap at R; wait until its bytes are free
+            const uint32_t pos = hpos, used = need;
             const int j = (int)(ublk % kJSlots);
             if (ublk >= kJSlots)
                 mbar_wait(&ctl->blk[j].oempty, ((ublk / kJSlots) - 1) & 1u);
             {
                 uint32_t backoff = 64;
-                while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
+                while (head + used - ctl->tail > R) {
                     __nanosleep(backoff);
                     backoff = backoff < 1024 ? backoff * 2 : 1024;
                 }
             }
             head += used;
-            hpos = pos + need == R ? 0 : pos + need;
-            char *blk = ring + pos;
+            hpos = pos + need >= R ? pos + need - R : pos + need;
             uint32_t sp[G][4];
 #pragma unroll
             for (int g = 0; g < G; g++) {
@@ -956,8 +956,14 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             for (int c = 0; c < P.nout; c++) {
                 const int w = P.out_w[c];
                 const char *src = loc_ptr(P.out_loc[c], st, scratch);
-                char *d = blk + coff;
+                const uint32_t so = (pos + coff) % R;
                 coff += al16j(tot * w);
+                if (so + tot * (uint32_t)w > R) {
+                    // this column's segment wraps at the ring's end: positions mod R
+                    wrap_scatter<NT, G>(ring, R, so, w, src, m, sp);
+                    continue;
+                }
+                char *d = ring + so;
 #pragma unroll
                 for (int g = 0; g < G; g++) {
                     const uint32_t m4 = (m >> (4 * g)) & 15u;

@@ -1087,17 +1087,24 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 for (int S = 2; S <= 8; S++) {
                     if (want_stages_e && S != want_stages_e) continue;
                     if (base + (size_t)S * SB > per_cta) break;
-                    size_t Rb = direct_e ? 0 : (per_cta - base - (size_t)S * SB) / 128 * 128;
-                    if (want_ring_e && !direct_e) Rb = std::min(Rb, want_ring_e);
-                    if (!direct_e && Rb < W) continue;
-                    const size_t smem = base + (size_t)S * SB + Rb;
+                    // compacted-tile rings: shared memory (the remaining bytes) for blocks up to
+                    // a quarter of it, and, when a worst-case block is larger than that, a
+                    // per-CTA slice of an L2-resident buffer for the large blocks (>= 4 of them)
+                    size_t Rs = direct_e ? 0 : (per_cta - base - (size_t)S * SB) / 128 * 128;
+                    if (want_ring_e && !direct_e) Rs = std::min(Rs, want_ring_e);
+                    if (p->o.reserved[6] == 9) Rs = 0;                   // diagnostics: L2 ring only
+                    size_t Rg = 0;
+                    if (!direct_e && W > Rs / 4 && p->o.reserved[6] != 8)
+                        Rg = std::max<size_t>(4 * W, 128 * 1024) / 128 * 128;
+                    if (!direct_e && !Rg && Rs < W) continue;
+                    const size_t smem = base + (size_t)S * SB + Rs;
+                    if (smem > per_cta) continue;
                     if (scan_emit_occupancy(v.nt, v.items, nbr > 1, smem) < occ_t) continue;
-                    // compacted blocks the ring holds while their offsets resolve (>= 2
-                    // worst-case blocks wanted), then input bytes in flight per SM (capped:
-                    // ~64 KB per SM covers the HBM latency), then the larger tile
-                    const double q = direct_e ? 4.0 : (double)Rb / (double)W;
-                    const double inflight = std::min<double>((double)occ_t * S * SB, 160.0 * 1024);
-                    const double sc = (q >= 1.9 ? 1e9 : q * 1e8) + inflight + (double)T * 64 + S;
+                    // input bytes in flight per SM (capped: 128 KB covers the HBM latency;
+                    // more stages only shrink the shared ring), the larger tile, then the
+                    // larger shared ring
+                    const double inflight = std::min<double>((double)occ_t * S * SB, 128.0 * 1024);
+                    const double sc = inflight * 1e3 + (double)T * 64 * 1e3 + (double)std::min<size_t>(Rs, 96 * 1024) + S;
                     if (sc > best) {
                         best = sc;
                         L.items = v.items;
@@ -1106,13 +1113,13 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                         L.stages = S;
                         L.smem = smem;
                         L.ctas = occ_t;
-                        L.out_bytes = (uint32_t)Rb;
+                        L.out_bytes = (uint32_t)Rs;
+                        L.gring_bytes = (uint32_t)Rg;
                     }
                 }
             }
         }
-        if (best < 0)
-            raise(RW_E_UNSUPPORTED, "fused group exceeds the shared-memory budget");
+        if (best >= 0) {
         layout(L.tile);
         for (int b = 0; b < nbr; b++)
             for (int c = b ? P.br_out_end[b - 1] : 0; c < (int)P.br_out_end[b]; c++) {
@@ -1123,6 +1130,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         L.direct = direct_e;
         L.delay = 0;
         return;
+        }
+        // rows too wide for two staged tiles and a ring in shared memory: the
+        // single-stage kernel with its compacted-tile ring in L2 below
     }
     // Scan kernel: S input stages (TMA ring), one scratch tile for computed
     // columns, and a byte ring of R bytes holding compacted tiles until their
@@ -1725,6 +1735,7 @@ void run_group(ExecCtx &X, int gi)
                 p->gring_cap = need;
             }
             TL.gring = p->gring;
+            TL.gring_bytes = L.gring_bytes;
         }
         TL.use_tma = aligned ? 1 : 0;
         TL.epoch = next_epoch(p);
@@ -1757,7 +1768,6 @@ void run_group(ExecCtx &X, int gi)
             TL.n_dev = n_dev;
             if (L.emit) {
                 TL.delay = L.delay;
-                TL.warp_buf = L.warp_buf;
                 cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream), "k_scan_emit");
             } else {
                 cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
@@ -1962,6 +1972,7 @@ void execute_multi(rw_plan *p, const rw_relation_in *in, int nin, const int32_t 
             p->gring_cap = need;
         }
         TL.gring = p->gring;
+        TL.gring_bytes = L.gring_bytes;
     }
     TL.use_tma = aligned ? 1 : 0;
     TL.epoch = next_epoch(p);
@@ -1976,7 +1987,6 @@ void execute_multi(rw_plan *p, const rw_relation_in *in, int nin, const int32_t 
     }
     if (L.emit) {
         TL.delay = L.delay;
-        TL.warp_buf = L.warp_buf;
         cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream), "k_scan_emit<multi>");
     } else {
         cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain<multi>");

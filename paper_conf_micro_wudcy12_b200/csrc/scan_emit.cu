@@ -35,6 +35,7 @@ struct EmitBlk {
     uint64_t aggr, oempty;                // block written (NW arrivals) / block copied out and released
     int64_t tile;
     uint32_t total, roff, used, br;
+    uint32_t where;                       // 0: shared-memory ring, 1: L2 ring
 };
 
 struct EmitCtl {
@@ -42,7 +43,7 @@ struct EmitCtl {
     int64_t tile[kEmitMaxStages];
     EmitBlk blk[kEmitSlots];
     uint32_t cnt[2][kMaxBranch][kEmitMaxCnt];   // double-buffered by tile parity
-    volatile uint32_t tail;                     // ring bytes released by the writers (monotone, wraps)
+    volatile uint32_t tail[2];                  // ring bytes released by the writers (monotone, wraps): smem, L2
 };
 
 static __host__ __device__ inline size_t al128e(size_t x) { return (x + 127) / 128 * 128; }
@@ -53,7 +54,7 @@ size_t emit_ctl_bytes() { return al128e(sizeof(EmitCtl)); }
 // copy `total` elements of one compacted column (16-byte aligned in the ring) to
 // dst[base ..): 16-byte shared loads, element-wide coalesced global stores (the
 // destination offset is arbitrary); rows at or beyond `cap` are dropped
-template <typename T>
+template <typename T, bool GR = false>
 __device__ __forceinline__ void emit_copy(T *dst, const T *src, int64_t base, uint32_t total, int64_t cap, int lane)
 {
     const int64_t lim = cap - base;
@@ -61,11 +62,27 @@ __device__ __forceinline__ void emit_copy(T *dst, const T *src, int64_t base, ui
     T *d = dst + base;
     uint32_t j0 = 0;
     if (sizeof(T) >= 4) {
+        // 16-byte loads, U of them in flight per lane (an L2 ring is ~1 us away)
         constexpr int V = 16 / sizeof(T);
+        constexpr int U = GR ? 8 : 2;
         const uint4 *s4 = (const uint4 *)src;
         const uint32_t nv = m / V;
-        for (uint32_t j = lane; j < nv; j += 32) {
-            const uint4 v = s4[j];
+        uint32_t j = lane;
+        for (; j + (U - 1) * 32 < nv; j += U * 32) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; u++)
+                v[u] = GR ? __ldcg(s4 + j + u * 32) : s4[j + u * 32];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const T *e = (const T *)&v[u];
+#pragma unroll
+                for (int x = 0; x < V; x++)
+                    d[(size_t)(j + u * 32) * V + x] = e[x];
+            }
+        }
+        for (; j < nv; j += 32) {
+            const uint4 v = GR ? __ldcg(s4 + j) : s4[j];
             const T *e = (const T *)&v;
 #pragma unroll
             for (int x = 0; x < V; x++)
@@ -74,9 +91,69 @@ __device__ __forceinline__ void emit_copy(T *dst, const T *src, int64_t base, ui
         j0 = nv * V;
     }
     for (uint32_t j = j0 + lane; j < m; j += 32)
-        d[j] = src[j];
+        d[j] = GR ? __ldcg(src + j) : src[j];
 }
 
+// The survivors (positions sp) of columns [c0, c1) of the staged tile into a compacted
+// block at byte `pos` of a circular ring of R bytes (shared or global: inlined per call
+// site, so each gets plain STS or STG); a column segment that wraps takes the slow path.
+template <int NT, int G>
+__device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1, const char *st, const char *scratch,
+                                              uint32_t m, const uint32_t (&sp)[G][4], uint32_t total, char *ring,
+                                              uint32_t R, uint32_t pos)
+{
+    uint32_t coff = 0;
+    for (int c = c0; c < c1; c++) {
+        const int w = P.out_w[c];
+        const char *src = loc_ptr(P.out_loc[c], st, scratch);
+        const uint32_t so = (pos + coff) % R;
+        coff += al16e(total * w);
+        if (so + total * (uint32_t)w > R) {
+            wrap_scatter<NT, G>(ring, R, so, w, src, m, sp);
+            continue;
+        }
+        char *d = ring + so;
+        if (w == 4) {
+#pragma unroll
+            for (int g = 0; g < G; g++) {
+                const uint32_t m4 = (m >> (4 * g)) & 15u;
+                if (!m4)
+                    continue;
+                const V4<uint32_t> x = ld4<uint32_t>(src, row4<NT>(g));
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    if ((m4 >> q) & 1u) ((uint32_t *)d)[sp[g][q]] = x.v[q];
+            }
+        } else if (w == 8) {
+#pragma unroll
+            for (int g = 0; g < G; g++) {
+                const uint32_t m4 = (m >> (4 * g)) & 15u;
+                if (!m4)
+                    continue;
+                const V4<uint64_t> x = ld4<uint64_t>(src, row4<NT>(g));
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    if ((m4 >> q) & 1u) ((uint64_t *)d)[sp[g][q]] = x.v[q];
+            }
+        } else {
+#pragma unroll
+            for (int g = 0; g < G; g++) {
+                const uint32_t m4 = (m >> (4 * g)) & 15u;
+                if (!m4)
+                    continue;
+                const V4<uint8_t> x = ld4<uint8_t>(src, row4<NT>(g));
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    if ((m4 >> q) & 1u) ((uint8_t *)d)[sp[g][q]] = x.v[q];
+            }
+        }
+    }
+}
+
+// Compacted tiles wait in one of two circular rings: small blocks in shared memory, blocks
+// larger than a quarter of it (high-selectivity chains) in a per-CTA slice of an
+// L2-resident global buffer, so that enough tiles stay in flight for any selectivity.
+// The choice depends only on the block size, so every compute warp makes the same one.
 template <int NT, int ITEMS, bool MULTI>
 __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_constant__ ChainProg P,
                                                                const __grid_constant__ TileLaunch L)
@@ -92,8 +169,10 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
     const uint32_t SB = P.stage_bytes;
     char *stages = (char *)smem_raw + al128e(sizeof(EmitCtl));
     char *scratch = stages + (size_t)S * SB;              // computed columns of the tile being evaluated
-    char *ring = scratch + P.scratch_bytes;
-    const uint32_t R = L.out_bytes;                       // ring bytes (multiple of 128)
+    const uint32_t Rs = L.out_bytes;                      // shared ring bytes (multiple of 128, may be 0)
+    const uint32_t Rg = L.gring ? L.gring_bytes : 0u;     // L2 ring bytes per CTA (0: none)
+    char *ring_s = scratch + P.scratch_bytes;
+    char *ring_g = L.gring ? L.gring + (size_t)blockIdx.x * Rg : nullptr;
     const int NB = MULTI ? P.nbranch : 1;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t n = L.n_ptr ? *L.n_ptr : L.n;
@@ -110,7 +189,8 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
             mbar_init(&ctl->blk[j].aggr, NW);          // one arrival per compute warp
             mbar_init(&ctl->blk[j].oempty, 1);
         }
-        ctl->tail = 0;
+        ctl->tail[0] = 0;
+        ctl->tail[1] = 0;
         fence_mbar_init();
     }
     __syncthreads();
@@ -173,23 +253,52 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                                                                           (L.dbg & 128) ? 0u : (L.dbg & 64) ? 256u : 1024u);
                 if (lane == 0 && t == ntiles - 1)
                     *(b ? L.br_n_dev[b] : L.n_dev) = excl + (int64_t)total;
-                const char *blk = ring + ctl->blk[j].roff;
+                const uint32_t roff = ctl->blk[j].roff;
                 const int64_t cap = b ? P.br_cap[b] : P.out_capacity;
+                const int where = (int)ctl->blk[j].where;
+                const uint32_t R = where ? Rg : Rs;
+                const char *ring = where ? ring_g : ring_s;
                 uint32_t coff = 0;
                 for (int c = b ? P.br_out_end[b - 1] : 0; c < (MULTI ? (int)P.br_out_end[b] : P.nout); c++) {
                     const int w = P.out_w[c];
-                    const char *src = blk + coff;
+                    // the ring is circular: a column's segment may wrap at R (16-byte
+                    // aligned, so no vector straddles the end) -> copied in two pieces
+                    const uint32_t so = (roff + coff) % R;
                     coff += al16e(total * w);
-                    if (w == 4) emit_copy<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, excl, total, cap, lane);
-                    else if (w == 8) emit_copy<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, excl, total, cap, lane);
-                    else emit_copy<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, excl, total, cap, lane);
+                    const uint32_t n1 = min(total, (R - so) / (uint32_t)w);
+                    for (int piece = 0; piece < 2; piece++) {
+                        const char *src = piece ? ring : ring + so;
+                        const int64_t at = piece ? excl + n1 : excl;
+                        const uint32_t cnt = piece ? total - n1 : n1;
+                        if (cnt == 0) continue;
+                        if (where) {
+                            if (w == 4) emit_copy<uint32_t, true>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, at, cnt, cap, lane);
+                            else if (w == 8) emit_copy<uint64_t, true>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, at, cnt, cap, lane);
+                            else emit_copy<uint8_t, true>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, at, cnt, cap, lane);
+                        } else {
+                            if (w == 4) emit_copy<uint32_t>((uint32_t *)P.out_ptr[c], (const uint32_t *)src, at, cnt, cap, lane);
+                            else if (w == 8) emit_copy<uint64_t>((uint64_t *)P.out_ptr[c], (const uint64_t *)src, at, cnt, cap, lane);
+                            else emit_copy<uint8_t>((uint8_t *)P.out_ptr[c], (const uint8_t *)src, at, cnt, cap, lane);
+                        }
+                    }
                 }
                 __syncwarp();
+                if (where) {
+                    // the block is copied out: drop its fully covered L2 lines, so the ring
+                    // never costs a DRAM write-back
+                    const uint32_t used_b = ctl->blk[j].used;
+                    for (uint32_t o = ((roff + 127u) & ~127u) + (uint32_t)lane * 128u; o + 128u <= roff + used_b; o += 32u * 128u)
+                        if (o + 128u <= R) discard_l2_line(ring_g + o);
+                    __syncwarp();
+                }
                 if (lane == 0) {
                     if (i > 0)   // ring bytes are released in block order
                         mbar_wait(&ctl->blk[(i - 1) % kEmitSlots].oempty, ((i - 1) / kEmitSlots) & 1u);
-                    __threadfence_block();
-                    ctl->tail = ctl->tail + ctl->blk[j].used;
+                    if (where)
+                        __threadfence();   // the discards land before the bytes are rewritten
+                    else
+                        __threadfence_block();
+                    ctl->tail[where] = ctl->tail[where] + ctl->blk[j].used;
                     mbar_arrive(&ctl->blk[j].oempty);
                 }
                 __syncwarp();
@@ -197,7 +306,7 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
         }
     } else {
         // ---------------- compute warps ----------------
-        uint32_t head = 0, hpos = 0;                    // ring reservation, replicated in every warp
+        uint32_t head_s = 0, hpos_s = 0, head_g = 0, hpos_g = 0;   // ring reservations, replicated in every warp
         uint32_t ublk = 0;                              // compacted blocks emitted (tiles x branches)
         int s = -1;
         uint32_t fph = 1;
@@ -329,31 +438,27 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 const int c0 = b ? P.br_out_end[b - 1] : 0, c1 = MULTI ? (int)P.br_out_end[b] : P.nout;
                 const uint32_t need = P.br_nw[b][0] * al16e(total) + P.br_nw[b][1] * al16e(total * 4u) +
                                       P.br_nw[b][2] * al16e(total * 8u);
-                uint32_t pos = hpos, used = need;
-                bool drain = false;
-                if (pos + need > R) {                   // skip the tail [pos, R)
-                    used += R - pos;
-                    pos = 0;
-                    if (used > R) {                     // cannot fit behind live blocks: wait for an empty ring
-                        used = need;
-                        drain = true;
-                    }
-                }
+                // circular rings: the block goes to the shared ring unless it is larger than a
+                // quarter of it (then to the L2 ring); wait until its bytes are free
+                const int where = Rg != 0u && (Rs == 0u || need > Rs / 4u) ? 1 : 0;
+                const uint32_t R = where ? Rg : Rs;
+                const uint32_t pos = where ? hpos_g : hpos_s, used = need;
+                const uint32_t hd = where ? head_g : head_s;
                 const int j = (int)(ublk % kEmitSlots);
                 if (ublk >= kEmitSlots)
                     mbar_wait(&ctl->blk[j].oempty, ((ublk / kEmitSlots) - 1) & 1u);
                 {
                     uint32_t backoff = 64;
-                    while (drain ? (head != ctl->tail) : (head + used - ctl->tail > R)) {
+                    while (hd + used - (where ? ctl->tail[1] : ctl->tail[0]) > R) {
                         __nanosleep(backoff);
                         backoff = backoff < 1024 ? backoff * 2 : 1024;
                     }
                 }
-                head += used;
-                hpos = pos + need == R ? 0 : pos + need;
+                const uint32_t np = pos + need >= R ? pos + need - R : pos + need;
+                if (where) { head_g = hd + used; hpos_g = np; }
+                else { head_s = hd + used; hpos_s = np; }
                 // compact the survivors into the block, tile order: each surviving row's
                 // position is computed once, then every column stores with it
-                char *blk = ring + pos;
                 uint32_t sp[G][4];
 #pragma unroll
                 for (int g = 0; g < G; g++) {
@@ -364,55 +469,21 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                         p += (m >> (4 * g + q)) & 1u;
                     }
                 }
-                uint32_t coff = 0;
-                for (int c = c0; c < c1; c++) {
-                    const int w = P.out_w[c];
-                    const char *src = loc_ptr(P.out_loc[c], st, scratch);
-                    char *d = blk + coff;
-                    coff += al16e(total * w);
-                    if (w == 4) {
-#pragma unroll
-                        for (int g = 0; g < G; g++) {
-                            const uint32_t m4 = (m >> (4 * g)) & 15u;
-                            if (!m4)
-                                continue;
-                            const V4<uint32_t> x = ld4<uint32_t>(src, row4<NT>(g));
-#pragma unroll
-                            for (int q = 0; q < 4; q++)
-                                if ((m4 >> q) & 1u) ((uint32_t *)d)[sp[g][q]] = x.v[q];
-                        }
-                    } else if (w == 8) {
-#pragma unroll
-                        for (int g = 0; g < G; g++) {
-                            const uint32_t m4 = (m >> (4 * g)) & 15u;
-                            if (!m4)
-                                continue;
-                            const V4<uint64_t> x = ld4<uint64_t>(src, row4<NT>(g));
-#pragma unroll
-                            for (int q = 0; q < 4; q++)
-                                if ((m4 >> q) & 1u) ((uint64_t *)d)[sp[g][q]] = x.v[q];
-                        }
-                    } else {
-#pragma unroll
-                        for (int g = 0; g < G; g++) {
-                            const uint32_t m4 = (m >> (4 * g)) & 15u;
-                            if (!m4)
-                                continue;
-                            const V4<uint8_t> x = ld4<uint8_t>(src, row4<NT>(g));
-#pragma unroll
-                            for (int q = 0; q < 4; q++)
-                                if ((m4 >> q) & 1u) ((uint8_t *)d)[sp[g][q]] = x.v[q];
-                        }
-                    }
-                }
+                if (where)
+                    compact_block<NT, G>(P, c0, c1, st, scratch, m, sp, total, ring_g, R, pos);
+                else
+                    compact_block<NT, G>(P, c0, c1, st, scratch, m, sp, total, ring_s, R, pos);
                 __syncwarp();
                 if (lane == 0) {
+                    if (where)
+                        __threadfence_block();
                     if (warp == 0) {
                         ctl->blk[j].tile = t;
                         ctl->blk[j].total = total;
                         ctl->blk[j].roff = pos;
                         ctl->blk[j].used = used;
                         ctl->blk[j].br = (uint32_t)b;
+                        ctl->blk[j].where = (uint32_t)where;
                     }
                     if (b == NB - 1)
                         mbar_arrive(&ctl->empty[s]);      // this warp is done with the stage
