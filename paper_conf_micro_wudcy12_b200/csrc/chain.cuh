@@ -649,8 +649,9 @@ __device__ inline void reg_agg_reduce_warp(const ChainProg &P, RegAgg &R, unsign
 // no per-row type dispatch); the one-hot over the groups becomes a jump to the
 // row's group, whose partials take predicated-free adds.
 // Narrow sums (a < NN) accumulate in 32-bit partials whose flush period comes from the
-// caller-declared bounds; their values are OR-ed into `orv` so that a value outside
-// [0, 2^narrow_bits) is reported (err[2]) instead of silently wrapping a partial.
+// caller-declared bounds; the values of the aggregated rows are OR-ed into `orv`, so that
+// a value outside [0, 2^narrow_bits) is reported (err[2]) instead of silently wrapping a
+// partial.
 template <int NT, int ITEMS, int NAGG, bool W64, int NN = 0, bool R4 = false>
 __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *at, const uint32_t *g, uint32_t ok,
                                              RegAgg &R, uint64_t &orv)
@@ -666,7 +667,7 @@ __device__ __forceinline__ void agg_rows_reg(const char *const *ab, const int *a
             v[a] = a < NAGG ? (W64 ? ((const uint64_t *)ab[a])[r] : ld_ext(ab[a], at[a], r)) : 0ull;
 #pragma unroll
         for (int a = 0; a < NN; a++)
-            if ((ok >> k) & 1u)
+            if ((ok >> k) & 1u)   // aggregated rows only (a ragged tile's tail holds stale data)
                 orv |= v[a];
 #pragma unroll
         for (int d = 0; d < kRegD; d++) {

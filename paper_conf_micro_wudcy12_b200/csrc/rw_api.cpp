@@ -1050,7 +1050,17 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         }
         return;
     }
-    if (!L.agg && p->o.reserved[6] != 3) {
+    // Kernel choice for compacting chains: the emitting kernel (4-row vectors, shared +
+    // L2 rings) when the chain filters at least twice (expected survival <= 1/4 under the
+    // 50%-per-atom reading, small compacted tiles) or not at all (rows stored in place);
+    // the L2-ring kernel below for single-atom filters (large compacted tiles) and for
+    // input-dependence branches, where it measured faster.
+    int npred_ops = 0;
+    for (const HOp &h : ops)
+        if (h.kind == K_PRED) npred_ops++;
+    const bool use_emit = p->o.reserved[6] == 10 ||
+                          (p->o.reserved[6] != 3 && nbr == 1 && (npred_ops == 0 || npred_ops >= 2));
+    if (!L.agg && use_emit) {
         // Emitting scan kernel (scan_emit.cu): S input stages, each with its own scratch
         // for computed columns (a stage holds its tile until the tile's offset resolves),
         // per-thread hold words, and one compaction buffer per compute warp (resource

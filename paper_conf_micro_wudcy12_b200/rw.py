@@ -177,7 +177,12 @@ class Plan:
         o.reserved[3] = ctypes.c_int32((dbg_ts >> 32) & 0xffffffff).value
         o.reserved[5] = items              # tuning: rows per thread of the scan tile (0 = auto)
         o.reserved[4] = variant            # tuning: 2 = 512x4, 3 = 512x8 compute threads x rows
-        o.reserved[6] = gring              # tuning: 1 = compacted-tile ring in global memory (L2)
+        # kernel / fusion switches (diagnostics and A/B measurements): 2 = L2-ring scan kernel
+        # with its ring in shared memory, 3 = L2-ring scan kernel for every compacting chain,
+        # 5 = no JOIN -> JOIN fusion, 6 = cp.async join gathers, 7 = no SELECT / PROJECT
+        # fusion upstream of a JOIN, 8 / 9 = emitting kernel with only its shared / only its
+        # L2 ring, 10 = emitting kernel for every compacting chain
+        o.reserved[6] = gring
         o.reserved[7] = agg_mode           # 1 = force the thread-private-partials aggregate terminal
         self.device = device
         h = ctypes.c_void_p()

@@ -1,5 +1,5 @@
 #!/bin/bash
-O=gpurun_out/r02ae; mkdir -p $O
+O=gpurun_out/r02ai2; mkdir -p $O
 for c in "--config c2" "--config c1" "--config c1 --rows 1073741824" "--config cd" "--config c3"; do for a in "" "--gring 9" "--gring 8"; do
   echo "== $c $a" >> $O/sweep.log
   timeout 300 python bench.py $c $a --no-cpu --no-e2e --no-sweep --steps 10 2>&1 | python -c "import json,sys
