@@ -22,6 +22,25 @@ DEV = "cuda:0"
 CH = 1 << 22
 
 
+def _comp(cols):
+    """(u32 key, u32 val) rows as one int64 whose order within a key is the val order."""
+    import torch
+    return ((cols[0].to(torch.int64) & 0xFFFFFFFF) << 32) | (cols[1].to(torch.int64) & 0xFFFFFFFF)
+
+
+def _greater_counts(Lc, Rc):
+    """For every row (k, v) of L: the rows (k, w) of R with w > v (u32 compare)."""
+    import torch
+    lc, rc = _comp(Lc), torch.sort(_comp(Rc)).values   # relations are sorted on the key only
+    pos = torch.searchsorted(rc, lc, right=True)
+    end = torch.searchsorted(rc, (lc & ~0xFFFFFFFF) | 0xFFFFFFFF, right=True)
+    return end - pos
+
+
+def _pairs_greater(Lc, Rc) -> int:
+    return int(_greater_counts(Lc, Rc).sum().item())
+
+
 def _host(cols, types, a, b):
     return oracle.Relation(types, [c[a:b].cpu().numpy().view(NPT[t]) for c, t in zip(cols, types)])
 
@@ -95,6 +114,9 @@ def test_c3_full_size_cardinality_and_key_ranges():
     common_r = torch.isin(kv, ku)
     total = int((cl[common_l] * cr[common_r]).sum().item())
     assert total > 0 and m <= total
+    # exact output count: for every L row (k, lval) the R rows of key k with rval > lval,
+    # by binary search in R's (key, val) order (torch.searchsorted, independent of librw)
+    assert m == _pairs_greater(ins["L"], ins["R"])
     okey = outs[0][:m].to(torch.int64) & 0xFFFFFFFF
     assert bool((okey[1:] >= okey[:-1]).all())
     hot = int(ku[torch.argmax(cl * common_l)].item())
@@ -168,3 +190,66 @@ def test_setop_full_size_key_ranges():
             oa, ob = int(torch.searchsorted(key, lo)), int(torch.searchsorted(key, hi))
             got = oracle.Relation(ref.types, [o[oa:ob].cpu().numpy().view(np.uint32) for o in outs])
             assert_same(got, ref)
+
+
+def test_c5_full_size_count_and_key_ranges():
+    """C5 (3 x 2^27 rows per GPU, JOIN -> JOIN -> SELECT(a < c)) in the bench launch
+    configuration (the fused 3-input group): the exact output count
+    sum over R rows (k, a) of m_S(k) * #{T rows (k, c): c > a} by binary searches, and
+    three key ranges compared element by element with the oracle on the sub-relations."""
+    import torch
+    n = 1 << 27
+    spec = workloads.c5_spec()
+    ins = workloads.c5_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    assert "3 inputs" in plan.explain(ids["s"])
+    cap = 3 * n
+    outs = [torch.empty(cap, dtype=torch.int32, device=DEV) for _ in range(4)]
+    m = plan.execute([(n, ins["R"]), (n, ins["S"]), (n, ins["T"])], ids["s"], outs, cap)
+    R, S, T = ins["R"], ins["S"], ins["T"]
+    rk = R[0].to(torch.int64) & 0xFFFFFFFF
+    sk = S[0].to(torch.int64) & 0xFFFFFFFF
+    ms = torch.searchsorted(sk, rk, right=True) - torch.searchsorted(sk, rk)
+    expect = int((ms * _greater_counts(R, T)).sum().item())
+    assert m == expect and m > 0.1 * n
+    okey = outs[0][:m].to(torch.int64) & 0xFFFFFFFF
+    assert bool((okey[1:] >= okey[:-1]).all())
+    tk = T[0].to(torch.int64) & 0xFFFFFFFF
+    for lo, hi in [(0, 1 << 14), (n // 2, n // 2 + (1 << 14)), (n - (1 << 14), n)]:
+        sub = {}
+        for name, keys in (("R", rk), ("S", sk), ("T", tk)):
+            a, b = int(torch.searchsorted(keys, lo)), int(torch.searchsorted(keys, hi))
+            sub[name] = [c[a:b] for c in ins[name]]
+        ref = run_oracle(spec, sub)
+        a = int(torch.searchsorted(okey, torch.tensor([lo], device=DEV)).item())
+        b = int(torch.searchsorted(okey, torch.tensor([hi], device=DEV)).item())
+        assert b - a == ref.n
+        got = oracle.Relation(ref.types, [o[a:b].cpu().numpy().view(np.uint32) for o in outs])
+        assert_same(got, ref)
+
+
+def test_host_streamed_full_size_equals_device_path():
+    """rw_plan_execute_host on C2's 2^29 x 4 i32 from pinned host memory with the default
+    2^25-row chunks (the e2e bench path): identical, row order included, to the device
+    execute (itself chunk-checked against the oracle above), and its first and last
+    streamed chunk's survivors equal the oracle on those rows."""
+    import torch
+    n = workloads.C2_ROWS
+    spec = workloads.c2_spec()
+    ins = workloads.c2_inputs(n, device=DEV)
+    plan, ids = build_gpu_plan(spec)
+    dev_out = [torch.empty(n // 2, dtype=torch.int32, device=DEV) for _ in range(3)]
+    m = plan.execute([(n, ins["R"])], ids["s2"], dev_out, n // 2)
+    host_in = [c.cpu().pin_memory() for c in ins["R"]]
+    host_out = [torch.empty(n // 2, dtype=torch.int32).pin_memory() for _ in range(3)]
+    mh = plan.execute_host([(n, host_in)], ids["s2"], host_out, n // 2)
+    assert mh == m
+    for h, d in zip(host_out, dev_out):
+        assert torch.equal(h[:m], d[:m].cpu())
+    C = 1 << 25
+    keep = (ins["R"][1] < workloads.thr_i32(0.5)) & (ins["R"][3] < workloads.thr_i32(0.5))
+    for a in (0, n - C):
+        ref = run_oracle(spec, {"R": [c[a:a + C] for c in ins["R"]]})
+        off = int(keep[:a].sum().item())
+        got = oracle.Relation(ref.types, [o[off:off + ref.n].numpy().view(np.int32) for o in host_out])
+        assert_same(got, ref)
