@@ -245,10 +245,28 @@ rw_status rw_split_by_splitters(const void *keys_dev, int64_t n, int32_t key_typ
  * lie concatenated in `cols` (run r = rows [run_off[r], run_off[r+1]) of every column;
  * run_off is a HOST array of nrun+1 entries) into one sequence sorted the same way,
  * written to out_cols (device, run_off[nrun] - run_off[0] rows).  Equal tuples keep run
- * order.  Pairwise merge-path tree (ceil(log2 nrun) passes); temporaries come from
- * cudaMallocAsync on the given stream. */
+ * order.  This is the merge after the key-range all-to-all (§4.3.2
+ * merge-path partitioning generalised to P inputs).  Tuples of <= 8 bytes with 2 <=
+ * nrun <= 32: one pass (read once, write once; merge_p.cu), each run < 2^32 rows, else
+ * RW_E_UNSUPPORTED.  Wider tuples or more runs: pairwise merge-path tree
+ * (ceil(log2 nrun) passes).  Temporaries come from cudaMallocAsync on the stream. */
 rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t ncols, const int64_t *run_off,
                         int32_t nrun, void *const *out_cols, void *cuda_stream);
+
+/* Order-preserving u64 image of each of n tuples whose columns total <= 8 bytes
+ * (columns concatenated, first column most significant, signed types with the sign bit
+ * flipped), so that u64 order = lexicographic tuple order in the declared types; written
+ * to packed_dev[0..n).  The exchange sends these images in ONE all-to-all instead of one
+ * per column.  Tuples wider than 8 bytes: RW_E_UNSUPPORTED. */
+rw_status rw_pack_tuples(const void *const *cols, const int32_t *types, int32_t ncols, int64_t n,
+                         uint64_t *packed_dev, void *cuda_stream);
+
+/* rw_merge_runs over runs of packed images (rw_pack_tuples layout): run r = entries
+ * [run_off[r], run_off[r+1]) of packed_dev (run_off on the HOST, nrun <= 32, each run
+ * < 2^32 rows); the merged tuples are unpacked into the ncols device columns out_cols
+ * (run_off[nrun] - run_off[0] rows).  One read and one write pass. */
+rw_status rw_merge_packed_runs(const uint64_t *packed_dev, const int32_t *types, int32_t ncols,
+                               const int64_t *run_off, int32_t nrun, void *const *out_cols, void *cuda_stream);
 
 /* Aggregate combine across row shards: an aggregate result is
  * exported as D * L dense int64 words (per group: a presence word, then per aggregate

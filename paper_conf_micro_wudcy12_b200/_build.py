@@ -5,7 +5,7 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librw.so")
-SOURCES = ["kernels.cu", "scan_emit.cu", "join2.cu", "setops.cu", "rw_api.cpp", "dist_kernels.cu"]
+SOURCES = ["kernels.cu", "scan_emit.cu", "join2.cu", "setops.cu", "rw_api.cpp", "dist_kernels.cu", "merge_p.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "-Xptxas", "-v"]

@@ -37,6 +37,35 @@ struct OutPtrs {
     void *col[kMaxOut];
 };
 
+// Single-pass P-way merge (merge_p.cu).  Runs lie at rows [run_off[q], run_off[q+1])
+// of every column (or of `packed`, u64 order-preserving tuple images); T = sample
+// spacing, G = samples per merge group, S = samples, NG = groups.
+constexpr int kMpThreads = 256;
+constexpr int kMpItems = 16;
+constexpr int kMpC = kMpThreads * kMpItems;   // elements one merge group may hold
+constexpr int kMpMaxRuns = 32;
+
+struct MpLaunch {
+    const void *col[kMaxMergeCols];
+    uint8_t types[kMaxMergeCols];
+    int32_t ncols;
+    const uint64_t *packed;              // packed u64 input (else nullptr: read col[])
+    int32_t nrun;
+    int32_t T;
+    int32_t G;
+    int64_t run_off[kMpMaxRuns + 1];
+    int64_t samp_base[kMpMaxRuns + 1];
+    int64_t S;
+    int64_t NG;
+    uint64_t *sv;                        // S sample images
+    uint32_t *cuts;                      // S x nrun
+    int64_t *bound;                      // NG group-start samples
+    void *out[kMaxMergeCols];
+};
+
+cudaError_t mp_merge_launch(const MpLaunch &M, int sms, cudaStream_t s);
+cudaError_t mp_pack_launch(const MpLaunch &M, int64_t n, uint64_t *dst, int sms, cudaStream_t s);
+
 cudaError_t split_bounds_launch(const void *keys, int64_t n, int key_type, const void *spl, int nsplit,
                                 int64_t *bounds, cudaStream_t s);
 cudaError_t merge2_launch(const MergeCols &A, int64_t na, const MergeCols &B, int64_t nb, const MergeOut &O,

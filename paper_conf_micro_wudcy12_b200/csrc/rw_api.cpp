@@ -2775,6 +2775,69 @@ rw_status rw_split_by_splitters(const void *keys_dev, int64_t n, int32_t key_typ
     RW_CATCH
 }
 
+// Single-pass P-way merge (merge_p.cu) of runs whose tuples pack into <= 8 bytes.
+// `packed` (u64 tuple images) or `cols` is the input; temporaries from cudaMallocAsync.
+static void merge_runs_single_pass(const void *const *cols, const uint64_t *packed, const int32_t *types,
+                                   int32_t ncols, const int64_t *run_off, int32_t nrun, void *const *out_cols,
+                                   cudaStream_t st)
+{
+    MpLaunch M{};
+    for (int c = 0; c < ncols; c++) {
+        M.col[c] = cols ? cols[c] : nullptr;
+        M.types[c] = (uint8_t)types[c];
+        M.out[c] = out_cols[c];
+    }
+    M.ncols = ncols;
+    M.packed = packed;
+    M.nrun = nrun;
+    M.G = nrun;
+    M.T = std::max(1, kMpC / (M.G + nrun));   // a group holds <= (G + P) * T <= kMpC elements
+    M.samp_base[0] = 0;
+    for (int q = 0; q <= nrun; q++) {
+        M.run_off[q] = run_off[q];
+        if (q < nrun) {
+            const int64_t nq = run_off[q + 1] - run_off[q];
+            if (nq >= (int64_t)UINT32_MAX)
+                raise(RW_E_UNSUPPORTED, "merge run of 2^32 rows or more");
+            M.samp_base[q + 1] = M.samp_base[q] + (nq + M.T - 1) / M.T;
+        }
+    }
+    M.S = M.samp_base[nrun];
+    M.NG = (M.S + M.G - 1) / M.G;
+    if (M.S == 0)
+        return;
+    int dev = 0, sms = 148;
+    cuda_check(cudaGetDevice(&dev), "cudaGetDevice");
+    cuda_check(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev), "attr");
+    void *sv = nullptr, *cuts = nullptr, *bound = nullptr;
+    cuda_check(cudaMallocAsync(&sv, (size_t)M.S * 8, st), "cudaMallocAsync");
+    cudaError_t e1 = cudaMallocAsync(&cuts, (size_t)M.S * nrun * 4, st);
+    cudaError_t e2 = cudaMallocAsync(&bound, (size_t)M.NG * 8, st);
+    cudaError_t e3 = cudaSuccess;
+    if (e1 == cudaSuccess && e2 == cudaSuccess) {
+        M.sv = (uint64_t *)sv;
+        M.cuts = (uint32_t *)cuts;
+        M.bound = (int64_t *)bound;
+        e3 = mp_merge_launch(M, sms, st);
+    }
+    cudaFreeAsync(sv, st);
+    if (cuts)
+        cudaFreeAsync(cuts, st);
+    if (bound)
+        cudaFreeAsync(bound, st);
+    cuda_check(e1, "cudaMallocAsync");
+    cuda_check(e2, "cudaMallocAsync");
+    cuda_check(e3, "k_mp_merge");
+}
+
+static bool packable(const int32_t *types, int32_t ncols)
+{
+    int bytes = 0;
+    for (int c = 0; c < ncols; c++)
+        bytes += type_width(types[c]);
+    return bytes <= 8;
+}
+
 rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t ncols, const int64_t *run_off,
                         int32_t nrun, void *const *out_cols, void *cuda_stream)
 {
@@ -2787,6 +2850,20 @@ rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t n
         check_type(types[c]);
         T.t[c] = (uint8_t)types[c];
     }
+    for (int r = 0; r < nrun; r++)
+        if (run_off[r + 1] < run_off[r])
+            raise(RW_E_ARG, "run offsets must be non-decreasing");
+    if (nrun >= 2 && nrun <= kMpMaxRuns && packable(types, ncols)) {
+        // one read and one write of the data (merge_p.cu)
+        std::vector<int64_t> off(run_off, run_off + nrun + 1);
+        for (auto &o : off)
+            o -= run_off[0];
+        std::vector<const void *> base(ncols);
+        for (int c = 0; c < ncols; c++)
+            base[c] = (const char *)cols[c] + (size_t)run_off[0] * type_width(types[c]);
+        merge_runs_single_pass(base.data(), nullptr, types, ncols, off.data(), nrun, out_cols, st);
+        return RW_OK;
+    }
     struct Run {
         MergeCols c;
         int64_t n;
@@ -2794,8 +2871,6 @@ rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t n
     };
     std::vector<Run> runs;
     for (int r = 0; r < nrun; r++) {
-        if (run_off[r + 1] < run_off[r])
-            raise(RW_E_ARG, "run offsets must be non-decreasing");
         Run x{};
         x.n = run_off[r + 1] - run_off[r];
         for (int c = 0; c < ncols; c++)
@@ -2815,7 +2890,8 @@ rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t n
                                            cudaMemcpyDeviceToDevice, st),
                            "copy run");
         }
-        // pairwise merge tree; the last round writes the caller's columns
+        // wide tuples / more than kMpMaxRuns runs: pairwise merge tree; the last round
+        // writes the caller's columns
         while (runs.size() > 1) {
             std::vector<Run> next;
             const bool last = runs.size() == 2;
@@ -2848,6 +2924,57 @@ rw_status rw_merge_runs(const void *const *cols, const int32_t *types, int32_t n
         throw;
     }
     release();
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_pack_tuples(const void *const *cols, const int32_t *types, int32_t ncols, int64_t n,
+                         uint64_t *packed_dev, void *cuda_stream)
+{
+    RW_TRY
+    if (ncols < 1 || ncols > kMaxMergeCols || n < 0 || !cols || !types || (n > 0 && !packed_dev))
+        raise(RW_E_ARG, "bad pack arguments");
+    for (int c = 0; c < ncols; c++)
+        check_type(types[c]);
+    if (!packable(types, ncols))
+        raise(RW_E_UNSUPPORTED, "tuple wider than 8 bytes");
+    MpLaunch M{};
+    for (int c = 0; c < ncols; c++) {
+        M.col[c] = cols[c];
+        M.types[c] = (uint8_t)types[c];
+    }
+    M.ncols = ncols;
+    int dev = 0, sms = 148;
+    cuda_check(cudaGetDevice(&dev), "cudaGetDevice");
+    cuda_check(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev), "attr");
+    cuda_check(mp_pack_launch(M, n, packed_dev, sms, (cudaStream_t)cuda_stream), "k_mp_pack");
+    return RW_OK;
+    RW_CATCH
+}
+
+rw_status rw_merge_packed_runs(const uint64_t *packed_dev, const int32_t *types, int32_t ncols,
+                               const int64_t *run_off, int32_t nrun, void *const *out_cols, void *cuda_stream)
+{
+    RW_TRY
+    if (ncols < 1 || ncols > kMaxMergeCols || nrun < 0 || nrun > kMpMaxRuns || !types || !run_off || !out_cols)
+        raise(RW_E_ARG, "bad merge arguments");
+    for (int c = 0; c < ncols; c++)
+        check_type(types[c]);
+    if (!packable(types, ncols))
+        raise(RW_E_UNSUPPORTED, "tuple wider than 8 bytes");
+    for (int r = 0; r < nrun; r++)
+        if (run_off[r + 1] < run_off[r])
+            raise(RW_E_ARG, "run offsets must be non-decreasing");
+    if (nrun == 0 || run_off[nrun] == run_off[0])
+        return RW_OK;
+    if (!packed_dev)
+        raise(RW_E_ARG, "bad merge arguments");
+    // nrun == 1 is a merge of one run: the same kernels unpack it
+    std::vector<int64_t> off(run_off, run_off + nrun + 1);
+    for (auto &o : off)
+        o -= run_off[0];
+    merge_runs_single_pass(nullptr, packed_dev + run_off[0], types, ncols, off.data(), nrun, out_cols,
+                           (cudaStream_t)cuda_stream);
     return RW_OK;
     RW_CATCH
 }

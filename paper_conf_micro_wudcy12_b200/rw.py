@@ -64,6 +64,7 @@ EXPORTS = ["rw_plan_create", "rw_plan_destroy", "rw_plan_add_input", "rw_plan_ad
            "rw_plan_add_project", "rw_plan_add_join", "rw_plan_add_setop", "rw_plan_add_agg", "rw_plan_node_schema",
            "rw_plan_execute", "rw_plan_execute_multi", "rw_plan_execute_host", "rw_plan_explain", "rw_plan_last_launches",
            "rw_status_str", "rw_last_error", "rw_split_by_splitters", "rw_merge_runs",
+           "rw_pack_tuples", "rw_merge_packed_runs",
            "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]
 
 _lib = None
@@ -100,13 +101,15 @@ def lib():
     L.rw_last_error.restype = ctypes.c_char_p
     L.rw_split_by_splitters.argtypes = [vp, i64, i32, vp, i32, vp, vp]
     L.rw_merge_runs.argtypes = [P(vp), P(i32), i32, P(i64), i32, P(vp), vp]
+    L.rw_pack_tuples.argtypes = [P(vp), P(i32), i32, i64, vp, vp]
+    L.rw_merge_packed_runs.argtypes = [vp, P(i32), i32, P(i64), i32, P(vp), vp]
     L.rw_plan_agg_limbs.argtypes = [vp, i32, P(i64)]
     L.rw_plan_agg_export.argtypes = [vp, i32, P(vp), vp, i64, vp]
     L.rw_plan_agg_import.argtypes = [vp, i32, vp, P(rw_relation_out)]
     for f in ["rw_plan_create", "rw_plan_add_input", "rw_plan_add_select", "rw_plan_add_project",
               "rw_plan_add_join", "rw_plan_add_setop", "rw_plan_add_agg", "rw_plan_node_schema", "rw_plan_execute",
               "rw_plan_execute_host", "rw_plan_execute_multi", "rw_plan_explain", "rw_split_by_splitters", "rw_merge_runs",
-              "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]:
+              "rw_pack_tuples", "rw_merge_packed_runs", "rw_plan_agg_limbs", "rw_plan_agg_export", "rw_plan_agg_import"]:
         getattr(L, f).restype = i32
     _lib = L
     return L
@@ -370,3 +373,17 @@ def merge_runs(cols, types, run_off, out_cols, stream) -> None:
     ro = (ctypes.c_int64 * len(run_off))(*[int(x) for x in run_off])
     o = (ctypes.c_void_p * len(out_cols))(*[_ptr(x) for x in out_cols])
     check(lib().rw_merge_runs(c, t, len(cols), ro, len(run_off) - 1, o, ctypes.c_void_p(stream.cuda_stream)))
+
+
+def pack_tuples(cols, types, n: int, packed, stream) -> None:
+    c = (ctypes.c_void_p * len(cols))(*[_ptr(x) for x in cols])
+    t = _i32arr([TYPES[x] for x in types])
+    check(lib().rw_pack_tuples(c, t, len(cols), n, ctypes.c_void_p(_ptr(packed)), ctypes.c_void_p(stream.cuda_stream)))
+
+
+def merge_packed_runs(packed, types, run_off, out_cols, stream) -> None:
+    t = _i32arr([TYPES[x] for x in types])
+    ro = (ctypes.c_int64 * len(run_off))(*[int(x) for x in run_off])
+    o = (ctypes.c_void_p * len(out_cols))(*[_ptr(x) for x in out_cols])
+    check(lib().rw_merge_packed_runs(ctypes.c_void_p(_ptr(packed)), t, len(types), ro, len(run_off) - 1, o,
+                                     ctypes.c_void_p(stream.cuda_stream)))

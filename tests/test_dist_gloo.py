@@ -27,7 +27,42 @@ def _np_backend():
     class NumpyBackend(rd.Backend):
         def split(self, keys, key_type, splitters):
             kv = rd.key_values(keys, key_type).numpy()
-            return [int(x) for x in np.searchsorted(kv, np.asarray(splitters, dtype=np.int64), side="left")]
+            return torch.from_numpy(np.searchsorted(kv, splitters.numpy(), side="left").astype(np.int64))
+
+        def pack(self, cols, types):
+            # order-preserving u64 image: columns concatenated, first most significant,
+            # signed types with the sign bit flipped (python ints, then int64 storage)
+            n = int(cols[0].numel())
+            img = [0] * n
+            for c, t in zip(cols, types):
+                w = rd.WIDTH[t] * 8
+                vals = c.numpy().astype(np.int64).tolist()
+                for i, v in enumerate(vals):
+                    u = v & ((1 << w) - 1)
+                    if t in ("i32", "i64"):
+                        u ^= 1 << (w - 1)
+                    img[i] = (img[i] << w) | u if w < 64 else u
+            return torch.tensor([x - (1 << 64) if x >= 1 << 63 else x for x in img], dtype=torch.int64)
+
+        def merge_packed(self, packed, types, run_off):
+            u = packed.numpy().view(np.uint64)
+            order = np.argsort(u, kind="stable")
+            srt = [int(x) for x in u[order]]
+            cols = []
+            shift = sum(rd.WIDTH[t] * 8 for t in types)
+            for t in types:
+                w = rd.WIDTH[t] * 8
+                shift -= w
+                vals = []
+                for x in srt:
+                    f = (x >> shift) & ((1 << w) - 1)
+                    if t in ("i32", "i64"):
+                        f ^= 1 << (w - 1)
+                    if f >= 1 << (w - 1) and t != "u8":
+                        f -= 1 << w
+                    vals.append(f)
+                cols.append(torch.tensor(vals, dtype=rd.STORAGE[t]))
+            return cols
 
         def merge(self, cols, types, run_off):
             # stable lexicographic sort over all columns (library sort; run order kept)

@@ -19,7 +19,7 @@ def simulated_exchange(backend, shards, types, splitters):
     pieces = [[None] * P for _ in range(P)]          # pieces[src][dst] = list of column slices
     for src, cols in enumerate(shards):
         n = int(cols[0].numel())
-        b = backend.split(cols[0], types[0], splitters)
+        b = backend.split(cols[0], types[0], torch.tensor(splitters, dtype=torch.int64, device=DEV)).tolist()
         cuts = [0] + b + [n]
         for dst in range(P):
             pieces[src][dst] = [c[cuts[dst]:cuts[dst + 1]] for c in cols]
@@ -105,7 +105,8 @@ def test_split_bounds_and_merge_small():
     from paper_conf_micro_wudcy12_b200 import dist as rd
     backend = rd.GpuBackend(0)
     keys = torch.tensor([1, 1, 3, 5, 5, 5, 9], dtype=torch.int32, device=DEV)
-    assert backend.split(keys, "i32", [0, 1, 2, 5, 6, 10]) == [0, 0, 2, 3, 6, 7]
+    spl = torch.tensor([0, 1, 2, 5, 6, 10], dtype=torch.int64, device=DEV)
+    assert backend.split(keys, "i32", spl).tolist() == [0, 0, 2, 3, 6, 7]
     a = [torch.tensor([1, 3, 3, 7], dtype=torch.int64, device=DEV), torch.tensor([0, 1, 2, 3], dtype=torch.int32, device=DEV)]
     b = [torch.tensor([0, 3, 8], dtype=torch.int64, device=DEV), torch.tensor([9, 1, 9], dtype=torch.int32, device=DEV)]
     cols = [torch.cat([a[0], b[0]]), torch.cat([a[1], b[1]])]
