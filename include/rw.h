@@ -40,7 +40,7 @@ typedef int32_t rw_status;
 #define RW_E_TYPE (-2)         /* type mismatch (col-vs-col atom, join key, group column) */
 #define RW_E_UNSORTED (-3)     /* JOIN input not declared sorted on the join key (A6) */
 #define RW_E_OVERFLOW (-4)     /* strict mode: i64/u64 expression may wrap (A8) */
-#define RW_E_UNSUPPORTED (-5)  /* outside what this build implements (e.g. nkey > 1) */
+#define RW_E_UNSUPPORTED (-5)  /* outside what this build implements (e.g. nkey > 2) */
 #define RW_E_CAPACITY (-6)     /* output capacity too small; required rows in out->n */
 #define RW_E_OOM (-7)
 #define RW_E_CUDA (-8)

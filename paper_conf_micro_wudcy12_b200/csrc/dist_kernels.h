@@ -43,6 +43,7 @@ struct OutPtrs {
 constexpr int kMpThreads = 256;
 constexpr int kMpItems = 16;
 constexpr int kMpC = kMpThreads * kMpItems;   // elements one merge group may hold
+constexpr int kMpCP = kMpC + kMpC / 16;      // shared-memory words of one buffer (padded)
 constexpr int kMpMaxRuns = 32;
 
 struct MpLaunch {
@@ -58,7 +59,7 @@ struct MpLaunch {
     int64_t S;
     int64_t NG;
     uint64_t *sv;                        // S sample images
-    uint32_t *cuts;                      // S x nrun
+    uint32_t *cuts;                      // NG x nrun: cut of every run at every group start
     int64_t *bound;                      // NG group-start samples
     void *out[kMaxMergeCols];
 };

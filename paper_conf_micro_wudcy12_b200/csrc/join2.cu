@@ -608,7 +608,7 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                 const int w = P.out_w[c];
                 // the ring is circular: a column's segment may wrap at R (16-byte aligned,
                 // so no vector straddles the end) -> copied in two pieces
-                const uint32_t so = (roff + coff) % R;
+                const uint32_t so = roff + coff >= R ? roff + coff - R : roff + coff;   // roff, coff < R
                 coff += al16j(tot * w);
                 const uint32_t n1 = min(tot, (R - so) / (uint32_t)w);
                 for (int piece = 0; piece < 2; piece++) {
@@ -956,7 +956,7 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             for (int c = 0; c < P.nout; c++) {
                 const int w = P.out_w[c];
                 const char *src = loc_ptr(P.out_loc[c], st, scratch);
-                const uint32_t so = (pos + coff) % R;
+                const uint32_t so = pos + coff >= R ? pos + coff - R : pos + coff;   // pos, coff < R
                 coff += al16j(tot * w);
                 if (so + tot * (uint32_t)w > R) {
                     // this column's segment wraps at the ring's end: positions mod R

@@ -1071,6 +1071,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         else if (p->o.reserved[4] == 2) vars.push_back({256, 4});
         else if (p->o.reserved[4] == 4) vars.push_back({256, 8});
         else if (p->o.reserved[4] == 5) vars.push_back({256, 16});
+        else if (p->o.reserved[4] == 6) vars.push_back({384, 8});
         else if (nbr > 1) vars = {{256, 8}, {256, 4}};
         else vars = {{256, 16}, {256, 8}, {256, 4}};
         const int want_stages_e = p->o.stages > 0 ? std::min(std::max(p->o.stages, 2), 8) : 0;
@@ -2811,7 +2812,7 @@ static void merge_runs_single_pass(const void *const *cols, const uint64_t *pack
     cuda_check(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev), "attr");
     void *sv = nullptr, *cuts = nullptr, *bound = nullptr;
     cuda_check(cudaMallocAsync(&sv, (size_t)M.S * 8, st), "cudaMallocAsync");
-    cudaError_t e1 = cudaMallocAsync(&cuts, (size_t)M.S * nrun * 4, st);
+    cudaError_t e1 = cudaMallocAsync(&cuts, (size_t)M.NG * nrun * 4, st);
     cudaError_t e2 = cudaMallocAsync(&bound, (size_t)M.NG * 8, st);
     cudaError_t e3 = cudaSuccess;
     if (e1 == cudaSuccess && e2 == cudaSuccess) {

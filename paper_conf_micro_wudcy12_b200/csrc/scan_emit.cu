@@ -106,7 +106,7 @@ __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1
     for (int c = c0; c < c1; c++) {
         const int w = P.out_w[c];
         const char *src = loc_ptr(P.out_loc[c], st, scratch);
-        const uint32_t so = (pos + coff) % R;
+        const uint32_t so = pos + coff >= R ? pos + coff - R : pos + coff;   // pos, coff < R
         coff += al16e(total * w);
         if (so + total * (uint32_t)w > R) {
             wrap_scatter<NT, G>(ring, R, so, w, src, m, sp);
@@ -263,7 +263,7 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                     const int w = P.out_w[c];
                     // the ring is circular: a column's segment may wrap at R (16-byte
                     // aligned, so no vector straddles the end) -> copied in two pieces
-                    const uint32_t so = (roff + coff) % R;
+                    const uint32_t so = roff + coff >= R ? roff + coff - R : roff + coff;   // roff, coff < R
                     coff += al16e(total * w);
                     const uint32_t n1 = min(total, (R - so) / (uint32_t)w);
                     for (int piece = 0; piece < 2; piece++) {
@@ -522,6 +522,8 @@ int scan_emit_occupancy(int nt, int items, bool multi, size_t smem)
         return items == 4 ? emit_occ<256, 4, true>(smem) : emit_occ<256, 8, true>(smem);
     if (nt == 512)
         return emit_occ<512, 8, false>(smem);
+    if (nt == 384)
+        return emit_occ<384, 8, false>(smem);
     return items == 4 ? emit_occ<256, 4, false>(smem) : items == 16 ? emit_occ<256, 16, false>(smem)
                                                       : emit_occ<256, 8, false>(smem);
 }
@@ -541,6 +543,8 @@ cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, in
         return items == 4 ? emit_go<256, 4, true>(P, L, smem, grid, s) : emit_go<256, 8, true>(P, L, smem, grid, s);
     if (nt == 512)
         return emit_go<512, 8, false>(P, L, smem, grid, s);
+    if (nt == 384)
+        return emit_go<384, 8, false>(P, L, smem, grid, s);
     return items == 4 ? emit_go<256, 4, false>(P, L, smem, grid, s)
                       : items == 16 ? emit_go<256, 16, false>(P, L, smem, grid, s) : emit_go<256, 8, false>(P, L, smem, grid, s);
 }
