@@ -66,6 +66,7 @@ def parse():
     ap.add_argument("--items", type=int, default=0, help="rows per thread of the scan tile (0 = auto)")
     ap.add_argument("--variant", type=int, default=0, help="2 = 512x4, 3 = 512x8 compute threads x rows")
     ap.add_argument("--gring", type=int, default=0, help="1 = compacted-tile ring in global memory (L2)")
+    ap.add_argument("--agg-mode", type=int, default=0, help="aggregate terminal switch (2 = Q1 shape through the interpreter)")
     return ap.parse_args()
 
 
@@ -395,7 +396,8 @@ def main():
 
     def make(fuse):
         plan, ids = build_gpu_plan(spec, device=local, stream=stream, fuse=fuse, stages=args.stages,
-                                   ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg, items=args.items, variant=args.variant, gring=args.gring)
+                                   ctas_per_sm=args.ctas, defer=args.defer, dbg=args.dbg, items=args.items, variant=args.variant, gring=args.gring,
+                                   agg_mode=args.agg_mode)
         if "outs" in spec:
             # input-dependence fusion: one output relation per branch
             cap = max(nrows.values())

@@ -777,6 +777,110 @@ __device__ inline void agg_tile_reg(const ChainProg &P, const char *stage, const
         atomicAdd(err + 2, 1);
 }
 
+// Fused row path of the kNarrowNT instance for the TPC-H Q1 program shape (host-checked,
+// ChainProg::q1fused, pattern (e) of Fig. 14): ops = [SELECT i32 column vs
+// constant, d = a * (k1 -/+ b), c = d * (k2 -/+ e)] and sums = [2 narrow stage columns,
+// 1 wide stage column, d, c].  The same arithmetic as the interpreter (wrap mod 2^64,
+// reading A8), evaluated per row in registers: the computed columns never touch shared
+// memory and there is no per-op dispatch (the paper generates this code per fused group,
+// P:177-179; here it is compiled ahead of time for this shape).
+template <int NT, int ITEMS>
+__device__ inline void agg_tile_q1(const ChainProg &P, const char *stage, uint32_t mask, RegAgg &R,
+                                   unsigned long long *cta_acc, int64_t &since_flush, int32_t *err)
+{
+    const int tid = threadIdx.x;
+    // SELECT atom: the common comparisons inline, the rest through the generic dispatch
+    const uint32_t pcode = P.ops[0].code;
+    const int64_t pk = P.ops[0].k;
+    const char *pa = stage + P.ops[0].a;
+    uint32_t ok;
+    if (pcode == T_I32 * 8 + C_LE)
+        ok = pred_loop<NT, ITEMS, int32_t, C_LE, false>(pa, nullptr, (int32_t)pk, mask);
+    else if (pcode == T_I32 * 8 + C_LT)
+        ok = pred_loop<NT, ITEMS, int32_t, C_LT, false>(pa, nullptr, (int32_t)pk, mask);
+    else
+        ok = run_pred<NT, ITEMS>(pcode, pk, pa, nullptr, mask);
+    // group codes (first group column slowest), out-of-domain rows counted
+    uint32_t g[ITEMS];
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++)
+        g[k] = 0;
+    const uint32_t sel = ok;
+    for (int c = 0; c < P.ngc; c++) {
+        const char *b = stage + P.g_loc[c];
+        const uint32_t dom = (uint32_t)P.gdomain[c];
+        switch (P.g_type[c]) {
+        case T_U8:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint8_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        case T_I32:
+        case T_U32:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint32_t v = ((const uint32_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + v;
+            }
+            break;
+        default:
+#pragma unroll
+            for (int k = 0; k < ITEMS; k++) {
+                const uint64_t v = ((const uint64_t *)b)[k * NT + tid];
+                if (v >= dom) ok &= ~(1u << k);
+                g[k] = g[k] * dom + (uint32_t)v;
+            }
+            break;
+        }
+    }
+    if (ok != sel)
+        atomicAdd(err, __popc(sel & ~ok));
+    const int rows = __popc(ok);
+    if (since_flush + rows > P.flush_rows) {
+        reg_agg_flush(P, R, cta_acc);
+        since_flush = 0;
+    }
+    since_flush += rows;
+    const uint64_t *xa = (const uint64_t *)(stage + P.ops[1].a);   // e.g. price
+    const uint64_t *xb = (const uint64_t *)(stage + P.ops[1].b);   // e.g. disc
+    const uint64_t *xe = (const uint64_t *)(stage + P.ops[2].b);   // e.g. tax
+    const uint64_t k1 = (uint64_t)P.ops[1].k, k2 = (uint64_t)P.ops[2].k;
+    const bool n1 = (P.ops[1].tb & kNegB) != 0, n2 = (P.ops[2].tb & kNegB) != 0;
+    const uint64_t *s0 = (const uint64_t *)(stage + P.agg_loc[0]);
+    const uint64_t *s1 = (const uint64_t *)(stage + P.agg_loc[1]);
+    const uint64_t *s2 = (const uint64_t *)(stage + P.agg_loc[2]);
+    uint64_t orv = 0;
+#pragma unroll
+    for (int k = 0; k < ITEMS; k++) {
+        const bool on = (ok >> k) & 1u;
+        const uint32_t gk = on ? g[k] : 0xffffffffu;   // failing rows match no group
+        const int r = k * NT + tid;
+        const uint64_t b = xb[r], e = xe[r];
+        const uint64_t d = xa[r] * (n1 ? k1 - b : k1 + b);
+        const uint64_t c = d * (n2 ? k2 - e : k2 + e);
+        const uint64_t v0 = s0[r], v1 = s1[r], v2 = s2[r];
+        if (on)
+            orv |= v0 | v1;
+#pragma unroll
+        for (int dd = 0; dd < kRegD; dd++) {
+            if (gk == (uint32_t)dd) {
+                R.c[dd] += 1u;
+                R.n[dd][0] += (uint32_t)v0;
+                R.n[dd][1] += (uint32_t)v1;
+                R.s[dd][2] += v2;
+                R.s[dd][3] += d;
+                R.s[dd][4] += c;
+            }
+        }
+    }
+    if (orv >> P.narrow_bits)
+        atomicAdd(err + 2, 1);
+}
+
 // End-of-kernel combine of the thread-private partials: one thread per (group,
 // aggregate) slot sums the NT partials exactly in 128 bits (no shared atomics, whose
 // 64-bit form is a CAS loop on sm_100), then adds the slot into cta_acc.

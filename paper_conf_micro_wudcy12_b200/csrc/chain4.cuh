@@ -66,8 +66,10 @@ __device__ __forceinline__ V4<uint64_t> ld4_ext(const char *base, int type, int 
     return o;
 }
 
+// (threadIdx.x % NT: the emitting scan kernel may run several teams of NT compute
+// threads, each on its own tiles; every other kernel's compute threads are [0, NT))
 template <int NT>
-__device__ __forceinline__ int row4(int g) { return (g * NT + (int)threadIdx.x) * 4; }
+__device__ __forceinline__ int row4(int g) { return (g * NT + (int)(threadIdx.x % NT)) * 4; }
 
 // SELECT atom over the thread's G x 4 rows: clears the bits of rows failing `a CMP b`
 template <int NT, int G, typename T, int CMP, bool BSLOT>

@@ -92,6 +92,7 @@ struct ChainProg {
     int32_t agg_mode;                   // 0: thread-private partials in smem; 2: register one-hot (D <= kRegD, nagg <= kRegA)
     int32_t agg_narrow;                 // mode 2: the first agg_narrow sums are non-negative with |v| < 2^16 and
                                         // accumulate in 32-bit registers (flush_rows keeps them below 2^32)
+    int32_t q1fused;                    // kNarrowNT instance: the Q1 program shape runs fused per row (agg_tile_q1)
     int32_t narrow_bits;                // every narrow value is < 2^narrow_bits (declared bounds); the kernel ORs
                                         // the narrow values of a tile and counts a violation into err[2]
     // input-dependence fusion (§4.4, Fig. 14(d)): nbranch chains over the same

@@ -367,6 +367,14 @@ __global__ void __launch_bounds__(NT + aux_threads(AGG), AGG ? 1 : 2) k_scan_cha
                     if (k * NT + tid < rows)
                         mask0 |= 1u << k;
             }
+            if constexpr (AGG && NT == kNarrowNT) {
+                if (P.q1fused) {
+                    // Q1 program shape: SELECT, arithmetic and aggregate fused per row
+                    agg_tile_q1<NT, ITEMS>(P, st, mask0, racc, cta_acc, since_flush, L.err);
+                    release_stage();
+                    continue;
+                }
+            }
             uint32_t mask = run_ops<NT, ITEMS>(P, 0, NB > 1 ? (int)P.br_op_end[0] : P.nops, st, scratch, mask0);
             if ((L.dbg & 4) && tid == 0)
                 L.dbg_ts[12 * t + 6] = globaltimer();

@@ -111,8 +111,8 @@ cudaError_t join_emit_launch(const ChainProg &P, const TileLaunch &L, const Join
 
 // emitting scan kernel (scan_emit.cu): compacting SELECT / PROJECT chains, 1..4 branches
 size_t emit_ctl_bytes();
-int scan_emit_occupancy(int nt, int items, bool multi, size_t smem);
+int scan_emit_occupancy(int nt, int items, bool multi, size_t smem, int teams = 1);
 cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, int items, size_t smem, int grid,
-                             cudaStream_t s);
+                             cudaStream_t s, int teams = 1);
 
 }  // namespace rw

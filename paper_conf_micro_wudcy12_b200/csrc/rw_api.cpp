@@ -92,7 +92,8 @@ struct Lowered {
     std::vector<int> in_src;      // input slot i <- source column in_src[i]
     int items = 8, stages = 2, ctas = 1;
     int tile = 2048;              // rows per tile
-    int nt = 256;                 // compute threads per CTA
+    int nt = 256;                 // compute threads per CTA (emit kernel: per team)
+    int teams = 1;                // emit kernel: teams of nt compute threads on alternate tiles
     uint32_t gring_bytes = 0;     // per-CTA global ring bytes (0: ring in smem)
     bool direct = false;          // no SELECT: outputs written at their row offsets
     int ring = 0;                 // scan kernel: output ring entries
@@ -1065,13 +1066,15 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         // for computed columns (a stage holds its tile until the tile's offset resolves),
         // per-thread hold words, and one compaction buffer per compute warp (resource
         // budget, §4.3.3).  Variants: compute threads x rows per thread.
-        struct EVar { int nt, items; };
+        struct EVar { int nt, items, teams = 1; };
         std::vector<EVar> vars;
         if (p->o.reserved[4] == 3) vars.push_back({512, 8});
         else if (p->o.reserved[4] == 2) vars.push_back({256, 4});
         else if (p->o.reserved[4] == 4) vars.push_back({256, 8});
         else if (p->o.reserved[4] == 5) vars.push_back({256, 16});
         else if (p->o.reserved[4] == 6) vars.push_back({384, 8});
+        else if (p->o.reserved[4] == 7 && nbr == 1) vars.push_back({128, 16, 2});
+        else if (p->o.reserved[4] == 8 && nbr == 1) vars.push_back({256, 8, 2});
         else if (nbr > 1) vars = {{256, 8}, {256, 4}};
         else vars = {{256, 16}, {256, 8}, {256, 4}};
         const int want_stages_e = p->o.stages > 0 ? std::min(std::max(p->o.stages, 2), 8) : 0;
@@ -1110,7 +1113,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                     if (!direct_e && !Rg && Rs < W) continue;
                     const size_t smem = base + (size_t)S * SB + Rs;
                     if (smem > per_cta) continue;
-                    if (scan_emit_occupancy(v.nt, v.items, nbr > 1, smem) < occ_t) continue;
+                    if (scan_emit_occupancy(v.nt, v.items, nbr > 1, smem, v.teams) < occ_t) continue;
                     // input bytes in flight per SM (capped: 128 KB covers the HBM latency;
                     // more stages only shrink the shared ring), the larger tile, then the
                     // larger shared ring
@@ -1120,6 +1123,7 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                         best = sc;
                         L.items = v.items;
                         L.nt = v.nt;
+                        L.teams = v.teams;
                         L.tile = T;
                         L.stages = S;
                         L.smem = smem;
@@ -1289,6 +1293,26 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
     // the kNarrowNT instance compiles only the 5-sum / 2-narrow / all-64-bit row loop
     if (L.agg && L.nt == kNarrowNT && !(P.nagg == 5 && P.agg_narrow == 2 && all64 && P.agg_mode == 2))
         raise(RW_E_STATE, "internal: Q1-specialised aggregate instance selected for another plan shape");
+    // ... and, for exactly the Q1 program shape, the fused row path (agg_tile_q1):
+    // SELECT on an i32 stage column vs a constant, then two i64 fixed-point factors
+    // d = a * (k -/+ b), c = d * (k -/+ e) over stage columns, summed as the last two of
+    // [narrow, narrow, wide stage column, d, c].  opts.reserved[7] == 2 keeps the interpreter.
+    P.q1fused = 0;
+    if (L.agg && L.nt == kNarrowNT && P.nops == 3 && p->o.reserved[7] != 2) {
+        const DevOp &o0 = P.ops[0], &o1 = P.ops[1], &o2 = P.ops[2];
+        const uint8_t mulaff = (uint8_t)(64 + T_I64 * 8 + E_MULAFF);
+        auto stage_loc = [](uint32_t loc) { return (loc & kLocScratch) == 0; };
+        const bool ok = o0.kind == K_PRED && o0.code < 64 && (o0.code >> 3) == T_I32 && stage_loc(o0.a) &&
+                        o1.kind == K_EXPR && o1.code == mulaff && o2.kind == K_EXPR && o2.code == mulaff &&
+                        o1.ta == T_I64 && (o1.tb & 0x7f) == T_I64 && o2.ta == T_I64 && (o2.tb & 0x7f) == T_I64 &&
+                        stage_loc(o1.a) && stage_loc(o1.b) && stage_loc(o2.b) && o2.a == o1.dst &&
+                        P.agg_loc[3] == o1.dst && P.agg_loc[4] == o2.dst && stage_loc(P.agg_loc[0]) &&
+                        stage_loc(P.agg_loc[1]) && stage_loc(P.agg_loc[2]);
+        bool gstage = true;
+        for (int c = 0; c < P.ngc; c++)
+            gstage = gstage && stage_loc(P.g_loc[c]);
+        P.q1fused = ok && gstage ? 1 : 0;
+    }
     if (global_ring && !L.direct) {
         size_t W = 0;
         for (int c = 0; c < P.nout; c++)
@@ -1779,7 +1803,7 @@ void run_group(ExecCtx &X, int gi)
             TL.n_dev = n_dev;
             if (L.emit) {
                 TL.delay = L.delay;
-                cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream), "k_scan_emit");
+                cuda_check(scan_emit_launch(L.P, TL, L.nt, L.items, L.smem, grid, p->stream, L.teams), "k_scan_emit");
             } else {
                 cuda_check(scan_chain_launch(L.P, TL, false, L.nt, L.items, L.smem, grid, p->stream), "k_scan_chain");
             }
@@ -2241,7 +2265,7 @@ std::string explain(rw_plan *p, int out_node)
             std::vector<int> st = g.kind == G_SCAN ? p->nodes[g.source].types : join_src_types(p, g);
             lower(p, g, st, L);
             if (L.emit)
-                s << " | emitting kernel k_scan_emit<" << L.nt << "," << L.items << ">"
+                s << " | emitting kernel k_scan_emit<" << L.nt << "," << L.items << (L.teams > 1 ? ",2 teams" : "") << ">"
                   << (L.direct ? ", direct (no SELECT)" : "");
             s << " | tile " << L.tile << " rows (" << L.items << "/thread), stages " << L.stages << ", out ring " << L.out_bytes << " B"
               << ", smem " << L.smem
@@ -2251,7 +2275,7 @@ std::string explain(rw_plan *p, int out_node)
             {
                 s << ", groups " << L.P.D << ", sums " << L.P.nagg;
                 if (L.P.agg_mode == 2)
-                    s << ", register one-hot terminal";
+                    s << ", register one-hot terminal" << (L.P.q1fused ? " (Q1 program fused per row)" : "");
                 else if (L.P.agg_mode == 3)
                     s << ", global-atomic terminal";
                 else

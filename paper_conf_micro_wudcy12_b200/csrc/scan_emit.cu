@@ -42,8 +42,12 @@ struct EmitCtl {
     uint64_t full[kEmitMaxStages], empty[kEmitMaxStages];
     int64_t tile[kEmitMaxStages];
     EmitBlk blk[kEmitSlots];
-    uint32_t cnt[2][kMaxBranch][kEmitMaxCnt];   // double-buffered by tile parity
+    uint32_t cnt[4][kMaxBranch][kEmitMaxCnt];   // [team * 2 + parity of the team's tile]
     volatile uint32_t tail[2];                  // ring bytes released by the writers (monotone, wraps): smem, L2
+    // two-team kernels: ring reservations are made in block order through this state
+    // (slot i & 3 holds the (head, pos) of both rings before block i)
+    volatile uint32_t rsv_seq;
+    volatile uint32_t rsv[4][4];
 };
 
 static __host__ __device__ inline size_t al128e(size_t x) { return (x + 127) / 128 * 128; }
@@ -154,13 +158,20 @@ __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1
 // larger than a quarter of it (high-selectivity chains) in a per-CTA slice of an
 // L2-resident global buffer, so that enough tiles stay in flight for any selectivity.
 // The choice depends only on the block size, so every compute warp makes the same one.
-template <int NT, int ITEMS, bool MULTI>
-__global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_constant__ ChainProg P,
-                                                               const __grid_constant__ TileLaunch L)
+//
+// TEAMS = 2: the compute warps form two teams of NT threads that take alternate tiles
+// (team = stage use mod 2), each with its own named barrier and count buffers, so one
+// team's barrier, prefix and compaction overlap the other's evaluation; the compacted
+// blocks still reserve their ring bytes in tile order (ctl->rsv_seq).
+template <int NT, int ITEMS, bool MULTI, int TEAMS = 1>
+__global__ void __launch_bounds__(NT * TEAMS + kEmitAux, 1) k_scan_emit(const __grid_constant__ ChainProg P,
+                                                                       const __grid_constant__ TileLaunch L)
 {
     constexpr int G = ITEMS / 4;
     constexpr int T = NT * ITEMS;
-    constexpr int NW = NT / 32;
+    constexpr int NW = NT / 32;                 // compute warps per team
+    constexpr int NWC = NW * TEAMS;             // compute warps
+    static_assert(TEAMS == 1 || !MULTI, "two-team kernel: single chain only");
     static_assert(ITEMS % 4 == 0 && G <= 4 && G * NW <= kEmitMaxCnt, "emit tile geometry");
     constexpr int NBR = MULTI ? kMaxBranch : 1;
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -191,11 +202,14 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
         }
         ctl->tail[0] = 0;
         ctl->tail[1] = 0;
+        ctl->rsv_seq = 0;
+        for (int q = 0; q < 4; q++)
+            ctl->rsv[0][q] = 0;
         fence_mbar_init();
     }
     __syncthreads();
 
-    if (warp == NW) {
+    if (warp == NWC) {
         // ---------------- producer warp ----------------
         if (lane == 0) {
             uint32_t tx_bytes = 0;
@@ -208,9 +222,10 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
             int64_t tn = (int64_t)atomicAdd(&L.ctrs[0], 1u);
             int s = 0;
             uint32_t eph = 1;                               // parity of the stage's previous use
+            int sentinels = 0;                              // one per team (tile = ntiles + team-order)
             for (uint32_t i = 0;; ++i) {
-                const int64_t t = tn;
-                if (t < ntiles)
+                const int64_t t = tn >= ntiles ? ntiles + sentinels : tn;
+                if (tn < ntiles)
                     tn = (int64_t)atomicAdd(&L.ctrs[0], 1u);
                 if (i >= (uint32_t)S)
                     mbar_wait(&ctl->empty[s], eph);
@@ -227,7 +242,7 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 } else {
                     mbar_arrive(&ctl->full[s]);
                 }
-                if (t >= ntiles)
+                if (t >= ntiles && ++sentinels == TEAMS)
                     break;
                 if (++s == S) {
                     s = 0;
@@ -235,9 +250,9 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 }
             }
         }
-    } else if (warp > NW) {
+    } else if (warp > NWC) {
         // ---------------- writer warps: look-back + copy-out, block i = wi mod kWriters ----------------
-        const int wi = warp - NW - 1;
+        const int wi = warp - NWC - 1;
         if (emit) {
             for (uint32_t i = wi;; i += kWriters) {
                 const int j = (int)(i % kEmitSlots);
@@ -306,21 +321,19 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
         }
     } else {
         // ---------------- compute warps ----------------
+        const int team = TEAMS > 1 ? warp / NW : 0;
+        const int ltid = tid - team * NT, lwarp = warp - team * NW;   // within the team
         uint32_t head_s = 0, hpos_s = 0, head_g = 0, hpos_g = 0;   // ring reservations, replicated in every warp
-        uint32_t ublk = 0;                              // compacted blocks emitted (tiles x branches)
-        int s = -1;
-        uint32_t fph = 1;
-        for (uint32_t i = 0;; ++i) {
-            if (++s == S) {
-                s = 0;
-            }
-            if (s == 0)
-                fph ^= 1u;
+        for (uint32_t i = team;; i += TEAMS) {
+            const int s = (int)(i % (uint32_t)S);
+            const uint32_t fph = (i / (uint32_t)S) & 1u;
+            uint32_t ublk = i * (uint32_t)NB;                // compacted blocks before this tile's (tile order)
             mbar_wait(&ctl->full[s], fph);
             const int64_t t = ctl->tile[s];
             if (t >= ntiles) {
-                if (emit && tid == 0) {
-                    // one sentinel block per writer warp (consecutive slots)
+                // the first sentinel's team sends one sentinel block per writer warp
+                // (consecutive slots after every real block)
+                if (emit && ltid == 0 && t == ntiles) {
                     for (uint32_t u = ublk; u < ublk + kWriters; ++u) {
                         const int ju = (int)(u % kEmitSlots);
                         if (u >= kEmitSlots)
@@ -394,7 +407,7 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
             // evaluate every branch: survivor masks and per-warp counts of each 4-row group
             // (a second branch recomputes into the same scratch, so branches are evaluated
             // and compacted one after the other; branch b's counts are published first)
-            const int par = (int)(i & 1u);
+            const int par = TEAMS > 1 ? team * 2 + (int)((i / TEAMS) & 1u) : (int)(i & 1u);
             for (int b = 0; b < NB; b++) {
                 const uint32_t m = run_ops4<NT, G>(P, b ? (int)P.br_op_end[b - 1] : 0, MULTI ? (int)P.br_op_end[b] : P.nops,
                                                    st, scratch, mask0);
@@ -413,9 +426,9 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 if (lane == 31)
 #pragma unroll
                     for (int g = 0; g < G; g++)
-                        ctl->cnt[par][b][g * NW + warp] = (inc >> (8 * g)) & 255u;
+                        ctl->cnt[par][b][g * NW + lwarp] = (inc >> (8 * g)) & 255u;
                 const uint32_t ex = inc - pk;
-                bar_sync(kComputeBarEmit, NT);
+                bar_sync(kComputeBarEmit + team, NT);
                 // block prefix of (group, warp) in tile order and the tile total
                 const uint32_t v = lane < G * NW ? ctl->cnt[par][b][lane] : 0u;
                 uint32_t bin = v;
@@ -429,8 +442,8 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 uint32_t pre[G];
 #pragma unroll
                 for (int g = 0; g < G; g++)
-                    pre[g] = __shfl_sync(0xffffffffu, bin - v, g * NW + warp) + ((ex >> (8 * g)) & 255u);
-                if (warp == 0 && lane == 0 && t > 0 && !(L.dbg & 1))
+                    pre[g] = __shfl_sync(0xffffffffu, bin - v, g * NW + lwarp) + ((ex >> (8 * g)) & 255u);
+                if (lwarp == 0 && lane == 0 && t > 0 && !(L.dbg & 1))
                     // publish the tile aggregate before anything can block this CTA
                     st_relaxed_u64(&L.status[b * L.status_stride + t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
                 // ring bytes of the compacted block (blocks never wrap); every warp computes
@@ -442,7 +455,22 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 // quarter of it (then to the L2 ring); wait until its bytes are free
                 const int where = Rg != 0u && (Rs == 0u || need > Rs / 4u) ? 1 : 0;
                 const uint32_t R = where ? Rg : Rs;
-                const uint32_t pos = where ? hpos_g : hpos_s, used = need;
+                const uint32_t used = need;
+                if constexpr (TEAMS > 1) {
+                    // the other team reserves the blocks in between: take the ring state
+                    // left by block ublk - 1 (slot ublk & 3 is not rewritten before every
+                    // warp of this team has passed its next barrier)
+                    if (lane == 0)
+                        while (ctl->rsv_seq < ublk)
+                            __nanosleep(20);
+                    __syncwarp();
+                    const uint32_t sl = ublk & 3u;
+                    head_s = ctl->rsv[sl][0];
+                    hpos_s = ctl->rsv[sl][1];
+                    head_g = ctl->rsv[sl][2];
+                    hpos_g = ctl->rsv[sl][3];
+                }
+                const uint32_t pos = where ? hpos_g : hpos_s;
                 const uint32_t hd = where ? head_g : head_s;
                 const int j = (int)(ublk % kEmitSlots);
                 if (ublk >= kEmitSlots)
@@ -457,6 +485,17 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 const uint32_t np = pos + need >= R ? pos + need - R : pos + need;
                 if (where) { head_g = hd + used; hpos_g = np; }
                 else { head_s = hd + used; hpos_s = np; }
+                if constexpr (TEAMS > 1) {
+                    if (lwarp == 0 && lane == 0) {
+                        const uint32_t sl = (ublk + 1) & 3u;
+                        ctl->rsv[sl][0] = head_s;
+                        ctl->rsv[sl][1] = hpos_s;
+                        ctl->rsv[sl][2] = head_g;
+                        ctl->rsv[sl][3] = hpos_g;
+                        __threadfence_block();
+                        ctl->rsv_seq = ublk + 1;
+                    }
+                }
                 // compact the survivors into the block, tile order: each surviving row's
                 // position is computed once, then every column stores with it
                 uint32_t sp[G][4];
@@ -477,7 +516,7 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
                 if (lane == 0) {
                     if (where)
                         __threadfence_block();
-                    if (warp == 0) {
+                    if (lwarp == 0) {
                         ctl->blk[j].tile = t;
                         ctl->blk[j].total = total;
                         ctl->blk[j].roff = pos;
@@ -505,19 +544,21 @@ __global__ void __launch_bounds__(NT + kEmitAux, 1) k_scan_emit(const __grid_con
 // ---------------------------------------------------------------------------
 // host side
 // ---------------------------------------------------------------------------
-template <int NT, int ITEMS, bool MULTI>
+template <int NT, int ITEMS, bool MULTI, int TEAMS = 1>
 static int emit_occ(size_t smem)
 {
-    auto f = k_scan_emit<NT, ITEMS, MULTI>;
+    auto f = k_scan_emit<NT, ITEMS, MULTI, TEAMS>;
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, NT + kEmitAux, smem) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, NT * TEAMS + kEmitAux, smem) != cudaSuccess)
         return 0;
     return n;
 }
 
-int scan_emit_occupancy(int nt, int items, bool multi, size_t smem)
+int scan_emit_occupancy(int nt, int items, bool multi, size_t smem, int teams)
 {
+    if (teams == 2)
+        return nt == 128 ? emit_occ<128, 16, false, 2>(smem) : emit_occ<256, 8, false, 2>(smem);
     if (multi)
         return items == 4 ? emit_occ<256, 4, true>(smem) : emit_occ<256, 8, true>(smem);
     if (nt == 512)
@@ -528,17 +569,19 @@ int scan_emit_occupancy(int nt, int items, bool multi, size_t smem)
                                                       : emit_occ<256, 8, false>(smem);
 }
 
-template <int NT, int ITEMS, bool MULTI>
+template <int NT, int ITEMS, bool MULTI, int TEAMS = 1>
 static cudaError_t emit_go(const ChainProg &P, const TileLaunch &L, size_t smem, int grid, cudaStream_t s)
 {
-    cudaFuncSetAttribute(k_scan_emit<NT, ITEMS, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k_scan_emit<NT, ITEMS, MULTI><<<grid, NT + kEmitAux, smem, s>>>(P, L);
+    cudaFuncSetAttribute(k_scan_emit<NT, ITEMS, MULTI, TEAMS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k_scan_emit<NT, ITEMS, MULTI, TEAMS><<<grid, NT * TEAMS + kEmitAux, smem, s>>>(P, L);
     return cudaGetLastError();
 }
 
 cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, int items, size_t smem, int grid,
-                             cudaStream_t s)
+                             cudaStream_t s, int teams)
 {
+    if (teams == 2 && P.nbranch == 1)
+        return nt == 128 ? emit_go<128, 16, false, 2>(P, L, smem, grid, s) : emit_go<256, 8, false, 2>(P, L, smem, grid, s);
     if (P.nbranch > 1)
         return items == 4 ? emit_go<256, 4, true>(P, L, smem, grid, s) : emit_go<256, 8, true>(P, L, smem, grid, s);
     if (nt == 512)

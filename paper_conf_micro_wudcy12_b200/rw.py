@@ -186,7 +186,7 @@ class Plan:
         # fusion upstream of a JOIN, 8 / 9 = emitting kernel with only its shared / only its
         # L2 ring, 10 = emitting kernel for every compacting chain
         o.reserved[6] = gring
-        o.reserved[7] = agg_mode           # 1 = force the thread-private-partials aggregate terminal
+        o.reserved[7] = agg_mode           # 1 = force the thread-private-partials aggregate terminal, 2 = no fused Q1 row path
         self.device = device
         h = ctypes.c_void_p()
         check(lib().rw_plan_create(ctypes.byref(h), ctypes.byref(o)))

@@ -8,10 +8,10 @@ for spec in ${PROFS:-"c4:k_scan_chain:1:1:22800000360" "cd:k_scan_chain:1:1:0" "
   IFS=: read CFG KREGEX SKIP CNT ALG <<< "$spec"
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:'^k_' -c 60 --csv \
       --log-file gpurun_out/launches_${CFG}.csv \
-      python bench.py --config $CFG --steps 3 --warmup 1 --no-e2e --no-cpu > gpurun_out/ncu_launch_${CFG}.log 2>&1
+      python bench.py --config $CFG --steps 3 --warmup 1 --no-e2e --no-cpu --no-unfused --no-sweep > gpurun_out/ncu_launch_${CFG}.log 2>&1
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"$KREGEX" -s $SKIP -c $CNT \
       -o /tmp/prof_${CFG} -f \
-      python bench.py --config $CFG --steps 2 --warmup 1 --no-e2e --no-unfused --no-cpu > gpurun_out/ncu_full_${CFG}.log 2>&1
+      python bench.py --config $CFG --steps 2 --warmup 1 --no-e2e --no-unfused --no-cpu --no-sweep > gpurun_out/ncu_full_${CFG}.log 2>&1
   RW_PROFILE_DIR=gpurun_out/profiles_out python scripts/summarize_ncu.py /tmp/prof_${CFG}.ncu-rep ${RW_ROUND_TAG:-r01e}_${CFG}_${KREGEX} $CFG $ALG > /dev/null 2>&1
   echo "$CFG prof rc=$?"
 done

@@ -31,6 +31,18 @@ def test_q1_both_agg_terminals(agg_mode):
     assert want in plan.explain(plan.out_id)
 
 
+@pytest.mark.parametrize("agg_mode", [0, 2])
+@pytest.mark.parametrize("n", [1, 2303, 2305, 300_001])
+def test_q1_fused_row_path_and_interpreter(agg_mode, n):
+    """The Q1 program shape runs fused per row in the 576-thread instance (agg_mode 0),
+    or through the micro-op interpreter (agg_mode 2): both equal the oracle."""
+    spec = workloads.c4_spec()
+    ins = workloads.c4_inputs(n, device=DEV, cfg=0x96)
+    got, plan = run_gpu(spec, ins, capacity=6, agg_mode=agg_mode)
+    assert_same(got, run_oracle(spec, ins))
+    assert ("Q1 program fused per row" in plan.explain(plan.out_id)) == (agg_mode == 0)
+
+
 @pytest.mark.parametrize("variant", [4, 5, 1, 6, 0])
 @pytest.mark.parametrize("n", [1, 1919, 1921, 300_001])
 def test_q1_wide_cta_variants(variant, n):

@@ -40,6 +40,30 @@ def test_selectivity_sweep(s):
     assert_same(got, run_oracle(spec, ins))
 
 
+@pytest.mark.parametrize("variant", [7, 8])          # two-team emitting kernels: 2 x 128 x 16, 2 x 256 x 8
+@pytest.mark.parametrize("n", SIZES + [300_001])
+def test_c2_two_team_kernel(variant, n):
+    """Two teams of compute warps on alternate tiles, ring reserved in tile order
+    (scan_emit.cu TEAMS = 2): same output, order included."""
+    spec = workloads.c2_spec()
+    ins = workloads.c2_inputs(n, device=DEV, cfg=0x8B)
+    got, plan = run_gpu(spec, ins, variant=variant)
+    assert_same(got, run_oracle(spec, ins))
+    if n > 0:
+        assert "2 teams" in plan.explain(plan.out_id)
+
+
+@pytest.mark.parametrize("variant", [7, 8])
+@pytest.mark.parametrize("s", [0.0, 0.1, 0.9, 1.0])
+def test_two_team_selectivity(variant, s):
+    """All-survive blocks go to the L2 ring, small ones to shared memory: both rings'
+    reservations pass between the teams."""
+    spec = workloads.c2_spec(s, s)
+    ins = workloads.c2_inputs(200_000, device=DEV, cfg=0x8C)
+    got, _ = run_gpu(spec, ins, variant=variant)
+    assert_same(got, run_oracle(spec, ins))
+
+
 @pytest.mark.parametrize("stages", [1, 2, 3, 4])
 def test_stage_counts(stages):
     spec = workloads.c2_spec()
