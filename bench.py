@@ -500,15 +500,20 @@ def main():
     ms_step = total_ms / args.steps
     value = n_in * world / (total_ms / 1e3 / args.steps)
 
-    # roofline of the dominant kernel.  C1/C2: the fused k_scan_chain is the whole step;
-    # C4: k_scan_chain<agg> (k_agg_finalize is a 1-CTA epilogue of a few us); C3/C5: the
-    # join pair (k_join_runs + k_join_expand), algorithmic bytes = inputs + output.
+    # roofline of the dominant kernel, timed as the step on the plan's stream (CUDA events).
+    # C1/C2: the fused k_scan_emit is the whole step; C4: k_scan_chain<576,4,agg> (the
+    # Q1 row path; k_agg_finalize is a 1-CTA epilogue of a few us); C3/C5: the join
+    # kernels (k_jsplit + k_jmatch + k_jtiles + k_join_emit); algorithmic bytes = inputs
+    # + output.
     alg_bytes = in_bytes + out_bytes
     peak, peak_src = measured_peak()
     kern_ms = statistics.mean(per)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
-    kname = {"c3": "k_join_runs + k_join_expand", "cc": "k_join_runs (key SELECTs fused) + k_join_expand", "c5": "exchange + k_join_runs + k_join_expand",
-             "cs": "k_set_splits + k_set_op x2 + k_set_scan"}.get(cfg, "k_scan_chain")
+    kname = {"c3": "k_jsplit + k_jmatch + k_jtiles + k_join_emit",
+             "cc": "k_jsplit + k_jmatch (key SELECTs fused) + k_jtiles + k_join_emit",
+             "c5": "exchange + 2 x (k_jsplit + k_jmatch) + k_jtiles + k_join_emit (3-input group)",
+             "cs": "k_set_splits + k_set_op", "c4": "k_scan_chain<576,4,agg> (Q1 row path) + k_agg_finalize",
+             "cd": "k_scan_chain<256,8,multi>"}.get(cfg, "k_scan_emit")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "frac_nominal": achieved / NOMINAL_HBM_GBS, "nominal_peak": NOMINAL_HBM_GBS,
                 "traffic": ncu_traffic(cfg), "kernel": kname,
