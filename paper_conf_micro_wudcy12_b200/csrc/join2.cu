@@ -288,16 +288,35 @@ __global__ void __launch_bounds__(kMatchThreads, 4) k_jmatch(const __grid_consta
             lb = last_lb;
         }
     };
+    // heads in batches of 4: a chained match's weight loads (global) are all in flight
+    // before any is used
+    constexpr int HB = 4;
     uint32_t nrun = 0;
     uint64_t ncand = 0;
-    for (int k = k0; k < k1; k++) {
-        uint32_t la, lb;
-        lens(k, la, lb);
-        const int ia = hia[k];
-        if (la > 0 && lb > 0 && key_pass<K>(M, sA[ia])) {
-            nrun++;
-            ncand += (M.wA ? M.wA[i0 + ia] : (uint64_t)la) * lb;
+    for (int kb = k0; kb < k1; kb += HB) {
+        uint32_t lb[HB];
+        uint64_t w[HB];
+        bool ok[HB];
+#pragma unroll
+        for (int u = 0; u < HB; u++) {
+            const int k = kb + u;
+            uint32_t la = 0;
+            lb[u] = 0;
+            ok[u] = false;
+            w[u] = 0;
+            if (k < k1) {
+                lens(k, la, lb[u]);
+                const int ia = hia[k];
+                ok[u] = la > 0 && lb[u] > 0 && key_pass<K>(M, sA[ia]);
+                w[u] = M.wA ? (ok[u] ? __ldg(M.wA + i0 + ia) : 0ull) : (uint64_t)la;
+            }
         }
+#pragma unroll
+        for (int u = 0; u < HB; u++)
+            if (ok[u]) {
+                nrun++;
+                ncand += w[u] * lb[u];
+            }
     }
     // 4. block exclusive scan of (runs, candidates) in head order
     uint32_t ir = nrun;
@@ -346,37 +365,64 @@ __global__ void __launch_bounds__(kMatchThreads, 4) k_jmatch(const __grid_consta
         }
     }
     __syncthreads();
-    // 6. records of the matched runs, in key order
+    // 6. records of the matched runs, in key order (heads in batches of 4: every global
+    //    load of a batch is issued before its records are stored)
     int64_t r = base_run + br;
     uint64_t off = base_cand + bc;
-    for (int k = k0; k < k1; k++) {
-        uint32_t la, lb;
-        lens(k, la, lb);
-        const int ia = hia[k];
-        if (!(la > 0 && lb > 0 && key_pass<K>(M, sA[ia])))
-            continue;
-        const int jb = hpos[k] - ia;
-        const int64_t ga = i0 + ia, gb = j0 + jb;
-        if (r < M.cap_runs) {
-            if (M.chain1) {
-                // 3-input composition: A element ga = first-level run
-                M.s0[r] = M.c_s0[ga];
-                M.s1[r] = M.c_s1[ga];
-                M.len1[r] = M.c_len1[ga];
-                M.s2[r] = (uint32_t)gb;
-                M.len2[r] = lb;
-            } else {
-                M.s0[r] = (uint32_t)ga;
-                M.s1[r] = (uint32_t)gb;
-                M.len1[r] = lb;
-                if (M.len0) M.len0[r] = la;
-                if (M.key_out) ((K *)M.key_out)[r] = sA[ia];
-                if (M.w_out) M.w_out[r] = (uint64_t)la * lb;
+    for (int kb = k0; kb < k1; kb += HB) {
+        uint32_t la[HB], lb[HB], x0[HB], x1[HB], x2[HB];
+        uint64_t w[HB];
+        int ia[HB], jb[HB];
+        bool ok[HB];
+#pragma unroll
+        for (int u = 0; u < HB; u++) {
+            const int k = kb + u;
+            ok[u] = false;
+            la[u] = lb[u] = x0[u] = x1[u] = x2[u] = 0;
+            w[u] = 0;
+            ia[u] = jb[u] = 0;
+            if (k < k1) {
+                lens(k, la[u], lb[u]);
+                ia[u] = hia[k];
+                jb[u] = hpos[k] - ia[u];
+                ok[u] = la[u] > 0 && lb[u] > 0 && key_pass<K>(M, sA[ia[u]]);
+                if (ok[u]) {
+                    const int64_t ga = i0 + ia[u];
+                    w[u] = M.wA ? __ldg(M.wA + ga) : (uint64_t)la[u];
+                    if (M.chain1) {
+                        // 3-input composition: A element ga = first-level run
+                        x0[u] = __ldg(M.c_s0 + ga);
+                        x1[u] = __ldg(M.c_s1 + ga);
+                        x2[u] = __ldg(M.c_len1 + ga);
+                    }
+                }
             }
-            M.off[r] = off;
         }
-        r++;
-        off += (M.wA ? M.wA[ga] : (uint64_t)la) * lb;
+#pragma unroll
+        for (int u = 0; u < HB; u++) {
+            if (!ok[u])
+                continue;
+            const int64_t ga = i0 + ia[u], gb = j0 + jb[u];
+            if (r < M.cap_runs) {
+                if (M.chain1) {
+                    M.s0[r] = x0[u];
+                    M.s1[r] = x1[u];
+                    M.len1[r] = x2[u];
+                    M.s2[r] = (uint32_t)gb;
+                    M.len2[r] = lb[u];
+                } else {
+                    M.s0[r] = (uint32_t)ga;
+                    M.s1[r] = (uint32_t)gb;
+                    M.len1[r] = lb[u];
+                    if (M.len0) M.len0[r] = la[u];
+                    if (M.key_out) ((K *)M.key_out)[r] = sA[ia[u]];
+                    if (M.w_out) M.w_out[r] = (uint64_t)la[u] * lb[u];
+                }
+                M.off[r] = off;
+            }
+            r++;
+            off += w[u] * lb[u];
+        }
     }
     cta_exit_reset(M.ctrs);
 }
@@ -661,29 +707,51 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
             const uint32_t *rs0 = rec_u32(s, 0), *rs1 = rec_u32(s, 1), *rl1 = rec_u32(s, 2);
             const uint32_t *rs2 = rec_u32(s, 3), *rl2 = rec_u32(s, 4);
             const int sh = ctl->rsh[s], nrec = ctl->nrec[s];
-            // (1) candidate -> run map: run starts scattered into a cleared array, then a
-            //     block max-scan (run indices increase with the candidate)
-#pragma unroll
-            for (int k = 0; k < ITEMS; k += 4)
-                *(uint2 *)&runidx[tid * ITEMS + k] = make_uint2(0u, 0u);
-            bar_sync(kJBar, NT);
-            for (int rr = 1 + tid; rr < nrec; rr += NT) {
-                const uint64_t o = roff[sh + rr] - c0g;
-                if (o < (uint64_t)rows) runidx[o] = (uint16_t)rr;
-            }
-            bar_sync(kJBar, NT);
+            // (1) candidate -> run.  Few runs in the tile (long runs, e.g. Zipf hot keys):
+            //     each thread binary-searches its first candidate over the staged run
+            //     offsets (strictly increasing: every recorded run has >= 1 candidate) and
+            //     walks forward, no block-wide step.  Many runs (short runs): run starts
+            //     scattered into a cleared array, then a block max-scan.  (nrec is
+            //     CTA-uniform, so is the branch.)
             uint16_t v[ITEMS];
+            if (nrec <= T / 16) {
+                const uint64_t cf = c0g + (uint64_t)(tid * ITEMS);
+                int lo = 0, hi = nrec;                  // roff[sh + 0] <= c0g <= cf
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (roff[sh + mid] <= cf) lo = mid;
+                    else hi = mid;
+                }
+                int r = lo;
+                uint64_t nxt = r + 1 < nrec ? roff[sh + r + 1] : ~0ull;
 #pragma unroll
-            for (int k = 0; k < ITEMS; k += 4) {
-                const uint2 x = *(const uint2 *)&runidx[tid * ITEMS + k];
-                v[k] = (uint16_t)x.x;
-                v[k + 1] = (uint16_t)(x.x >> 16);
-                v[k + 2] = (uint16_t)x.y;
-                v[k + 3] = (uint16_t)(x.y >> 16);
-            }
+                for (int k = 0; k < ITEMS; k++) {
+                    while (cf + k >= nxt) {
+                        ++r;
+                        nxt = r + 1 < nrec ? roff[sh + r + 1] : ~0ull;
+                    }
+                    v[k] = (uint16_t)r;
+                }
+            } else {
 #pragma unroll
-            for (int k = 1; k < ITEMS; k++) v[k] = max(v[k], v[k - 1]);
-            {
+                for (int k = 0; k < ITEMS; k += 4)
+                    *(uint2 *)&runidx[tid * ITEMS + k] = make_uint2(0u, 0u);
+                bar_sync(kJBar, NT);
+                for (int rr = 1 + tid; rr < nrec; rr += NT) {
+                    const uint64_t o = roff[sh + rr] - c0g;
+                    if (o < (uint64_t)rows) runidx[o] = (uint16_t)rr;
+                }
+                bar_sync(kJBar, NT);
+#pragma unroll
+                for (int k = 0; k < ITEMS; k += 4) {
+                    const uint2 x = *(const uint2 *)&runidx[tid * ITEMS + k];
+                    v[k] = (uint16_t)x.x;
+                    v[k + 1] = (uint16_t)(x.x >> 16);
+                    v[k + 2] = (uint16_t)x.y;
+                    v[k + 3] = (uint16_t)(x.y >> 16);
+                }
+#pragma unroll
+                for (int k = 1; k < ITEMS; k++) v[k] = max(v[k], v[k - 1]);
                 uint32_t mx = v[ITEMS - 1];
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
