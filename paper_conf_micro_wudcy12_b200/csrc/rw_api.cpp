@@ -1026,8 +1026,11 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                 if (Rb < W) continue;
                 const size_t smem = base + S * RS + Rb;
                 if (join_emit_occupancy(ntj, items, ways, smem, L.agg) < occ_t) continue;
+                // measured (C3, C5): more compute warps first (512 x 4 beats 256 x 8 and,
+                // for the 3-input group, 256 x 4 with the larger ring), then the tile, then
+                // the ring's worst-case blocks
                 const double q = (double)Rb / (double)W;
-                const double sc = (q >= 2.0 ? 1e9 : q * 1e8) + T * 1e3 + ntj + S;
+                const double sc = ntj * 1e6 + T * 1e2 + std::min(q, 4.0) * 10 + S;
                 if (sc > best) {
                     best = sc;
                     L.items = items;
@@ -1073,10 +1076,14 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         else if (p->o.reserved[4] == 4) vars.push_back({256, 8});
         else if (p->o.reserved[4] == 5) vars.push_back({256, 16});
         else if (p->o.reserved[4] == 6) vars.push_back({384, 8});
+        else if (p->o.reserved[4] == 9) vars.push_back({384, 16});
+        else if (p->o.reserved[4] == 11) vars.push_back({512, 12});
         else if (p->o.reserved[4] == 7 && nbr == 1) vars.push_back({128, 16, 2});
         else if (p->o.reserved[4] == 8 && nbr == 1) vars.push_back({256, 8, 2});
         else if (nbr > 1) vars = {{256, 8}, {256, 4}};
-        else vars = {{256, 16}, {256, 8}, {256, 4}};
+        // 384 x 16: 12 compute warps on 6144-row tiles (measured C2 2.29 -> 2.06 ms: the
+        // per-tile chain is latency-bound, so more warps and a larger tile both pay)
+        else vars = {{384, 16}, {256, 16}, {256, 8}, {256, 4}};
         const int want_stages_e = p->o.stages > 0 ? std::min(std::max(p->o.stages, 2), 8) : 0;
         bool direct_e = nbr == 1;
         for (const HOp &h : ops)

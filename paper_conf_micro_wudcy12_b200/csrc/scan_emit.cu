@@ -25,7 +25,7 @@
 namespace rw {
 
 constexpr int kEmitMaxStages = 8;
-constexpr int kEmitMaxCnt = 32;           // G * NW counters per branch (G <= 4 groups of 4 rows, NW warps)
+constexpr int kEmitMaxCnt = 64;           // G * NW counters per branch (G <= 4 groups of 4 rows, NW warps)
 constexpr uint32_t kComputeBarEmit = 1;   // named barrier of the compute warps
 constexpr int kWriters = 4;               // look-back + copy-out warps
 constexpr int kEmitAux = 32 * (1 + kWriters);
@@ -429,8 +429,10 @@ __global__ void __launch_bounds__(NT * TEAMS + kEmitAux, 1) k_scan_emit(const __
                         ctl->cnt[par][b][g * NW + lwarp] = (inc >> (8 * g)) & 255u;
                 const uint32_t ex = inc - pk;
                 bar_sync(kComputeBarEmit + team, NT);
-                // block prefix of (group, warp) in tile order and the tile total
-                const uint32_t v = lane < G * NW ? ctl->cnt[par][b][lane] : 0u;
+                // block prefix of (group, warp) in tile order and the tile total (G * NW
+                // counters: one per lane, or two when there are more than 32)
+                constexpr int GN = G * NW;
+                const uint32_t v = lane < GN ? ctl->cnt[par][b][lane] : 0u;
                 uint32_t bin = v;
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
@@ -438,11 +440,34 @@ __global__ void __launch_bounds__(NT * TEAMS + kEmitAux, 1) k_scan_emit(const __
                     if (lane >= o)
                         bin += y;
                 }
-                const uint32_t total = __shfl_sync(0xffffffffu, bin, 31);
+                uint32_t total = __shfl_sync(0xffffffffu, bin, 31);
+                uint32_t v2 = 0, bin2 = 0;
+                const uint32_t total0 = total;
+                if constexpr (GN > 32) {
+                    v2 = lane + 32 < GN ? ctl->cnt[par][b][lane + 32] : 0u;
+                    bin2 = v2;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(0xffffffffu, bin2, o);
+                        if (lane >= o)
+                            bin2 += y;
+                    }
+                    total = total0 + __shfl_sync(0xffffffffu, bin2, 31);
+                }
                 uint32_t pre[G];
 #pragma unroll
-                for (int g = 0; g < G; g++)
-                    pre[g] = __shfl_sync(0xffffffffu, bin - v, g * NW + lwarp) + ((ex >> (8 * g)) & 255u);
+                for (int g = 0; g < G; g++) {
+                    const int idx = g * NW + lwarp;
+                    uint32_t e;
+                    if constexpr (GN > 32) {
+                        const uint32_t e0 = __shfl_sync(0xffffffffu, bin - v, idx & 31);
+                        const uint32_t e1 = __shfl_sync(0xffffffffu, bin2 - v2, idx & 31) + total0;
+                        e = idx < 32 ? e0 : e1;
+                    } else {
+                        e = __shfl_sync(0xffffffffu, bin - v, idx);
+                    }
+                    pre[g] = e + ((ex >> (8 * g)) & 255u);
+                }
                 if (lwarp == 0 && lane == 0 && t > 0 && !(L.dbg & 1))
                     // publish the tile aggregate before anything can block this CTA
                     st_relaxed_u64(&L.status[b * L.status_stride + t], ((uint64_t)L.epoch << 48) | (1ull << 46) | total);
@@ -562,9 +587,9 @@ int scan_emit_occupancy(int nt, int items, bool multi, size_t smem, int teams)
     if (multi)
         return items == 4 ? emit_occ<256, 4, true>(smem) : emit_occ<256, 8, true>(smem);
     if (nt == 512)
-        return emit_occ<512, 8, false>(smem);
+        return items == 12 ? emit_occ<512, 12, false>(smem) : emit_occ<512, 8, false>(smem);
     if (nt == 384)
-        return emit_occ<384, 8, false>(smem);
+        return items == 16 ? emit_occ<384, 16, false>(smem) : emit_occ<384, 8, false>(smem);
     return items == 4 ? emit_occ<256, 4, false>(smem) : items == 16 ? emit_occ<256, 16, false>(smem)
                                                       : emit_occ<256, 8, false>(smem);
 }
@@ -585,9 +610,9 @@ cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, in
     if (P.nbranch > 1)
         return items == 4 ? emit_go<256, 4, true>(P, L, smem, grid, s) : emit_go<256, 8, true>(P, L, smem, grid, s);
     if (nt == 512)
-        return emit_go<512, 8, false>(P, L, smem, grid, s);
+        return items == 12 ? emit_go<512, 12, false>(P, L, smem, grid, s) : emit_go<512, 8, false>(P, L, smem, grid, s);
     if (nt == 384)
-        return emit_go<384, 8, false>(P, L, smem, grid, s);
+        return items == 16 ? emit_go<384, 16, false>(P, L, smem, grid, s) : emit_go<384, 8, false>(P, L, smem, grid, s);
     return items == 4 ? emit_go<256, 4, false>(P, L, smem, grid, s)
                       : items == 16 ? emit_go<256, 16, false>(P, L, smem, grid, s) : emit_go<256, 8, false>(P, L, smem, grid, s);
 }

@@ -40,6 +40,19 @@ def test_selectivity_sweep(s):
     assert_same(got, run_oracle(spec, ins))
 
 
+@pytest.mark.parametrize("variant", [5, 6, 9])
+@pytest.mark.parametrize("n", [1, 6143, 6144, 6145, 300_001])
+def test_c2_emit_variants(variant, n):
+    """Emitting kernel geometries: 256 x 16, 384 x 8, 384 x 16 (the default for C2;
+    48 (group, warp) counters, so the block prefix takes two per lane)."""
+    spec = workloads.c2_spec()
+    ins = workloads.c2_inputs(n, device=DEV, cfg=0x8D)
+    got, plan = run_gpu(spec, ins, variant=variant)
+    assert_same(got, run_oracle(spec, ins))
+    if n > 0:
+        assert {5: "k_scan_emit<256,16>", 6: "k_scan_emit<384,8>", 9: "k_scan_emit<384,16>"}[variant] in plan.explain(plan.out_id)
+
+
 @pytest.mark.parametrize("variant", [7, 8])          # two-team emitting kernels: 2 x 128 x 16, 2 x 256 x 8
 @pytest.mark.parametrize("n", SIZES + [300_001])
 def test_c2_two_team_kernel(variant, n):
