@@ -1077,7 +1077,6 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         else if (p->o.reserved[4] == 5) vars.push_back({256, 16});
         else if (p->o.reserved[4] == 6) vars.push_back({384, 8});
         else if (p->o.reserved[4] == 9) vars.push_back({384, 16});
-        else if (p->o.reserved[4] == 11) vars.push_back({512, 12});
         else if (p->o.reserved[4] == 7 && nbr == 1) vars.push_back({128, 16, 2});
         else if (p->o.reserved[4] == 8 && nbr == 1) vars.push_back({256, 8, 2});
         else if (nbr > 1) vars = {{256, 8}, {256, 4}};

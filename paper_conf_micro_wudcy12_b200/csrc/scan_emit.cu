@@ -587,7 +587,7 @@ int scan_emit_occupancy(int nt, int items, bool multi, size_t smem, int teams)
     if (multi)
         return items == 4 ? emit_occ<256, 4, true>(smem) : emit_occ<256, 8, true>(smem);
     if (nt == 512)
-        return items == 12 ? emit_occ<512, 12, false>(smem) : emit_occ<512, 8, false>(smem);
+        return emit_occ<512, 8, false>(smem);
     if (nt == 384)
         return items == 16 ? emit_occ<384, 16, false>(smem) : emit_occ<384, 8, false>(smem);
     return items == 4 ? emit_occ<256, 4, false>(smem) : items == 16 ? emit_occ<256, 16, false>(smem)
@@ -610,7 +610,7 @@ cudaError_t scan_emit_launch(const ChainProg &P, const TileLaunch &L, int nt, in
     if (P.nbranch > 1)
         return items == 4 ? emit_go<256, 4, true>(P, L, smem, grid, s) : emit_go<256, 8, true>(P, L, smem, grid, s);
     if (nt == 512)
-        return items == 12 ? emit_go<512, 12, false>(P, L, smem, grid, s) : emit_go<512, 8, false>(P, L, smem, grid, s);
+        return emit_go<512, 8, false>(P, L, smem, grid, s);
     if (nt == 384)
         return items == 16 ? emit_go<384, 16, false>(P, L, smem, grid, s) : emit_go<384, 8, false>(P, L, smem, grid, s);
     return items == 4 ? emit_go<256, 4, false>(P, L, smem, grid, s)
