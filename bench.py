@@ -449,7 +449,8 @@ def main():
                 mine = rdist.exchange_all(backend, ins, schema, world)
                 loc_in = [(int(mine[k][0].numel()), mine[k]) for k in spec["inputs"]]
                 plan.execute(loc_in, node, outs, cap, n_dev=n_dev)
-                return plan.last_launches() + 3 * (2 + (world - 1).bit_length())
+                # per relation: k_split_bounds, k_mp_pack, k_mp_samples/rank/cuts/merge
+                return plan.last_launches() + 6 * len(spec["inputs"])
             return step
 
         def step():

@@ -12,8 +12,10 @@ pytestmark = pytest.mark.gpu
 DEV = "cuda:0"
 
 
-def simulated_exchange(backend, shards, types, splitters):
-    """What exchange() does with all_to_all_single, done in-process for P virtual ranks."""
+def simulated_exchange(backend, shards, types, splitters, packed=False):
+    """What exchange_all() does with all_to_all_single, done in-process for P virtual
+    ranks: per-column pieces + rw_merge_runs, or (packed) one u64 image per tuple
+    (rw_pack_tuples) + rw_merge_packed_runs, as the product path sends them."""
     import torch
     P = len(shards)
     pieces = [[None] * P for _ in range(P)]          # pieces[src][dst] = list of column slices
@@ -29,12 +31,17 @@ def simulated_exchange(backend, shards, types, splitters):
         run_off = [0]
         for src in range(P):
             run_off.append(run_off[-1] + int(pieces[src][dst][0].numel()))
-        out.append(backend.merge(recv, types, run_off))
+        if packed:
+            buf = torch.cat([backend.pack(pieces[src][dst], types) for src in range(P)])
+            out.append(backend.merge_packed(buf, types, run_off))
+        else:
+            out.append(backend.merge(recv, types, run_off))
     return out
 
 
+@pytest.mark.parametrize("packed", [False, True])
 @pytest.mark.parametrize("P", [2, 3, 8])
-def test_key_range_sharded_three_way_join_equals_single_gpu(P):
+def test_key_range_sharded_three_way_join_equals_single_gpu(P, packed):
     import torch
     from paper_conf_micro_wudcy12_b200 import dist as rd
     n = 20_000
@@ -53,7 +60,7 @@ def test_key_range_sharded_three_way_join_equals_single_gpu(P):
     allk = torch.cat([rd.key_values(k, t) for k, t in keys])
     allk, _ = torch.sort(allk)
     spl = [int(allk[(allk.numel() * (r + 1)) // P].item()) for r in range(P - 1)]
-    ex = {k: simulated_exchange(backend, shards[k], ["u32", "u32"], spl) for k in "RST"}
+    ex = {k: simulated_exchange(backend, shards[k], ["u32", "u32"], spl, packed) for k in "RST"}
     # each virtual rank's range, merged, equals the slice of the globally sorted relation
     for k in "RST":
         cat = [torch.cat([ex[k][r][c] for r in range(P)]) for c in range(2)]

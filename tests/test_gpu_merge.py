@@ -103,6 +103,17 @@ def test_merge_large_p8():
         np.testing.assert_array_equal(g, e)
 
 
+@pytest.mark.parametrize("types", [["u32", "u32"], ["i64"], ["i32", "u8"]])
+def test_packed_single_run_roundtrip(types):
+    """One received run (P = 1, or the other ranks sent nothing): pack, then unpack
+    through the merge kernels, is the identity."""
+    rng = np.random.default_rng(11)
+    runs = make_runs(rng, types, [70_001], 1 << 20)
+    got = run_merge(runs, types, True)
+    for g, e in zip(got, runs[0]):
+        np.testing.assert_array_equal(g, e)
+
+
 @pytest.mark.parametrize("types", [["i64", "i32"], ["u32", "u32"]])
 def test_merge_tree_fallback(types):
     """Tuples over 8 bytes, or more than 32 runs, take the pairwise merge tree."""
