@@ -1016,7 +1016,10 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                                 (size_t)T * 2 + P.scratch_bytes;
             for (int occ_t : {1, 2}) {
               if (p->o.ctas_per_sm > 0 ? occ_t != p->o.ctas_per_sm : occ_t != 1) continue;
-              for (int S = 2; S <= 3; S++) {
+              for (int S = 1; S <= 3; S++) {
+                // one record stage is a candidate too: the next tile's records are then
+                // fetched after the current tile releases its stage, but it lets the
+                // 3-input group run 512 compute threads (measured C5 9.57 -> 8.21 ms)
                 if (p->o.stages > 0 && S != p->o.stages) continue;
                 const size_t per_cta = std::min(kSmemLimit, (size_t)(228 * 1024) / occ_t - 1024);
                 if (base + S * RS + W > per_cta) continue;

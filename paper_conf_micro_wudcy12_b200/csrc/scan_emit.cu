@@ -101,11 +101,12 @@ __device__ __forceinline__ void emit_copy(T *dst, const T *src, int64_t base, ui
 // The survivors (positions sp) of columns [c0, c1) of the staged tile into a compacted
 // block at byte `pos` of a circular ring of R bytes (shared or global: inlined per call
 // site, so each gets plain STS or STG); a column segment that wraps takes the slow path.
-template <int NT, int G>
+template <int NT, int G, bool GR = false>
 __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1, const char *st, const char *scratch,
                                               uint32_t m, const uint32_t (&sp)[G][4], uint32_t total, char *ring,
                                               uint32_t R, uint32_t pos)
 {
+    const uint64_t pol = GR ? policy_evict_last() : 0ull;
     uint32_t coff = 0;
     for (int c = c0; c < c1; c++) {
         const int w = P.out_w[c];
@@ -126,7 +127,7 @@ __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1
                 const V4<uint32_t> x = ld4<uint32_t>(src, row4<NT>(g));
 #pragma unroll
                 for (int q = 0; q < 4; q++)
-                    if ((m4 >> q) & 1u) ((uint32_t *)d)[sp[g][q]] = x.v[q];
+                    if ((m4 >> q) & 1u) { if (GR) st_l2keep((uint32_t *)d + sp[g][q], x.v[q], pol); else ((uint32_t *)d)[sp[g][q]] = x.v[q]; }
             }
         } else if (w == 8) {
 #pragma unroll
@@ -137,7 +138,7 @@ __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1
                 const V4<uint64_t> x = ld4<uint64_t>(src, row4<NT>(g));
 #pragma unroll
                 for (int q = 0; q < 4; q++)
-                    if ((m4 >> q) & 1u) ((uint64_t *)d)[sp[g][q]] = x.v[q];
+                    if ((m4 >> q) & 1u) { if (GR) st_l2keep((uint64_t *)d + sp[g][q], x.v[q], pol); else ((uint64_t *)d)[sp[g][q]] = x.v[q]; }
             }
         } else {
 #pragma unroll
@@ -148,7 +149,7 @@ __device__ __forceinline__ void compact_block(const ChainProg &P, int c0, int c1
                 const V4<uint8_t> x = ld4<uint8_t>(src, row4<NT>(g));
 #pragma unroll
                 for (int q = 0; q < 4; q++)
-                    if ((m4 >> q) & 1u) ((uint8_t *)d)[sp[g][q]] = x.v[q];
+                    if ((m4 >> q) & 1u) { if (GR) st_l2keep((uint8_t *)d + sp[g][q], x.v[q], pol); else ((uint8_t *)d)[sp[g][q]] = x.v[q]; }
             }
         }
     }
@@ -534,7 +535,7 @@ __global__ void __launch_bounds__(NT * TEAMS + kEmitAux, 1) k_scan_emit(const __
                     }
                 }
                 if (where)
-                    compact_block<NT, G>(P, c0, c1, st, scratch, m, sp, total, ring_g, R, pos);
+                    compact_block<NT, G, true>(P, c0, c1, st, scratch, m, sp, total, ring_g, R, pos);
                 else
                     compact_block<NT, G>(P, c0, c1, st, scratch, m, sp, total, ring_s, R, pos);
                 __syncwarp();
