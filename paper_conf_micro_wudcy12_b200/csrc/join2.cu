@@ -144,7 +144,46 @@ __device__ __forceinline__ K *stage_keys(const KeySrc &S, int64_t i0, int64_t n_
         }
         return raw + (i0 - i0a);
     } else {
-        for (int r = tid; r < n_load; r += kMatchThreads)
+        if (S.img && ((uintptr_t)S.img & 15) == 0) {
+            // precomputed images (a chained match's first-level run keys): the same
+            // 16-byte vector staging, no sign flip
+            constexpr int V = 16 / sizeof(K);
+            const int64_t i0a = i0 & ~(int64_t)(V - 1);
+            const int nvec = (int)((i0 + n_load - i0a + V - 1) / V);
+            const uint4 *src = (const uint4 *)((const K *)S.img + i0a);
+            for (int v = tid; v < nvec; v += kMatchThreads)
+                ((uint4 *)raw)[v] = src[v];
+            return raw + (i0 - i0a);
+        }
+        if (!S.img && S.ncol == 1 && type_width(S.type[0]) == (int)sizeof(K) && ((uintptr_t)S.col[0] & 15) == 0) {
+            // one raw key column of the image width (the other side of a chained match)
+            constexpr int V = 16 / sizeof(K);
+            const int64_t i0a = i0 & ~(int64_t)(V - 1);
+            const int nvec = (int)((i0 + n_load - i0a + V - 1) / V);
+            const K flip = S.type[0] == T_I32 || S.type[0] == T_I64 ? (K)((K)1 << (8 * sizeof(K) - 1)) : (K)0;
+            const uint4 *src = (const uint4 *)((const K *)S.col[0] + i0a);
+            for (int v = tid; v < nvec; v += kMatchThreads) {
+                uint4 x = src[v];
+                K *e = (K *)&x;
+#pragma unroll
+                for (int q = 0; q < V; q++)
+                    e[q] ^= flip;
+                ((uint4 *)raw)[v] = x;
+            }
+            return raw + (i0 - i0a);
+        }
+        // element-wise images, 4 loads in flight per thread
+        int r = tid;
+        for (; r + 3 * kMatchThreads < n_load; r += 4 * kMatchThreads) {
+            K x[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+                x[u] = key_img<K>(S, i0 + r + u * kMatchThreads);
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+                raw[r + u * kMatchThreads] = x[u];
+        }
+        for (; r < n_load; r += kMatchThreads)
             raw[r] = key_img<K>(S, i0 + r);
         return raw;
     }
