@@ -896,18 +896,30 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                     // plain loads into registers (a run's repeated left row is one broadcast
                     // sector; cp.async would serialise identical addresses), stored into the
                     // tile at the top of the next iteration, so they fly during compaction
+                    // (the column's side and width are warp-uniform: selected once per
+                    // column, so the row loop is a plain gather; rows past the tile's end
+                    // read row 0 of their side, which exists since the tile is not empty)
+#define RW_JGATHER(T_, ROWS_)                                                              \
+    {                                                                                      \
+        const T_ *sp_ = (const T_ *)src;                                                   \
+        _Pragma("unroll") for (int q = 0; q < ITEMS; q++) gv[cc][q] = (uint32_t)__ldg(sp_ + ROWS_[q]); \
+    }
 #pragma unroll
                     for (int cc = 0; cc < kJRegCols; cc++) {
                         if (cc >= ncols) break;
                         const char *src = (const char *)X.src[cc];
                         const int w = X.w[cc], side = X.side[cc];
-#pragma unroll
-                        for (int q = 0; q < ITEMS; q++) {
-                            const int cand = wbase + q * 32 + lane;
-                            const uint32_t row = side == 0 ? rA[q] : side == 1 ? rB[q] : rC[WAYS == 3 ? q : 0];
-                            gv[cc][q] = cand < rows ? (w == 4 ? __ldg((const uint32_t *)src + row) : (uint32_t)__ldg((const uint8_t *)src + row)) : 0u;
+                        if (w == 4) {
+                            if (side == 0) RW_JGATHER(uint32_t, rA)
+                            else if (side == 1) RW_JGATHER(uint32_t, rB)
+                            else if (WAYS == 3) RW_JGATHER(uint32_t, rC)
+                        } else {
+                            if (side == 0) RW_JGATHER(uint8_t, rA)
+                            else if (side == 1) RW_JGATHER(uint8_t, rB)
+                            else if (WAYS == 3) RW_JGATHER(uint8_t, rC)
                         }
                     }
+#undef RW_JGATHER
                     pend_st = st;
                     pend_rows = rows;
                 }
@@ -962,14 +974,14 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                 for (int cc = 0; cc < kJRegCols; cc++) {
                     if (cc >= X.ncols) break;
                     char *dst = pend_st + P.slot[cc].off;
-                    const int w = X.w[cc];
+                    if (X.w[cc] == 4) {
 #pragma unroll
-                    for (int q = 0; q < ITEMS; q++) {
-                        const int cand = wbase + q * 32 + lane;
-                        if (cand < pend_rows) {
-                            if (w == 4) ((uint32_t *)dst)[cand] = gv[cc][q];
-                            else ((uint8_t *)dst)[cand] = (uint8_t)gv[cc][q];
-                        }
+                        for (int q = 0; q < ITEMS; q++)
+                            if (wbase + q * 32 + lane < pend_rows) ((uint32_t *)dst)[wbase + q * 32 + lane] = gv[cc][q];
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < ITEMS; q++)
+                            if (wbase + q * 32 + lane < pend_rows) ((uint8_t *)dst)[wbase + q * 32 + lane] = (uint8_t)gv[cc][q];
                     }
                 }
             } else {
