@@ -896,9 +896,11 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                     // plain loads into registers (a run's repeated left row is one broadcast
                     // sector; cp.async would serialise identical addresses), stored into the
                     // tile at the top of the next iteration, so they fly during compaction
-                    // (the column's side and width are warp-uniform: selected once per
-                    // column, so the row loop is a plain gather; rows past the tile's end
-                    // read row 0 of their side, which exists since the tile is not empty)
+                    // 3-input groups: the column's side and width are warp-uniform, selected
+                    // once per column, so the row loop is a plain gather (rows past the
+                    // tile's end read row 0 of their side, which exists since the tile is
+                    // not empty; measured C5 7.95 -> 7.69 ms).  2-input groups keep the
+                    // per-element form, which measured faster there (C3 5.20 vs 5.37 ms).
 #define RW_JGATHER(T_, ROWS_)                                                              \
     {                                                                                      \
         const T_ *sp_ = (const T_ *)src;                                                   \
@@ -909,14 +911,23 @@ __global__ void __launch_bounds__(NT + kJAux, 1) k_join_emit(const __grid_consta
                         if (cc >= ncols) break;
                         const char *src = (const char *)X.src[cc];
                         const int w = X.w[cc], side = X.side[cc];
-                        if (w == 4) {
-                            if (side == 0) RW_JGATHER(uint32_t, rA)
-                            else if (side == 1) RW_JGATHER(uint32_t, rB)
-                            else if (WAYS == 3) RW_JGATHER(uint32_t, rC)
+                        if constexpr (WAYS == 3) {
+                            if (w == 4) {
+                                if (side == 0) RW_JGATHER(uint32_t, rA)
+                                else if (side == 1) RW_JGATHER(uint32_t, rB)
+                                else RW_JGATHER(uint32_t, rC)
+                            } else {
+                                if (side == 0) RW_JGATHER(uint8_t, rA)
+                                else if (side == 1) RW_JGATHER(uint8_t, rB)
+                                else RW_JGATHER(uint8_t, rC)
+                            }
                         } else {
-                            if (side == 0) RW_JGATHER(uint8_t, rA)
-                            else if (side == 1) RW_JGATHER(uint8_t, rB)
-                            else if (WAYS == 3) RW_JGATHER(uint8_t, rC)
+#pragma unroll
+                            for (int q = 0; q < ITEMS; q++) {
+                                const int cand = wbase + q * 32 + lane;
+                                const uint32_t row = side == 0 ? rA[q] : rB[q];
+                                gv[cc][q] = cand < rows ? (w == 4 ? __ldg((const uint32_t *)src + row) : (uint32_t)__ldg((const uint8_t *)src + row)) : 0u;
+                            }
                         }
                     }
 #undef RW_JGATHER
