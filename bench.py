@@ -287,7 +287,8 @@ def run_reference(args):
     ms = statistics.median(dt for _, dt, _ in vals) * 1e3
     line = {"metric": "input tuples/sec per fused chain", "value": value, "unit": "tuples/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "int64" if cfg == "c4" else ("u32" if cfg in ("c1", "c3", "c5", "cs", "cc") else "i32"),
             "data": "synthetic (rwgen seeded generators)", "impl": "reference",
             "config": {"workload": CONFIGS[cfg]["name"], "sample_rows": vals[0][2],
                        "note": "reference arm = the CPU oracle (single thread) on a bounded prefix sample"},
