@@ -1083,6 +1083,9 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
         else if (p->o.reserved[4] == 7 && nbr == 1) vars.push_back({128, 16, 2});
         else if (p->o.reserved[4] == 8 && nbr == 1) vars.push_back({256, 8, 2});
         else if (nbr > 1) vars = {{256, 8}, {256, 4}};
+        // 384 x 16: 12 compute warps on 6144-row tiles (measured C2 2.29 -> 2.06 ms: the
+        // per-tile chain is latency-bound, so more warps and a larger tile both pay)
+        else vars = {{384, 16}, {256, 16}, {256, 8}, {256, 4}};
         if (nbr > 1) {
             // the branch-loop (MULTI) instances exist for 256 x 8 and 256 x 4 (a 384 x 16
             // one measured slower on pattern (d): 5.24 vs 4.81 ms with the L2-ring kernel)
@@ -1092,9 +1095,6 @@ void lower(rw_plan *p, const Group &g, const std::vector<int> &src_types, Lowere
                     v2.push_back(v);
             vars = v2.empty() ? std::vector<EVar>{{256, 8}, {256, 4}} : v2;
         }
-        // 384 x 16: 12 compute warps on 6144-row tiles (measured C2 2.29 -> 2.06 ms: the
-        // per-tile chain is latency-bound, so more warps and a larger tile both pay)
-        else vars = {{384, 16}, {256, 16}, {256, 8}, {256, 4}};
         const int want_stages_e = p->o.stages > 0 ? std::min(std::max(p->o.stages, 2), 8) : 0;
         bool direct_e = nbr == 1;
         for (const HOp &h : ops)

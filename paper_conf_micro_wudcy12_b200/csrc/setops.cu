@@ -139,6 +139,30 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
     // every partition a CTA waits for has been claimed by a running CTA (no assumption
     // that the whole grid is resident); the count pass walks them statically
     const bool claim = WRITE && S.status != nullptr;
+    // (u32 | i32) x 2 tuples with 16-byte aligned columns take the vector staging
+    const bool two4 = PACKED && S.ncols == 2 && type_width(S.types[0]) == 4 && type_width(S.types[1]) == 4 &&
+                      (((uintptr_t)S.x[0] | (uintptr_t)S.x[1] | (uintptr_t)S.y[0] | (uintptr_t)S.y[1]) & 15) == 0;
+    const uint32_t f0 = S.types[0] == T_I32 ? 0x80000000u : 0u, f1 = S.types[1] == T_I32 ? 0x80000000u : 0u;
+    // rows [start, start + n) of a two-column relation into dst[0, n): the aligned span
+    // is read in 16-byte vectors (a vector never crosses a 16-byte boundary, so bytes
+    // read past a column's end stay inside its allocation), out-of-range lanes skipped
+    auto stage_two4 = [&](const void *const *cols, int64_t start, int n, uint64_t *dst) {
+        const int64_t sa = start & ~(int64_t)3;
+        const int nvec = (int)((start + n - sa + 3) / 4);
+        const uint4 *c0 = (const uint4 *)((const uint32_t *)cols[0] + sa);
+        const uint4 *c1 = (const uint4 *)((const uint32_t *)cols[1] + sa);
+        const int sh = (int)(start - sa);
+        for (int v = tid; v < nvec; v += kThreads) {
+            const uint4 a = c0[v], b = c1[v];
+            const uint32_t av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const int r = 4 * v + q - sh;
+                if (r >= 0 && r < n)
+                    dst[r] = ((uint64_t)(av[q] ^ f0) << 32) | (uint64_t)(bv[q] ^ f1);
+            }
+        }
+    };
     for (int64_t it = 0;; ++it) {
         int64_t p = (int64_t)blockIdx.x + it * gridDim.x;
         if (claim) {
@@ -155,7 +179,12 @@ __global__ void __launch_bounds__(kThreads) k_set_op(const __grid_constant__ Set
         const int nX = (int)(i1 - i0), nY = (int)(j1 - j0), m = (int)(d1 - d0);
         __syncthreads();
         // stage x rows at [0, nX), y rows at [nX, nX + nY), pred at kSetT, succ at kSetT + 1
-        if (PACKED) {
+        if (PACKED && two4) {
+            // two 4-byte columns: 16-byte vector loads of both columns (4 tuples per
+            // thread and load, all in flight), packed key = col0 image << 32 | col1 image
+            stage_two4(S.x, i0, nX, s);
+            stage_two4(S.y, j0, nY, s + nX);
+        } else if (PACKED) {
             for (int r = tid; r < nX; r += kThreads)
                 s[r] = pack_row(S, S.x, i0 + r);
             for (int r = tid; r < nY; r += kThreads)
